@@ -1,0 +1,290 @@
+"""Pins for the oracle planner: max-flow, time bisection, closed-form plan
+times (R11), request routing (R12) and DDAK (Eq. 2).
+
+Max-flow: brute-force minimum s-t cut over all 2^(n-2) cuts (max-flow = min-cut theorem), SciPy's
+maximum_flow and networkx on random graphs with parallel, antiparallel, zero and INF links; closed
+forms (series = min, parallel = sum); flow certificate (capacity, conservation, value).
+Time bisection: single path ceil(D/c), parallel paths ceil(D/sum c), a two-socket closed form, and a
+linear scan over T for tiny demands. DDAK: exhaustive enumeration of tiny instances, the closed-form
+2:1 fill ratio, hierarchy, pool semantics.
+"""
+import itertools
+
+import networkx as nx
+import numpy as np
+import pytest
+from scipy.sparse import csr_matrix
+from scipy.sparse.csgraph import maximum_flow
+
+INF = np.iinfo(np.int64).max
+
+
+def random_links(n, m, rng, inf_prob=0.05, zero_prob=0.05, maxcap=50):
+    links = []
+    for _ in range(m):
+        u, v = rng.integers(0, n, 2)
+        if u == v:
+            continue
+        r = rng.random()
+        cap = INF if r < inf_prob else (0 if r < inf_prob + zero_prob else int(rng.integers(1, maxcap)))
+        links.append((int(u), int(v), cap))
+        if rng.random() < 0.2:  # antiparallel partner
+            links.append((int(v), int(u), int(rng.integers(1, maxcap))))
+        if rng.random() < 0.1:  # parallel partner
+            links.append((int(u), int(v), int(rng.integers(0, maxcap))))
+    return links
+
+
+def brute_min_cut(n, links, s, t):
+    others = [x for x in range(n) if x not in (s, t)]
+    best = None
+    for mask in range(1 << len(others)):
+        S = {s} | {others[i] for i in range(len(others)) if mask >> i & 1}
+        c = 0
+        for u, v, cap in links:
+            if u in S and v not in S:
+                c = INF if cap == INF or c == INF else c + cap
+        best = c if best is None else min(best, c)
+    return best
+
+
+def check_certificate(n, links, s, t, value, flow):
+    bal = [0] * n
+    for (u, v, cap), f in zip(links, flow):
+        assert 0 <= f and (cap == INF or f <= cap)
+        bal[u] -= int(f)
+        bal[v] += int(f)
+    for x in range(n):
+        if x not in (s, t):
+            assert bal[x] == 0
+    assert bal[t] == value and -bal[s] == value
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_maxflow_vs_brute_min_cut(orc, seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(2, 11))
+    links = random_links(n, int(rng.integers(1, 3 * n)), rng)
+    s, t = 0, n - 1
+    cut = brute_min_cut(n, links, s, t)
+    if cut == INF:
+        with pytest.raises(orc.OracleError) as e:
+            orc.maxflow(n, links, s, t)
+        assert e.value.status == orc.EINVAL
+        return
+    val, flow = orc.maxflow(n, links, s, t)
+    assert val == cut
+    check_certificate(n, links, s, t, val, flow)
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_maxflow_vs_scipy_networkx(orc, seed):
+    rng = np.random.default_rng(1000 + seed)
+    n = 40
+    links = random_links(n, 200, rng, inf_prob=0.0, zero_prob=0.1, maxcap=10**6)
+    val, flow = orc.maxflow(n, links, 0, n - 1)
+    check_certificate(n, links, 0, n - 1, val, flow)
+    # scipy wants one entry per (u, v): merge parallel links
+    agg = {}
+    for u, v, c in links:
+        agg[(u, v)] = agg.get((u, v), 0) + c
+    rows = [k[0] for k in agg]
+    cols = [k[1] for k in agg]
+    data = np.array([agg[k] for k in agg], np.int32)
+    M = csr_matrix((data, (rows, cols)), shape=(n, n))
+    assert maximum_flow(M, 0, n - 1).flow_value == val
+    G = nx.DiGraph()
+    G.add_nodes_from(range(n))
+    for (u, v), c in agg.items():
+        G.add_edge(u, v, capacity=c)
+    assert nx.maximum_flow_value(G, 0, n - 1) == val
+
+
+def test_maxflow_closed_forms(orc):
+    # series: min; parallel: sum; INF links are transparent when a finite link bounds the path
+    assert orc.maxflow(4, [(0, 1, 7), (1, 2, 3), (2, 3, 9)], 0, 3)[0] == 3
+    assert orc.maxflow(2, [(0, 1, 7), (0, 1, 3), (0, 1, 0)], 0, 1)[0] == 10
+    assert orc.maxflow(3, [(0, 1, INF), (1, 2, 5)], 0, 2)[0] == 5
+    assert orc.maxflow(3, [(0, 1, 5)], 0, 2)[0] == 0  # t unreachable
+    with pytest.raises(orc.OracleError):
+        orc.maxflow(3, [(0, 1, INF), (1, 2, INF)], 0, 2)  # unbounded
+
+
+def _tb(orc, n, links, supply_idx, s, t):
+    sup = [1 if i in supply_idx else 0 for i in range(len(links))]
+    return orc.time_bisect(n, links, sup, s, t)
+
+
+def test_time_bisect_closed_forms(orc):
+    # single path: s -(D)-> bin -> x -> gpu -> t(INF); T* = ceil(D / c)
+    for D, c in [(1, 1), (100, 7), (10**9, 13), (5, 10)]:
+        links = [(0, 1, D), (1, 2, c), (2, 3, INF)]
+        T, _ = _tb(orc, 4, links, {0}, 0, 3)
+        assert T == -(-D // c)
+    # parallel paths: T* = ceil(D / sum c)
+    links = [(0, 1, 1000), (1, 2, 3), (1, 2, 4), (1, 2, 6), (2, 3, INF)]
+    assert _tb(orc, 4, links, {0}, 0, 3)[0] == -(-1000 // 13)
+    # zero demand
+    assert _tb(orc, 4, [(0, 1, 0), (1, 2, 5), (2, 3, INF)], {0}, 0, 3)[0] == 0
+    # infeasible: demanded bin unreachable
+    with pytest.raises(orc.OracleError) as e:
+        _tb(orc, 4, [(0, 1, 5), (2, 3, INF)], {0}, 0, 3)
+    assert e.value.status == orc.EINFEASIBLE
+
+
+@pytest.mark.parametrize("S0,S1,p,u", [(800, 200, 10, 5), (1000, 1000, 3, 50), (5000, 0, 7, 1), (300, 250, 2, 0)])
+def test_time_bisect_two_socket(orc, S0, S1, p, u):
+    # two host bins (one per socket), 4 GPU ports per socket of capacity p, UPI u each way.
+    # T* = max(ceil((S0+S1)/(8p)), ceil(S0/(4p+u)), ceil(S1/(4p+u)))
+    s, h0, h1, c0, c1, t = 0, 1, 2, 3, 4, 5
+    gpus = list(range(6, 14))
+    links = [(s, h0, S0), (s, h1, S1), (h0, c0, INF), (h1, c1, INF), (c0, c1, u), (c1, c0, u)]
+    for i, g in enumerate(gpus):
+        links.append((c0 if i < 4 else c1, g, p))
+        links.append((g, t, INF))
+    T, flow = _tb(orc, 14, links, {0, 1}, s, t)
+    want = max(-(-(S0 + S1) // (8 * p)), -(-S0 // (4 * p + u)), -(-S1 // (4 * p + u)))
+    assert T == want
+
+
+def test_time_bisect_linear_scan(orc):
+    rng = np.random.default_rng(3)
+    for trial in range(15):
+        n = 7
+        links = [(0, 1, int(rng.integers(1, 40))), (0, 2, int(rng.integers(0, 40)))]
+        for _ in range(10):
+            u = int(rng.integers(1, 5))
+            v = int(rng.integers(3, 6))
+            if u != v:
+                links.append((u, v, int(rng.integers(1, 6))))
+        links += [(5, 6, INF), (3, 6, INF), (4, 6, INF)]
+        D = links[0][2] + links[1][2]
+        try:
+            T, _ = _tb(orc, n, links, {0, 1}, 0, 6)
+        except orc.OracleError as e:
+            assert e.status == orc.EINFEASIBLE
+            continue
+        # brute force: smallest T with maxflow(T) == D
+        for Tb in range(0, T + 1):
+            sc = [(u, v, c if i < 2 else (c if c == INF else c * Tb)) for i, (u, v, c) in enumerate(links)]
+            if orc.maxflow(n, sc, 0, 6)[0] == D:
+                break
+        assert Tb == T
+
+
+def test_plan_closed_forms_hand_worked(orc):
+    # k = 2, HBM bins 0 (GPU0), 1 (GPU1), host bin 2; per GPU per batch d = [100, 60, 40];
+    # x for host bin: 30 bytes enter via GPU0, 10 via GPU1 (W = 40).
+    own = [0, 1, -1]
+    d = [100, 60, 40]
+    x = [[0, 0], [0, 0], [30, 10]]
+    # GPU0: in = 60 (peer HBM1) + ceil(40*10/40)=10 -> 70; out = 100 (HBM0 to GPU1) + ceil(1*40*30/40)=30 -> 130
+    # GPU1: in = 100 + ceil(40*30/40)=30 -> 130; out = 60 + ceil(40*10/40)=10 -> 70
+    # max = 130; nvlink cap 7 -> ceil(130/7) = 19
+    # HBM: GPU0 = 2*100 + 200 = 400, GPU1 = 2*60 + 200 = 320 -> ceil(400/9) = 45
+    tn, th = orc.plan_closed_forms(2, own, d, x, 7, 9)
+    assert (tn, th) == (19, 45)
+    # single GPU, all local: no NVLink bytes
+    tn, th = orc.plan_closed_forms(1, [0], [500], [[0]], 0, 100)
+    assert (tn, th) == (0, 10)
+
+
+def test_bucket_hand_worked_and_properties(orc):
+    # one host bin, k = 2, x = [3, 1] (W = 4), 10 requests of rank g = 0:
+    # slot = floor(r*4/10) = 0,0,0,1,1,2,2,2,3,3 -> via GPU0 while slot < 3 (r = 0..7), GPU1 for r = 8, 9
+    route, qoff, qpos = orc.bucket(0, 2, [-1], [[3, 1]], [0] * 10)
+    assert list(route) == [0] * 8 + [1] * 2
+    assert list(qoff) == [0, 8, 10]
+    rng = np.random.default_rng(0)
+    own = [0, 1, 2, -1, -1]
+    x = [[0, 0, 0], [0, 0, 0], [0, 0, 0], [5, 3, 2], [0, 0, 0]]
+    bins = rng.integers(0, 5, 1000)
+    for g in range(3):
+        route, qoff, qpos = orc.bucket(g, 3, own, x, bins)
+        assert sorted(qpos.tolist()) == list(range(1000))  # every request in exactly one queue
+        for q in range(15):
+            seg = qpos[qoff[q]: qoff[q + 1]]
+            assert (np.diff(seg) > 0).all()  # stable
+            assert (route[seg] == q).all()
+        for i, b in enumerate(bins):
+            if own[b] >= 0:
+                assert route[i] == b * 3 + own[b]
+            if b == 4:  # W = 0: direct
+                assert route[i] == 4 * 3 + g
+        nj = int((bins == 3).sum())
+        for h in range(3):
+            cnt = int((route == 3 * 3 + h).sum())
+            assert abs(cnt - nj * x[3][h] / 10) <= 1
+
+
+def brute_ddak_feasible(hot, caps):
+    nb = len(caps)
+    sols = []
+    for assign in itertools.product(range(nb), repeat=len(hot)):
+        used = [assign.count(b) for b in range(nb)]
+        if all(used[b] <= caps[b] for b in range(nb)):
+            sols.append(assign)
+    return sols
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_ddak_exhaustive_small(orc, seed):
+    rng = np.random.default_rng(seed)
+    nv = int(rng.integers(1, 8))
+    nb = int(rng.integers(1, 4))
+    hot = rng.integers(0, 20, nv)
+    tier = sorted(rng.integers(0, 2, nb).tolist())
+    caps = rng.integers(0, nv + 1, nb)
+    if caps.sum() < nv:
+        caps[-1] += nv - caps.sum()
+    traffic = rng.integers(0, 10, nb)
+    sols = brute_ddak_feasible(hot.tolist(), caps.tolist())
+    assert sols  # instance is feasible
+    for pool in (1, 2, 100):
+        bin_of, slot_of, A, U = orc.ddak(hot, tier, caps, traffic, pool)
+        assert tuple(bin_of.tolist()) in set(sols)  # a feasible assignment
+        for b in range(nb):
+            mine = np.where(bin_of == b)[0]
+            assert U[b] == len(mine) <= caps[b]
+            assert sorted(slot_of[mine].tolist()) == list(range(len(mine)))
+            assert A[b] == hot[mine].sum()
+        if pool == 1:
+            # hierarchy: every vertex placed in the best tier having traffic is at least
+            # as hot as every vertex placed in a worse tier.
+            best = min((tier[b] for b in range(nb) if traffic[b] > 0), default=None)
+            if best is not None:
+                hb = [hot[v] for v in range(nv) if tier[bin_of[v]] == best and traffic[bin_of[v]] > 0]
+                hw = [hot[v] for v in range(nv) if tier[bin_of[v]] > best]
+                if hb and hw:
+                    assert min(hb) >= max(hw)
+
+
+def test_ddak_closed_form_ratio(orc):
+    # uniform hotness, T = (4, 1), equal capacity: priority ~ U^2 / T equalises at U0 = 2 U1.
+    n = 3000
+    _, _, _, U = orc.ddak(np.ones(n, np.uint64), [0, 0], [10**6, 10**6], [4, 1], 1)
+    assert U.sum() == n
+    assert abs(U[0] - 2 * U[1]) <= 2
+    # with pooling the ratio holds to within a pool
+    _, _, _, U = orc.ddak(np.ones(n, np.uint64), [0, 0], [10**6, 10**6], [4, 1], 100)
+    assert abs(U[0] - 2 * U[1]) <= 200
+
+
+def test_ddak_single_bin_and_pool_semantics(orc):
+    hot = np.array([5, 9, 1, 9, 0, 3], np.uint64)
+    bin_of, slot_of, A, U = orc.ddak(hot, [0], [6], [1], 1)
+    # single bin fills in hotness order (desc, id asc): 1, 3, 0, 5, 2, 4
+    order = [1, 3, 0, 5, 2, 4]
+    assert [int(slot_of[v]) for v in order] == list(range(6))
+    # pool >= capacity: the first chosen bin fills completely before the next takes anything
+    bin_of, slot_of, A, U = orc.ddak(hot, [0, 0], [4, 4], [1, 1], 100)
+    assert list(U) == [4, 2]
+    assert set(np.where(bin_of == 0)[0].tolist()) == {1, 3, 0, 5}
+    # infeasible: total capacity below n
+    with pytest.raises(orc.OracleError) as e:
+        orc.ddak(hot, [0], [5], [1], 1)
+    assert e.value.status == orc.EINFEASIBLE
+    # host tier only used once the GPU tier is full
+    bin_of, _, _, U = orc.ddak(hot, [0, 1], [2, 10], [1, 100], 1)
+    assert list(U) == [2, 4]
+    assert set(np.where(bin_of == 0)[0].tolist()) == {1, 3}
