@@ -1,0 +1,288 @@
+/*
+ * moment.h — C ABI of the B200-native Moment hot path (Shi et al., "Moment: Co-optimizing Physical
+ * Communication Topology and Data Placement for Multi-GPU Out-of-core GNN Training", SC '25).
+ *
+ * Citations "P:Lnnn" are lines of the paper text (/root/reference/PAPER.md at build time; the file is
+ * not needed at run time). Readings of ambiguous passages are DESIGN.md §3 items "R#".
+ *
+ * Conventions (all entry points):
+ *  - Every call returns moment_status: MOMENT_OK (0) or a negative error code. A human-readable message
+ *    for the last failing call on the calling thread is returned by moment_last_error().
+ *  - Plain pointers and sizes only. "host" pointers are ordinary CPU memory; "device" pointers are CUDA
+ *    device (or UVA-mapped) memory of the context's device. Streams are passed as void* (cudaStream_t;
+ *    NULL = legacy default stream).
+ *  - Ownership: every array passed in stays owned by the caller. Opaque handles (topo, plan, ctx) are
+ *    owned by the library and released with the matching *_free call. A ctx RETAINS the device pointers
+ *    given to moment_ctx_create (CSR, bins, placement map); the caller keeps them alive until ctx_free.
+ *  - Units: bytes, microseconds (us), bytes/us (= MB/s); all int64. Vertex ids are int64 at the boundary.
+ *  - Device calls enqueue on the stream and return; argument, shape and range errors are detected on the
+ *    host before anything is enqueued (MOMENT_EINVAL / MOMENT_EOVERFLOW). Asynchronous CUDA faults surface
+ *    at the next call as MOMENT_ECUDA. No device call synchronises the host or allocates memory: every
+ *    workspace is sized once in moment_ctx_create, so the calls are CUDA-graph capturable.
+ *  - Determinism: sample outputs are a bitwise function of (CSR, seeds, fanout, rng_seed, flags),
+ *    independent of launch configuration; gathered rows are a bitwise function of (ids, feature rows),
+ *    independent of placement and routing.
+ */
+#ifndef MOMENT_H
+#define MOMENT_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t moment_status;
+enum {
+    MOMENT_OK = 0,
+    MOMENT_EINVAL = -1,       /* bad argument, shape, id or graph */
+    MOMENT_ENOMEM = -2,       /* host or device allocation failed */
+    MOMENT_ECUDA = -3,        /* CUDA runtime error (message holds cudaGetErrorString) */
+    MOMENT_ENCCL = -4,        /* reserved: collective transport error */
+    MOMENT_EINFEASIBLE = -5,  /* demand cannot be met / knapsack capacities too small */
+    MOMENT_EOVERFLOW = -6,    /* a capacity or workspace bound is too small (message holds the need) */
+    MOMENT_EUNSUPPORTED = -7, /* valid request outside what this build implements */
+    MOMENT_ETIMEDOUT = -8     /* cross-GPU wait exceeded its watchdog */
+};
+
+/* "virtual edges have infinite bandwidth" (Figure 9 caption; c(v_c, t) = inf) */
+#define MOMENT_CAP_INF INT64_MAX
+
+const char* moment_last_error(void);
+/* Library version, (major << 16) | minor. */
+int32_t moment_version(void);
+
+/* ================================================================================================
+ * P1 — communication topology graph (§3.2)
+ * G = (V, E), V = V_s (storage) ∪ V_c (computation) ∪ V_i (interconnect) ∪ {s, t};
+ * E = E_p (physical) ∪ E_v (virtual); flow direction source -> storage -> interconnect -> computation
+ * -> sink. Capacity c(u, v) = profiled throughput upper limit, int64 bytes/us.
+ * ================================================================================================ */
+enum { MOMENT_NODE_SOURCE = 0, MOMENT_NODE_SINK = 1, MOMENT_NODE_STORAGE = 2, MOMENT_NODE_INTERCONNECT = 3,
+       MOMENT_NODE_COMPUTE = 4 };
+/* Storage hierarchy GPU > CPU > SSD: tier rank = tier - 1 (smaller is better). */
+enum { MOMENT_TIER_NONE = 0, MOMENT_TIER_GPU_HBM = 1, MOMENT_TIER_HOST_DRAM = 2, MOMENT_TIER_SSD = 3 };
+
+typedef struct {
+    int32_t kind;     /* MOMENT_NODE_* */
+    int32_t tier;     /* MOMENT_TIER_* (STORAGE nodes); NONE otherwise */
+    int32_t device;   /* GPU rank for HBM storage / COMPUTE nodes, NUMA node for host storage, else -1 */
+    int32_t reserved; /* must be 0 */
+} moment_node;
+
+typedef struct {
+    int32_t from, to; /* node indices */
+    int64_t cap;      /* bytes/us, >= 0, or MOMENT_CAP_INF */
+} moment_link;
+
+typedef struct moment_topo_s* moment_topo_t;
+
+/* Validate and build the graph. Allowed links: SOURCE->STORAGE, STORAGE->INTERCONNECT,
+ * STORAGE->COMPUTE, INTERCONNECT->INTERCONNECT, INTERCONNECT->COMPUTE, COMPUTE->SINK. At most one
+ * SOURCE and one SINK; if absent they are appended (source = n_nodes, sink = n_nodes + 1, in that order).
+ * Every STORAGE node without a source link gets s->v_s with c(s, v_s) = sum of its outgoing capacities
+ * ("c(s, v_s) = c(v_s, v_i)", R8), every COMPUTE node without a sink link gets v_c->t = INF
+ * (P:L221). Added links are appended after the caller's links, storage nodes first, in node order.
+ * nodes/links: host arrays, copied. Errors: EINVAL (kind, index, self-loop, negative capacity, direction). */
+moment_status moment_topology(const moment_node* nodes, int32_t n_nodes, const moment_link* links,
+                              int32_t n_links, moment_topo_t* out);
+/* Sizes of the augmented graph and the indices of s and t. Any out pointer may be NULL. */
+moment_status moment_topology_info(moment_topo_t topo, int32_t* n_nodes, int32_t* n_links, int32_t* source,
+                                   int32_t* sink);
+/* Copy the augmented graph into caller arrays of the sizes reported by moment_topology_info. */
+moment_status moment_topology_export(moment_topo_t topo, moment_node* nodes, moment_link* links);
+moment_status moment_topology_free(moment_topo_t topo);
+
+/* ================================================================================================
+ * P3 — rate max-flow (§3.2 LP): maximise F = net flow out of s subject to 0 <= f <= c
+ * and conservation at every node other than s, t (R7, R9 garbles). Dinic's algorithm.
+ * value: F (bytes/us). link_flow: host int64[n_links] (augmented graph) or NULL. Max-flow values are
+ * unique; per-link flows are not (R20) — callers check them by certificate.
+ * Errors: EINVAL if an s-t path of INF links exists (unbounded), EOVERFLOW if F exceeds int64.
+ * ================================================================================================ */
+moment_status moment_maxflow(moment_topo_t topo, int64_t* value, int64_t* link_flow);
+
+/* ================================================================================================
+ * P4 — DDAK placement (§3.3, Eq. 2 at P:L247; readings R13-R17)
+ * Vertices sorted by (hotness desc, id asc); for each pool of `pool` vertices the bin with the least
+ * Eq. 2 priority (A/T)(U/C) among the non-full bins of the best tier that has traffic takes as many as fit.
+ * ================================================================================================ */
+enum { MOMENT_PLACE_DDAK = 0, MOMENT_PLACE_HASH = 1 };
+
+typedef struct {
+    int64_t n_vertices;
+    const uint64_t* hotness;          /* host [n_vertices]: pre-sampling access counts */
+    int32_t n_bins;                   /* storage bins */
+    const int32_t* bin_node;          /* host [n_bins]: topology STORAGE node of each bin, or NULL = the
+                                         topology's STORAGE nodes in node order (topo required) */
+    const int32_t* bin_tier;          /* host [n_bins]: MOMENT_TIER_*, or NULL = from the topology */
+    const int64_t* bin_capacity_rows; /* host [n_bins]: Bin_Capacity in rows (R6) */
+    const int64_t* bin_traffic;       /* host [n_bins]: Bin_traffic, or NULL = f(s, bin) of the rate
+                                         max-flow of topo ("modeled by maximum flow", R7) */
+    int64_t pool;                     /* vertices per decision; <= 0 means 100 */
+    int32_t mode;                     /* MOMENT_PLACE_DDAK, or MOMENT_PLACE_HASH (uniform baseline) */
+} moment_place_args;
+
+typedef struct {
+    int32_t* bin_of;           /* host [n_vertices] */
+    int64_t* slot_of;          /* host [n_vertices]: row slot inside the bin, dense from 0 */
+    uint64_t* bin_access;      /* host [n_bins] or NULL: final Bin_access (sum of hotness) */
+    int64_t* bin_rows_used;    /* host [n_bins] or NULL: final Bin_currentCapacity */
+    int64_t* bin_traffic_used; /* host [n_bins] or NULL: the Bin_traffic the decision used */
+} moment_place_out;
+
+/* topo may be NULL when bin_tier and bin_traffic are given. Errors: EINVAL, EINFEASIBLE (sum of
+ * capacities < n_vertices), ENOMEM. Host-only; multithreaded sort, deterministic result. */
+moment_status moment_place(moment_topo_t topo, const moment_place_args* args, moment_place_out* out);
+/* packed[v] = ((uint64)bin_of[v] << 40) | slot_of[v] — the device placement map layout (D3). */
+moment_status moment_place_pack(int64_t n_vertices, const int32_t* bin_of, const int64_t* slot_of,
+                                uint64_t* packed);
+
+/* ================================================================================================
+ * P5 — time-bisection plan + quotas (ingest model R10-R12)
+ * Ingest graph: the topology with supply links s->HOST bin j of k*d_j bytes (every active GPU reads d_j
+ * bytes of bin j per batch), no supply on HBM bins, physical links carrying cap*T bytes in T us, v_c->t
+ * INF for active GPUs only. T_ingest = min{T : maxflow(T) = sum supplies}. x[j][h] = bytes of host bin
+ * j entering GPU h (path decomposition of the flow at T_ingest). GPU g then forwards x[j][h]/W_j of its
+ * bin-j requests through GPU h over NVLink ("alternative paths"). T_nvlink and T_hbm are the
+ * closed forms of R11; T* = max(T_ingest, T_nvlink, T_hbm).
+ * ================================================================================================ */
+typedef struct moment_plan_s* moment_plan_t;
+
+typedef struct {
+    int32_t k;                       /* active GPUs */
+    const int32_t* gpu_node;         /* host [k]: COMPUTE node of rank r */
+    const int64_t* bin_demand_bytes; /* host [n_nodes of the augmented topo]: d_b for STORAGE nodes
+                                        (bytes one GPU reads from b per batch); other entries ignored */
+    int64_t nvlink_cap;              /* bytes/us per GPU per direction; 0 = no NVLink (no relay) */
+    int64_t hbm_cap;                 /* bytes/us per GPU, read + write */
+} moment_plan_args;
+
+moment_status moment_plan(moment_topo_t topo, const moment_plan_args* args, moment_plan_t* out);
+/* Any out pointer may be NULL. link_flow: [n_links] ingest flow at T_ingest; quota: [n_nodes][k]
+ * row-major x[node][rank] in bytes (non-zero only on HOST storage rows). */
+moment_status moment_plan_info(moment_plan_t plan, int64_t* t_star, int64_t* t_ingest, int64_t* t_nvlink,
+                               int64_t* t_hbm, int64_t* link_flow, int64_t* quota);
+moment_status moment_plan_free(moment_plan_t plan);
+
+/* ================================================================================================
+ * Device context: one per GPU rank; owns all device workspaces (no allocation on the hot path).
+ * ================================================================================================ */
+typedef struct moment_ctx_s* moment_ctx_t;
+
+#define MOMENT_MAX_BINS 64
+
+typedef struct {
+    int32_t rank, world;      /* this rank, number of ranks (world = 1 for a single GPU) */
+    int32_t device;           /* CUDA device ordinal of this rank */
+    int64_t n_vertices;       /* |V| of the CSR graph (< 2^31) */
+    int64_t max_seeds;        /* largest batch passed to moment_sample */
+    int32_t max_hops;         /* largest number of hops */
+    const int32_t* max_fanout;/* host [max_hops]: largest fanout per hop (workspace bounds) */
+    int64_t row_bytes;        /* R: feature row bytes, multiple of 16 */
+    int64_t row_stride;       /* bytes between consecutive slots of a bin (>= R, multiple of 16) */
+    int32_t n_bins;           /* storage bins (<= MOMENT_MAX_BINS); 0 = no gather */
+    const int32_t* bin_owner; /* host [n_bins]: owning rank of an HBM bin, -1 for a host-DRAM bin */
+    void* const* bin_ptr;     /* host [n_bins]: base of each bin as addressable from THIS device: local
+                                 HBM, a peer-mapped HBM pointer (NVLink) or a mapped pinned-host pointer */
+    const uint64_t* placement;/* device [n_vertices]: (bin << 40) | slot (moment_place_pack), or NULL:
+                                 replicated table in bin 0 at slot = vertex id (all features local) */
+    const int64_t* quota;     /* host [n_bins][world] x[j][h] bytes from moment_plan_info, or NULL
+                                 (every host row read directly) */
+} moment_ctx_args;
+
+moment_status moment_ctx_create(const moment_ctx_args* args, moment_ctx_t* out);
+moment_status moment_ctx_free(moment_ctx_t ctx);
+/* Bytes of device workspace the ctx holds. */
+moment_status moment_ctx_workspace_bytes(moment_ctx_t ctx, int64_t* bytes);
+
+/* ================================================================================================
+ * H1-H3 — multi-hop neighbour sampling with dedup/relabel (R3-R6)
+ * F_0 = seeds; for h < H: every v in F_h draws min(deg, fanout[h]) distinct CSR positions (Floyd with
+ * Philox draws keyed on (rng_seed, v, h, i)), grouped by destination, CSR-position order;
+ * F_{h+1} = F_h ++ ascending new ids; src = index of the neighbour in F_{h+1}.
+ * ================================================================================================ */
+typedef struct {
+    const int64_t* indptr;  /* device [n_vertices + 1] */
+    const int32_t* indices; /* device [n_edges] */
+    int64_t n_vertices;
+    int64_t n_edges;
+} moment_csr;
+
+#define MOMENT_SAMPLE_REPLACE 1u  /* sample with replacement (k draws whenever deg > 0) */
+#define MOMENT_SAMPLE_CHECK 2u    /* device-side check of seed range / uniqueness (sets EINVAL flag) */
+
+typedef struct {
+    int32_t n_hops;         /* H <= max_hops */
+    const int32_t* fanout;  /* host [H], 1 <= fanout[h] <= max_fanout[h] and <= 1024 */
+    uint64_t rng_seed;      /* per-batch Philox key (R1) */
+    uint32_t flags;         /* MOMENT_SAMPLE_* */
+} moment_sample_params;
+
+typedef struct {
+    int64_t* nodes;   /* device [cap_nodes]: F_H (F_h is a prefix of it) */
+    int64_t* offsets; /* device [cap_offsets]: per hop h, |F_h|+1 offsets relative to the hop, blocks packed
+                         back to back by actual size */
+    int32_t* src;     /* device [cap_edges]: per hop, E_h local ids, packed back to back */
+    int64_t* counts;  /* device [2H+1]: |F_0| .. |F_H|, E_0 .. E_{H-1} */
+    int64_t cap_nodes, cap_offsets, cap_edges;
+} moment_sample_out;
+
+/* Upper bounds without dedup: |F_{h+1}| <= min(|F_h|(1 + f_h), n_vertices). */
+moment_status moment_sample_bounds(int64_t n_seeds, const int32_t* fanout, int32_t n_hops, int64_t n_vertices,
+                                   int64_t* max_nodes, int64_t* max_offsets, int64_t* max_edges);
+/* seeds: device [n_seeds], distinct ids in [0, n_vertices) (checked only with MOMENT_SAMPLE_CHECK). */
+moment_status moment_sample(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
+                            const moment_sample_params* params, const moment_sample_out* out, void* stream);
+/* Host-side read of the device error flag raised by MOMENT_SAMPLE_CHECK (synchronises the stream). */
+moment_status moment_sample_check(moment_ctx_t ctx, void* stream);
+
+/* ================================================================================================
+ * P2 — hotness by pre-sampling: hot[v] += 1 for every v in ids[0 .. *n).
+ * ================================================================================================ */
+moment_status moment_hotness(moment_ctx_t ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n,
+                             uint64_t* hot, void* stream);
+
+/* ================================================================================================
+ * H4 — placement lookup + bucketing ("retrieves the SSD ID and vertex offset"; R12)
+ * For request i of this rank: (b, slot) = placement[ids[i]]; via = owner for HBM bins; for host bin j,
+ * with n_j requests of bin j and r the rank of i among them (F_H order), slot' = floor(r W_j / n_j),
+ * via = first h with slot' < cumsum_h x[j][h] (direct when W_j = 0). Queue q = b * world + via.
+ * route: device int32 [max_n] (q per request); qoff: device int64 [n_bins*world + 1];
+ * qpos: device int64 [max_n] (requests stably sorted by q). n_dev: device count (or NULL = max_n).
+ * ================================================================================================ */
+moment_status moment_bucket(moment_ctx_t ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n,
+                            int32_t* route, int64_t* qoff, int64_t* qpos, void* stream);
+
+/* ================================================================================================
+ * H5-H7 — topology-aware gather (P:L93 feature extraction; P:L391-393 relay)
+ * out[i * R .. (i+1) * R) = row of ids[i], read from wherever the placement put it: local HBM, a peer's
+ * HBM (NVLink load through bin_ptr) or pinned host DRAM (zero-copy PCIe read), 128-bit vectors.
+ * Rows routed through a relay GPU h != rank are read by h from host DRAM and stored into this rank's out
+ * over NVLink; moment_gather is then collective over the ranks of moment_gather_group.
+ * ids: device [max_n]; n_dev: device count or NULL (= max_n); out: device [max_n * R].
+ * ================================================================================================ */
+moment_status moment_gather(moment_ctx_t ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n,
+                            void* out, void* stream);
+
+/* Collective gather of `world` ranks driven from ONE host thread on ONE stream ("logical ranks": all
+ * ranks' bins and outputs addressable from the stream's device, e.g. k ranks sharing one GPU, or k
+ * GPUs of one process with peer access enabled). Phase 1: bucketing + request publication for every
+ * rank; phase 2: every rank's direct gather and relay service; stream order is the barrier.
+ * ctxs/ids/n_dev/out: host arrays [world] of per-rank handles / device pointers. */
+moment_status moment_gather_group(moment_ctx_t const* ctxs, int32_t world, const int64_t* const* ids,
+                                  const int64_t* const* n_dev, int64_t max_n, void* const* out, void* stream);
+
+/* ================================================================================================
+ * End-to-end step with HOST buffers (the e2e leg of the benchmark): copies seeds host->device, samples,
+ * gathers F_H into d_out, copies the 2H+1 counts device->host (into counts_host), and synchronises.
+ * seeds_host / counts_host should be pinned for asynchronous copies.
+ * ================================================================================================ */
+moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds_host,
+                               int64_t n_seeds, const moment_sample_params* params,
+                               const moment_sample_out* out, void* d_rows, int64_t* counts_host, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MOMENT_H */

@@ -1,0 +1,288 @@
+// ctx.cu — device context (workspace sized once, no allocation on the hot path) and the device entry
+// points of include/moment.h: moment_sample, moment_gather, moment_gather_group, moment_bucket,
+// moment_hotness, moment_step_host.
+#include <algorithm>
+#include <new>
+
+#include "ctx.h"
+
+using namespace moment;
+
+namespace {
+
+struct Carver {
+    int64_t off = 0;
+    template <typename T>
+    int64_t take(int64_t count) {
+        off = (off + 255) & ~int64_t(255);
+        int64_t at = off;
+        off += std::max<int64_t>(count, 1) * (int64_t)sizeof(T);
+        return at;
+    }
+};
+
+moment_status check_ctx(moment_ctx_t ctx, const char* what) {
+    if (!ctx) return fail(MOMENT_EINVAL, "%s: null ctx", what);
+    int dev = -1;
+    MOMENT_TRY(cuda_check(cudaGetDevice(&dev), what));
+    if (dev != ctx->device) return fail(MOMENT_EINVAL, "%s: current device %d is not the ctx device %d", what, dev, ctx->device);
+    return MOMENT_OK;
+}
+
+bool has_remote_relay(const moment_ctx_s* c) {
+    for (int b = 0; b < c->n_bins; b++) {
+        if (c->bin_owner[b] >= 0 || c->quota.empty()) continue;
+        for (int h = 0; h < c->world; h++)
+            if (h != c->rank && c->quota[(size_t)b * c->world + h] > 0) return true;
+    }
+    return false;
+}
+
+}  // namespace
+
+extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_t* out) {
+    if (!a || !out) return fail(MOMENT_EINVAL, "moment_ctx_create: null argument");
+    *out = nullptr;
+    if (a->world < 1 || a->rank < 0 || a->rank >= a->world || a->world > 64)
+        return fail(MOMENT_EINVAL, "moment_ctx_create: rank %d / world %d invalid", a->rank, a->world);
+    if (a->n_vertices <= 0 || a->n_vertices >= (int64_t(1) << 31))
+        return fail(MOMENT_EINVAL, "moment_ctx_create: n_vertices %lld must be in [1, 2^31)", (long long)a->n_vertices);
+    if (a->max_seeds < 0 || a->max_hops < 0 || a->max_hops > 16 || (a->max_hops > 0 && !a->max_fanout))
+        return fail(MOMENT_EINVAL, "moment_ctx_create: bad max_seeds / max_hops / max_fanout");
+    if (a->n_bins < 0 || a->n_bins > MOMENT_MAX_BINS) return fail(MOMENT_EINVAL, "moment_ctx_create: n_bins %d", a->n_bins);
+    if (a->n_bins > 0) {
+        if (a->row_bytes <= 0 || a->row_bytes % 16 || a->row_stride < a->row_bytes || a->row_stride % 16)
+            return fail(MOMENT_EINVAL, "moment_ctx_create: row_bytes %lld / row_stride %lld must be positive multiples of 16",
+                        (long long)a->row_bytes, (long long)a->row_stride);
+        if (!a->bin_ptr || !a->bin_owner) return fail(MOMENT_EINVAL, "moment_ctx_create: bin_ptr / bin_owner null");
+        for (int b = 0; b < a->n_bins; b++) {
+            if (!a->bin_ptr[b] || (reinterpret_cast<uintptr_t>(a->bin_ptr[b]) & 15))
+                return fail(MOMENT_EINVAL, "moment_ctx_create: bin %d pointer null or not 16-byte aligned", b);
+            if (a->bin_owner[b] < -1 || a->bin_owner[b] >= a->world)
+                return fail(MOMENT_EINVAL, "moment_ctx_create: bin %d owner %d", b, a->bin_owner[b]);
+        }
+        if (!a->placement && a->n_bins != 1)
+            return fail(MOMENT_EINVAL, "moment_ctx_create: a NULL placement means one replicated bin");
+        if (a->quota)
+            for (int64_t i = 0; i < (int64_t)a->n_bins * a->world; i++)
+                if (a->quota[i] < 0) return fail(MOMENT_EINVAL, "moment_ctx_create: negative quota");
+    }
+    for (int h = 0; h < a->max_hops; h++)
+        if (a->max_fanout[h] < 1 || a->max_fanout[h] > kMaxFanout)
+            return fail(MOMENT_EINVAL, "moment_ctx_create: max_fanout[%d] = %d outside [1, %d]", h, a->max_fanout[h], kMaxFanout);
+    int cur = -1;
+    MOMENT_TRY(cuda_check(cudaGetDevice(&cur), "moment_ctx_create"));
+    if (cur != a->device) MOMENT_TRY(cuda_check(cudaSetDevice(a->device), "moment_ctx_create: set device"));
+
+    auto* c = new (std::nothrow) moment_ctx_s;
+    if (!c) return fail(MOMENT_ENOMEM, "moment_ctx_create: out of host memory");
+    c->rank = a->rank;
+    c->world = a->world;
+    c->device = a->device;
+    c->n_vertices = a->n_vertices;
+    c->max_seeds = a->max_seeds;
+    c->max_hops = a->max_hops;
+    c->max_fanout.assign(a->max_fanout, a->max_fanout + a->max_hops);
+    c->row_bytes = a->row_bytes;
+    c->row_stride = a->row_stride;
+    c->n_bins = a->n_bins;
+    c->bin_owner.assign(a->bin_owner, a->bin_owner + a->n_bins);
+    c->bin_ptr.assign(a->bin_ptr, a->bin_ptr + a->n_bins);
+    c->placement = a->placement;
+    if (a->quota) c->quota.assign(a->quota, a->quota + (size_t)a->n_bins * a->world);
+    // bounds per hop
+    c->max_F.resize(a->max_hops + 1);
+    c->max_E.resize(a->max_hops);
+    int64_t F = std::min(a->max_seeds, a->n_vertices);
+    c->max_F[0] = F;
+    for (int h = 0; h < a->max_hops; h++) {
+        c->max_E[h] = F * a->max_fanout[h];
+        c->max_edges += c->max_E[h];
+        c->max_offsets += F + 1;
+        F = std::min(F + F * (int64_t)a->max_fanout[h], a->n_vertices);
+        c->max_F[h + 1] = F;
+    }
+    c->max_nodes = std::max<int64_t>(F, a->max_seeds);
+    c->n_words = (a->n_vertices + 31) / 32;
+    c->max_requests = c->max_nodes;
+    // carve the workspace
+    Carver cv;
+    const int64_t o_lidx = cv.take<int32_t>(a->n_vertices);
+    const int64_t n_words_pad = (c->n_words + kBitscanTileWords - 1) / kBitscanTileWords * kBitscanTileWords;
+    const int64_t o_newbits = cv.take<uint32_t>(n_words_pad);
+    const int64_t o_visited = cv.take<uint32_t>(n_words_pad);
+    const int64_t scan_tiles = n_words_pad / kBitscanTileWords;
+    c->sample_tiles_off.resize(a->max_hops);
+    c->bitscan_tiles_off.resize(a->max_hops);
+    int64_t nts = 0;
+    for (int h = 0; h < a->max_hops; h++) {
+        c->sample_tiles_off[h] = nts;
+        nts += std::max<int64_t>(1, (c->max_F[h] + kSampleTile - 1) / kSampleTile);
+        c->bitscan_tiles_off[h] = nts;
+        nts += scan_tiles;
+    }
+    c->n_tile_status = std::max<int64_t>(nts, 1);
+    const int64_t o_tiles = cv.take<uint64_t>(c->n_tile_status);
+    const int64_t o_tickets = cv.take<uint32_t>(2 * std::max(1, a->max_hops));
+    const int64_t o_err = cv.take<uint32_t>(1);
+    const int32_t Q = std::max(1, a->n_bins * a->world);
+    const int64_t bk_tiles = (c->max_requests + kBucketTile - 1) / kBucketTile + 1;
+    int64_t o_bk_tc = 0, o_bk_tot = 0, o_bk_qoff = 0, o_bk_route = 0, o_bk_qpos = 0, o_quota = 0, o_owner = 0;
+    if (a->n_bins > 0) {
+        o_bk_tc = cv.take<int64_t>(bk_tiles * std::max<int64_t>(Q, a->n_bins));
+        o_bk_tot = cv.take<int64_t>(a->n_bins);
+        o_bk_qoff = cv.take<int64_t>(Q + 1);
+        o_bk_route = cv.take<int32_t>(c->max_requests);
+        o_bk_qpos = cv.take<int64_t>(c->max_requests);
+        o_quota = cv.take<int64_t>(Q);
+        o_owner = cv.take<int32_t>(a->n_bins);
+    }
+    const int64_t o_seed = cv.take<int64_t>(a->max_seeds);
+    c->ws_bytes = cv.off;
+    cudaError_t e = cudaMalloc(&c->ws, c->ws_bytes);
+    if (e != cudaSuccess) {
+        delete c;
+        return fail(MOMENT_ENOMEM, "moment_ctx_create: cudaMalloc(%lld bytes): %s", (long long)cv.off, cudaGetErrorString(e));
+    }
+    char* w = static_cast<char*>(c->ws);
+    c->lidx = reinterpret_cast<int32_t*>(w + o_lidx);
+    c->newbits = reinterpret_cast<uint32_t*>(w + o_newbits);
+    c->visited = reinterpret_cast<uint32_t*>(w + o_visited);
+    c->tile_status = reinterpret_cast<uint64_t*>(w + o_tiles);
+    c->tickets = reinterpret_cast<uint32_t*>(w + o_tickets);
+    c->error_flag = reinterpret_cast<uint32_t*>(w + o_err);
+    if (a->n_bins > 0) {
+        c->bk_tile_counts = reinterpret_cast<int64_t*>(w + o_bk_tc);
+        c->bk_bin_total = reinterpret_cast<int64_t*>(w + o_bk_tot);
+        c->bk_qoff = reinterpret_cast<int64_t*>(w + o_bk_qoff);
+        c->bk_route = reinterpret_cast<int32_t*>(w + o_bk_route);
+        c->bk_qpos = reinterpret_cast<int64_t*>(w + o_bk_qpos);
+        c->d_quota = reinterpret_cast<int64_t*>(w + o_quota);
+        c->d_bin_owner = reinterpret_cast<int32_t*>(w + o_owner);
+    }
+    c->d_seed_stage = reinterpret_cast<int64_t*>(w + o_seed);
+    moment_status st = MOMENT_OK;
+    do {
+        if ((st = cuda_check(cudaMemset(c->ws, 0, c->ws_bytes), "moment_ctx_create: memset")) != MOMENT_OK) break;
+        if ((st = cuda_check(cudaMemset(c->lidx, 0xFF, a->n_vertices * sizeof(int32_t)), "moment_ctx_create: memset")) != MOMENT_OK) break;
+        if (a->n_bins > 0) {
+            std::vector<int64_t> q((size_t)Q, 0);
+            if (!c->quota.empty()) std::copy(c->quota.begin(), c->quota.end(), q.begin());
+            if ((st = cuda_check(cudaMemcpy(c->d_quota, q.data(), Q * sizeof(int64_t), cudaMemcpyHostToDevice), "quota")) != MOMENT_OK) break;
+            if ((st = cuda_check(cudaMemcpy(c->d_bin_owner, c->bin_owner.data(), a->n_bins * sizeof(int32_t), cudaMemcpyHostToDevice), "owner")) != MOMENT_OK) break;
+        }
+        st = cuda_check(cudaDeviceSynchronize(), "moment_ctx_create: sync");
+    } while (0);
+    if (cur != a->device) cudaSetDevice(cur);
+    if (st != MOMENT_OK) {
+        cudaFree(c->ws);
+        delete c;
+        return st;
+    }
+    *out = c;
+    return MOMENT_OK;
+}
+
+extern "C" moment_status moment_ctx_free(moment_ctx_t ctx) {
+    if (!ctx) return MOMENT_OK;
+    int cur = -1;
+    cudaGetDevice(&cur);
+    cudaSetDevice(ctx->device);
+    cudaError_t e = cudaFree(ctx->ws);
+    cudaSetDevice(cur);
+    delete ctx;
+    return cuda_check(e, "moment_ctx_free");
+}
+
+extern "C" moment_status moment_ctx_workspace_bytes(moment_ctx_t ctx, int64_t* bytes) {
+    if (!ctx || !bytes) return fail(MOMENT_EINVAL, "moment_ctx_workspace_bytes: null argument");
+    *bytes = ctx->ws_bytes;
+    return MOMENT_OK;
+}
+
+extern "C" moment_status moment_sample(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
+                                       const moment_sample_params* params, const moment_sample_out* out, void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_sample"));
+    return launch_sample(ctx, csr, seeds, n_seeds, params, out, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" moment_status moment_sample_check(moment_ctx_t ctx, void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_sample_check"));
+    uint32_t flag = 0;
+    MOMENT_TRY(cuda_check(cudaMemcpyAsync(&flag, ctx->error_flag, sizeof(flag), cudaMemcpyDeviceToHost,
+                                          static_cast<cudaStream_t>(stream)), "moment_sample_check"));
+    MOMENT_TRY(cuda_check(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)), "moment_sample_check"));
+    MOMENT_TRY(cuda_check(cudaMemsetAsync(ctx->error_flag, 0, sizeof(uint32_t), static_cast<cudaStream_t>(stream)), "moment_sample_check"));
+    if (flag & 1u) return fail(MOMENT_EINVAL, "moment_sample: a seed was out of range");
+    if (flag & 2u) return fail(MOMENT_EINVAL, "moment_sample: a seed was repeated");
+    return MOMENT_OK;
+}
+
+extern "C" moment_status moment_hotness(moment_ctx_t ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n,
+                                        uint64_t* hot, void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_hotness"));
+    if (max_n < 0 || (max_n > 0 && (!ids || !hot))) return fail(MOMENT_EINVAL, "moment_hotness: null argument");
+    return launch_hotness(ids, n_dev, max_n, hot, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" moment_status moment_bucket(moment_ctx_t ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n,
+                                       int32_t* route, int64_t* qoff, int64_t* qpos, void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_bucket"));
+    if (max_n < 0 || (max_n > 0 && (!ids || !route || !qoff || !qpos))) return fail(MOMENT_EINVAL, "moment_bucket: null argument");
+    if (ctx->n_bins <= 0) return fail(MOMENT_EINVAL, "moment_bucket: ctx has no bins");
+    return launch_bucket(ctx, ids, n_dev, max_n, route, qoff, qpos, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" moment_status moment_gather(moment_ctx_t ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n, void* out,
+                                       void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_gather"));
+    if (ctx->world > 1 && has_remote_relay(ctx))
+        return fail(MOMENT_EUNSUPPORTED, "moment_gather: the quota relays host rows through other ranks; use moment_gather_group");
+    return launch_gather(ctx, ids, n_dev, max_n, out, nullptr, ctx->rank, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" moment_status moment_gather_group(moment_ctx_t const* ctxs, int32_t world, const int64_t* const* ids,
+                                             const int64_t* const* n_dev, int64_t max_n, void* const* out, void* stream) {
+    if (!ctxs || !ids || !out || world < 1) return fail(MOMENT_EINVAL, "moment_gather_group: null argument");
+    for (int r = 0; r < world; r++) {
+        MOMENT_TRY(check_ctx(ctxs[r], "moment_gather_group"));
+        if (ctxs[r]->world != world || ctxs[r]->rank != r)
+            return fail(MOMENT_EINVAL, "moment_gather_group: ctxs[%d] has rank %d / world %d", r, ctxs[r]->rank, ctxs[r]->world);
+        if (ctxs[r]->row_bytes != ctxs[0]->row_bytes || !ctxs[r]->placement)
+            return fail(MOMENT_EINVAL, "moment_gather_group: ctxs disagree on row_bytes or lack a placement map");
+        if (max_n > ctxs[r]->max_requests)
+            return fail(MOMENT_EOVERFLOW, "moment_gather_group: max_n %lld > workspace %lld", (long long)max_n, (long long)ctxs[r]->max_requests);
+    }
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const int64_t* nd;
+    // phase 1: every rank buckets its requests (publishes its relay queues)
+    for (int r = 0; r < world; r++) {
+        nd = n_dev ? n_dev[r] : nullptr;
+        MOMENT_TRY(launch_bucket(ctxs[r], ids[r], nd, max_n, ctxs[r]->bk_route, ctxs[r]->bk_qoff, ctxs[r]->bk_qpos, s));
+    }
+    // phase 2: direct reads (local / peer / host) by each requester, relays served by each relay rank
+    for (int r = 0; r < world; r++) {
+        nd = n_dev ? n_dev[r] : nullptr;
+        MOMENT_TRY(launch_gather(ctxs[r], ids[r], nd, max_n, out[r], ctxs[r]->bk_route, r, s));
+        for (int g = 0; g < world; g++) {
+            if (g == r) continue;
+            MOMENT_TRY(launch_relay(ctxs[r], ctxs[g], ids[g], ctxs[g]->bk_route, ctxs[g]->bk_qoff, ctxs[g]->bk_qpos, out[g], s));
+        }
+    }
+    return MOMENT_OK;
+}
+
+extern "C" moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds_host, int64_t n_seeds,
+                                          const moment_sample_params* params, const moment_sample_out* out, void* d_rows,
+                                          int64_t* counts_host, void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_step_host"));
+    if (!params || !out || !counts_host || (n_seeds > 0 && !seeds_host)) return fail(MOMENT_EINVAL, "moment_step_host: null argument");
+    if (n_seeds > ctx->max_seeds) return fail(MOMENT_EINVAL, "moment_step_host: n_seeds > max_seeds");
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    MOMENT_TRY(cuda_check(cudaMemcpyAsync(ctx->d_seed_stage, seeds_host, n_seeds * sizeof(int64_t), cudaMemcpyHostToDevice, s), "moment_step_host: H2D"));
+    MOMENT_TRY(launch_sample(ctx, csr, ctx->d_seed_stage, n_seeds, params, out, s));
+    const int H = params->n_hops;
+    if (d_rows) MOMENT_TRY(launch_gather(ctx, out->nodes, out->counts + H, out->cap_nodes, d_rows, nullptr, ctx->rank, s));
+    MOMENT_TRY(cuda_check(cudaMemcpyAsync(counts_host, out->counts, (2 * H + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "moment_step_host: D2H"));
+    return cuda_check(cudaStreamSynchronize(s), "moment_step_host: sync");
+}

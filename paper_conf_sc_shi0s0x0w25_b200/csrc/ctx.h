@@ -1,0 +1,81 @@
+// ctx.h — device context of one rank and the small device helpers shared by the kernels.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <vector>
+
+#include "moment.h"
+#include "status.h"
+
+struct moment_ctx_s {
+    int32_t rank = 0, world = 1, device = 0;
+    int64_t n_vertices = 0;
+    int64_t max_seeds = 0;
+    int32_t max_hops = 0;
+    std::vector<int32_t> max_fanout;
+    std::vector<int64_t> max_F;  // per hop h = 0..max_hops: bound on |F_h|
+    std::vector<int64_t> max_E;  // per hop: bound on E_h
+    int64_t max_nodes = 0, max_edges = 0, max_offsets = 0;
+    int64_t row_bytes = 0, row_stride = 0;
+    int32_t n_bins = 0;
+    std::vector<int32_t> bin_owner;
+    std::vector<void*> bin_ptr;
+    const uint64_t* placement = nullptr;
+    std::vector<int64_t> quota;  // [n_bins][world]
+
+    // device workspace (one allocation, carved)
+    void* ws = nullptr;
+    int64_t ws_bytes = 0;
+    int32_t* lidx = nullptr;        // [n_vertices]: local index of v in the current batch (valid for F_H)
+    uint32_t* newbits = nullptr;    // [n_words]: ids emitted at the current hop
+    uint32_t* visited = nullptr;    // [n_words]: F_h membership
+    int64_t n_words = 0;
+    uint64_t* tile_status = nullptr;  // decoupled look-back descriptors, all hops, both scans
+    int64_t n_tile_status = 0;
+    std::vector<int64_t> sample_tiles_off, bitscan_tiles_off;  // per hop offsets into tile_status
+    uint32_t* tickets = nullptr;      // [2 * max_hops] tile tickets
+    uint32_t* error_flag = nullptr;   // device error bits (seed check)
+    // bucketing workspace
+    int64_t max_requests = 0;
+    int64_t* bk_tile_counts = nullptr;  // [n_tiles][n_bins]
+    int64_t* bk_bin_total = nullptr;    // [n_bins]
+    int64_t* bk_qoff = nullptr;         // [n_bins * world + 1] (internal, when caller passes none)
+    int32_t* bk_route = nullptr;        // [max_requests]
+    int64_t* bk_qpos = nullptr;         // [max_requests]
+    int64_t* d_quota = nullptr;         // [n_bins * world]
+    int32_t* d_bin_owner = nullptr;     // [n_bins]
+    int64_t* d_seed_stage = nullptr;    // [max_seeds] for moment_step_host
+    int64_t* d_counts_stage = nullptr;  // unused placeholder
+};
+
+namespace moment {
+
+inline moment_status cuda_check(cudaError_t e, const char* what) {
+    if (e != cudaSuccess) return fail(MOMENT_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+    return MOMENT_OK;
+}
+
+// Report a pending asynchronous CUDA fault (from earlier work) without synchronising.
+inline moment_status cuda_pending(const char* what) { return cuda_check(cudaPeekAtLastError(), what); }
+
+constexpr int kSampleTile = 256;     // frontier nodes per sampler tile
+constexpr int kBitscanWordsPerThread = 8;
+constexpr int kBitscanThreads = 256;
+constexpr int kBitscanTileWords = kBitscanWordsPerThread * kBitscanThreads;  // 2048 words = 65536 ids
+constexpr int kBucketTile = 1024;    // requests per bucketing tile
+constexpr int kMaxFanout = 1024;
+
+// Launchers (defined in sample.cu / gather.cu).
+moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
+                            const moment_sample_params* p, const moment_sample_out* out, cudaStream_t stream);
+moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n, void* out,
+                            const int32_t* route, int32_t serve_rank, cudaStream_t stream);
+moment_status launch_bucket(moment_ctx_s* ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n,
+                            int32_t* route, int64_t* qoff, int64_t* qpos, cudaStream_t stream);
+moment_status launch_relay(moment_ctx_s* server, moment_ctx_s* requester, const int64_t* ids, const int32_t* route,
+                           const int64_t* qoff, const int64_t* qpos, void* requester_out, cudaStream_t stream);
+moment_status launch_hotness(const int64_t* ids, const int64_t* n_dev, int64_t max_n, uint64_t* hot,
+                             cudaStream_t stream);
+
+}  // namespace moment

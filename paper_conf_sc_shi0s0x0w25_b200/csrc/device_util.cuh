@@ -1,0 +1,90 @@
+// device_util.cuh — device-side building blocks: Philox4x32-10, block scan, decoupled look-back.
+#pragma once
+#include <cuda/atomic>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+namespace moment {
+namespace dev {
+
+// Philox4x32-10 (Salmon et al., SC '11): the counter-based stream the sampler draws from (R1).
+__device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 k) {
+#pragma unroll
+    for (int r = 0; r < 10; r++) {
+        const uint32_t lo0 = 0xD2511F53u * c.x, hi0 = __umulhi(0xD2511F53u, c.x);
+        const uint32_t lo1 = 0xCD9E8D57u * c.z, hi1 = __umulhi(0xCD9E8D57u, c.z);
+        c = make_uint4(hi1 ^ c.y ^ k.x, lo1, hi0 ^ c.w ^ k.y, lo0);
+        k.x += 0x9E3779B9u;
+        k.y += 0xBB67AE85u;
+    }
+    return c;
+}
+
+// draw(seed, v, h, i): word i & 3 of Philox(ctr = (lo v, hi v, h, i >> 2), key = (lo seed, hi seed)).
+__device__ __forceinline__ uint32_t draw(uint64_t seed, int64_t v, int32_t h, int32_t i) {
+    const uint4 r = philox4x32_10(make_uint4((uint32_t)v, (uint32_t)((uint64_t)v >> 32), (uint32_t)h, (uint32_t)(i >> 2)),
+                                  make_uint2((uint32_t)seed, (uint32_t)(seed >> 32)));
+    const int w = i & 3;
+    return w == 0 ? r.x : (w == 1 ? r.y : (w == 2 ? r.z : r.w));
+}
+
+// Integer in [0, m) from a 32-bit draw: floor(r m / 2^32) (R2).
+__device__ __forceinline__ uint32_t uniform(uint32_t r, uint32_t m) {
+    return (uint32_t)(((uint64_t)r * (uint64_t)m) >> 32);
+}
+
+// Block-wide exclusive scan of one int64 per thread (blockDim.x == NT, multiple of 32).
+template <int NT>
+__device__ __forceinline__ int64_t block_exclusive_scan(int64_t x, int64_t* total, int64_t* warp_sums) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    int64_t incl = x;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        int64_t y = __shfl_up_sync(0xffffffffu, incl, d);
+        if (lane >= d) incl += y;
+    }
+    if (lane == 31) warp_sums[wid] = incl;
+    __syncthreads();
+    if (wid == 0) {
+        int64_t w = lane < NT / 32 ? warp_sums[lane] : 0;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            int64_t y = __shfl_up_sync(0xffffffffu, w, d);
+            if (lane >= d) w += y;
+        }
+        if (lane < NT / 32) warp_sums[lane] = w;  // inclusive
+    }
+    __syncthreads();
+    const int64_t warp_base = wid > 0 ? warp_sums[wid - 1] : 0;
+    *total = warp_sums[NT / 32 - 1];
+    return warp_base + incl - x;
+}
+
+// Decoupled look-back (single-pass chained scan). Descriptor: bits 62..63 = state (0 empty,
+// 1 aggregate, 2 inclusive prefix), bits 0..61 = value. Called by ONE thread per tile; tiles are taken
+// in increasing order through an atomic ticket, so every predecessor tile is owned by a running block.
+constexpr uint64_t kFlagAgg = 1ull << 62, kFlagPrefix = 2ull << 62, kValMask = (1ull << 62) - 1;
+
+__device__ __forceinline__ int64_t lookback(uint64_t* status, int64_t tile, int64_t aggregate) {
+    using ref = cuda::atomic_ref<unsigned long long, cuda::thread_scope_device>;
+    if (tile == 0) {
+        ref(*reinterpret_cast<unsigned long long*>(&status[0])).store(kFlagPrefix | (uint64_t)aggregate, cuda::memory_order_release);
+        return 0;
+    }
+    ref(*reinterpret_cast<unsigned long long*>(&status[tile])).store(kFlagAgg | (uint64_t)aggregate, cuda::memory_order_release);
+    int64_t exclusive = 0;
+    for (int64_t j = tile - 1; j >= 0;) {
+        const uint64_t s = ref(*reinterpret_cast<unsigned long long*>(&status[j])).load(cuda::memory_order_acquire);
+        const uint64_t flag = s & ~kValMask;
+        if (flag == 0) continue;  // predecessor not published yet: spin
+        exclusive += (int64_t)(s & kValMask);
+        if (flag == kFlagPrefix) break;
+        j--;
+    }
+    ref(*reinterpret_cast<unsigned long long*>(&status[tile])).store(kFlagPrefix | (uint64_t)(exclusive + aggregate), cuda::memory_order_release);
+    return exclusive;
+}
+
+}  // namespace dev
+}  // namespace moment

@@ -1,0 +1,347 @@
+// gather.cu — H4-H7 and P2 on sm_100a: placement lookup + bucketing, the 128-bit tiered row gather
+// (local HBM / NVLink peer HBM / zero-copy pinned host), the relay of host rows for another rank, and
+// the hotness histogram of pre-sampling.
+#include <algorithm>
+
+#include "ctx.h"
+#include "device_util.cuh"
+
+namespace moment {
+namespace {
+
+constexpr int kGatherThreads = 256;
+constexpr int kGatherUnroll = 8;  // 16-byte loads in flight per thread
+constexpr uint64_t kSlotMask = (1ull << 40) - 1;
+constexpr int kMaxQueues = 128;  // n_bins * world
+
+struct BinTable {
+    const int4* base[MOMENT_MAX_BINS];  // bin base as addressable from the launching device
+    int8_t owner[MOMENT_MAX_BINS];      // owning rank of an HBM bin, -1 for a host-DRAM bin
+};
+
+__device__ __forceinline__ int4 ld_stream(const int4* p) {
+    int4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+                 : "l"(p));
+    return r;
+}
+
+// Division of a 32-bit index by the runtime row width: q = umulhi64(e, ceil(2^64 / d)) is exact for
+// e < 2^32 (Lemire et al., "Faster remainder by direct computation").
+struct FastDiv {
+    uint64_t m;
+    uint32_t d;
+};
+__device__ __forceinline__ uint32_t fdiv(uint32_t e, const FastDiv& f) {
+    return f.d == 1 ? e : (uint32_t)__umul64hi((uint64_t)e, f.m);
+}
+
+FastDiv make_fastdiv(uint32_t d) { return FastDiv{d == 1 ? 0ull : (~0ull / d + 1), d}; }
+
+// out[i] = row(ids[i]) for i < n, one 16-byte vector per thread step, kGatherUnroll loads in flight.
+// placement == nullptr: replicated table in bin 0 at slot = id. route != nullptr: requests whose route
+// says "relay through rank != self" are skipped (the relay rank writes them).
+__global__ void __launch_bounds__(kGatherThreads) gather_kernel(BinTable bins, const uint64_t* __restrict__ placement,
+                                                                const int64_t* __restrict__ ids, const int64_t* n_dev,
+                                                                int64_t max_n, FastDiv rv, int64_t stride_vec,
+                                                                const int32_t* __restrict__ route, int32_t world,
+                                                                int32_t self, int4* __restrict__ out) {
+    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+    const uint32_t total = (uint32_t)(n * rv.d);
+    const uint32_t step = gridDim.x * kGatherThreads * kGatherUnroll;
+    for (uint32_t base = blockIdx.x * kGatherThreads * kGatherUnroll + threadIdx.x; base < total; base += step) {
+        int4 val[kGatherUnroll];
+        bool live[kGatherUnroll];
+#pragma unroll
+        for (int u = 0; u < kGatherUnroll; u++) {
+            const uint32_t e = base + u * kGatherThreads;
+            live[u] = e < total;
+            if (live[u]) {
+                const uint32_t row = fdiv(e, rv);
+                const uint32_t col = e - row * rv.d;
+                const int64_t id = __ldg(ids + row);
+                const int4* src;
+                if (placement) {
+                    const uint64_t p = __ldg(placement + id);
+                    const int b = (int)(p >> 40);
+                    if (route && bins.owner[b] < 0 && (__ldg(route + row) % world) != self) {
+                        live[u] = false;
+                        continue;
+                    }
+                    src = bins.base[b] + (int64_t)(p & kSlotMask) * stride_vec + col;
+                } else {
+                    src = bins.base[0] + id * stride_vec + col;
+                }
+                val[u] = ld_stream(src);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kGatherUnroll; u++)
+            if (live[u]) out[base + u * kGatherThreads] = val[u];
+    }
+}
+
+// Relay service (H7): this rank (server) reads the host rows that `requester` routed through it and
+// stores them into the requester's output (an NVLink store when the requester is another GPU).
+// Requests are the queue segments q = j * world + server of every host bin j.
+__global__ void __launch_bounds__(kGatherThreads) relay_kernel(BinTable bins, const uint64_t* __restrict__ placement,
+                                                               const int64_t* __restrict__ ids,
+                                                               const int64_t* __restrict__ qoff,
+                                                               const int64_t* __restrict__ qpos, int32_t n_bins,
+                                                               int32_t world, int32_t server, FastDiv rv,
+                                                               int64_t stride_vec, int4* __restrict__ out) {
+    for (int b = 0; b < n_bins; b++) {
+        if (bins.owner[b] >= 0) continue;  // HBM bins are read by the requester itself (peer load)
+        const int q = b * world + server;
+        const int64_t lo = qoff[q], cnt = qoff[q + 1] - lo;
+        const uint32_t total = (uint32_t)(cnt * rv.d);
+        for (uint32_t e = blockIdx.x * kGatherThreads + threadIdx.x; e < total; e += gridDim.x * kGatherThreads) {
+            const uint32_t r = fdiv(e, rv);
+            const uint32_t col = e - r * rv.d;
+            const int64_t i = __ldg(qpos + lo + r);
+            const uint64_t p = __ldg(placement + __ldg(ids + i));
+            const int4 v = ld_stream(bins.base[(int)(p >> 40)] + (int64_t)(p & kSlotMask) * stride_vec + col);
+            out[i * rv.d + col] = v;
+        }
+    }
+}
+
+// ---- bucketing (H4) -------------------------------------------------------------------------------
+// Pass 1: per tile of kBucketTile requests, per-bin counts.
+__global__ void bucket_count_kernel(const uint64_t* __restrict__ placement, const int64_t* __restrict__ ids,
+                                    const int64_t* n_dev, int64_t max_n, int32_t n_bins, int64_t* tile_counts) {
+    __shared__ int s_cnt[MOMENT_MAX_BINS];
+    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+    const int64_t n_tiles_max = (max_n + kBucketTile - 1) / kBucketTile;
+    for (int64_t tile = blockIdx.x; tile < n_tiles_max; tile += gridDim.x) {
+        for (int b = threadIdx.x; b < n_bins; b += blockDim.x) s_cnt[b] = 0;
+        __syncthreads();
+        for (int64_t i = tile * kBucketTile + threadIdx.x; i < min(n, (tile + 1) * kBucketTile); i += blockDim.x) {
+            const int b = (int)(__ldg(placement + __ldg(ids + i)) >> 40);
+            atomicAdd(&s_cnt[b], 1);
+        }
+        __syncthreads();
+        for (int b = threadIdx.x; b < n_bins; b += blockDim.x) tile_counts[tile * n_bins + b] = s_cnt[b];
+        __syncthreads();
+    }
+}
+
+// Pass 2 (one block): exclusive scan over tiles per bin; bin totals.
+__global__ void bucket_scan_kernel(int64_t* tile_counts, int64_t n_tiles, int32_t n_bins, int64_t* bin_total) {
+    for (int b = threadIdx.x; b < n_bins; b += blockDim.x) {
+        int64_t run = 0;
+        for (int64_t t = 0; t < n_tiles; t++) {
+            const int64_t c = tile_counts[t * n_bins + b];
+            tile_counts[t * n_bins + b] = run;
+            run += c;
+        }
+        bin_total[b] = run;
+    }
+}
+
+// Pass 3: stable rank r of each request inside its bin -> route. A host bin j with W = sum_h x[j][h]
+// sends rank r through the first h with floor(r W / n_j) < cumsum_h x[j][.]; equivalently rank r goes
+// to h iff r_lo(h) <= r < r_lo(h+1), r_lo(h) = ceil(C_h n_j / W), C_h = sum_{h'<h} x[j][h'].
+__global__ void __launch_bounds__(kBucketTile) bucket_route_kernel(
+    const uint64_t* __restrict__ placement, const int64_t* __restrict__ ids, const int64_t* n_dev, int64_t max_n,
+    int32_t n_bins, int32_t world, int32_t self, const int32_t* __restrict__ bin_owner_dev,
+    const int64_t* __restrict__ quota, const int64_t* __restrict__ tile_base, const int64_t* __restrict__ bin_total,
+    int32_t* __restrict__ route) {
+    __shared__ int s_warp_cnt[kBucketTile / 32][MOMENT_MAX_BINS];
+    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+    const int64_t n_tiles_max = (max_n + kBucketTile - 1) / kBucketTile;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    for (int64_t tile = blockIdx.x; tile < n_tiles_max; tile += gridDim.x) {
+        const int64_t i = tile * kBucketTile + threadIdx.x;
+        const bool live = i < n;
+        const int b = live ? (int)(__ldg(placement + __ldg(ids + i)) >> 40) : -1;
+        // rank within the warp among equal bins, then within the tile via per-warp counts
+        const unsigned peers = __match_any_sync(0xffffffffu, b);
+        const int in_warp = __popc(peers & ((1u << lane) - 1));
+        for (int q = lane; q < n_bins; q += 32) s_warp_cnt[wid][q] = 0;
+        __syncwarp();
+        if (live && in_warp == 0) s_warp_cnt[wid][b] = __popc(peers);
+        __syncthreads();
+        if (live) {
+            int before = 0;
+            for (int w = 0; w < wid; w++) before += s_warp_cnt[w][b];
+            const int64_t r = tile_base[tile * n_bins + b] + before + in_warp;
+            int via;
+            const int owner = bin_owner_dev[b];
+            if (owner >= 0) {
+                via = owner;
+            } else {
+                const int64_t* x = quota + (int64_t)b * world;
+                int64_t W = 0;
+                for (int h = 0; h < world; h++) W += x[h];
+                if (W == 0) {
+                    via = self;
+                } else {
+                    const int64_t nj = bin_total[b];
+                    // slot = floor(r W / nj) (int128), via = first h with slot < cumsum
+                    const unsigned __int128 prod = (unsigned __int128)r * (unsigned __int128)W;
+                    const int64_t slot = (int64_t)(prod / (unsigned __int128)nj);
+                    int64_t cum = 0;
+                    via = world - 1;
+                    for (int h = 0; h < world; h++) {
+                        cum += x[h];
+                        if (slot < cum) { via = h; break; }
+                    }
+                }
+            }
+            route[i] = b * world + via;
+        }
+        __syncthreads();
+    }
+}
+
+// Queue layout: stable counting sort of requests by route (q = bin * world + via).
+__global__ void queue_count_kernel(const int32_t* __restrict__ route, const int64_t* n_dev, int64_t max_n, int32_t Q,
+                                   int64_t* tile_counts) {
+    __shared__ int s_cnt[kMaxQueues];
+    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+    const int64_t n_tiles_max = (max_n + kBucketTile - 1) / kBucketTile;
+    for (int64_t tile = blockIdx.x; tile < n_tiles_max; tile += gridDim.x) {
+        for (int q = threadIdx.x; q < Q; q += blockDim.x) s_cnt[q] = 0;
+        __syncthreads();
+        for (int64_t i = tile * kBucketTile + threadIdx.x; i < min(n, (tile + 1) * kBucketTile); i += blockDim.x)
+            atomicAdd(&s_cnt[route[i]], 1);
+        __syncthreads();
+        for (int q = threadIdx.x; q < Q; q += blockDim.x) tile_counts[tile * Q + q] = s_cnt[q];
+        __syncthreads();
+    }
+}
+
+// One block: qoff[q] = sum of all counts of queues < q; tile_counts -> absolute tile bases.
+__global__ void queue_scan_kernel(int64_t* tile_counts, int64_t n_tiles, int32_t Q, int64_t* qoff) {
+    __shared__ int64_t s_tot[kMaxQueues + 1];
+    for (int q = threadIdx.x; q < Q; q += blockDim.x) {
+        int64_t run = 0;
+        for (int64_t t = 0; t < n_tiles; t++) {
+            const int64_t c = tile_counts[t * Q + q];
+            tile_counts[t * Q + q] = run;
+            run += c;
+        }
+        s_tot[q] = run;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int64_t run = 0;
+        for (int q = 0; q < Q; q++) {
+            qoff[q] = run;
+            run += s_tot[q];
+        }
+        qoff[Q] = run;
+    }
+    __syncthreads();
+    for (int q = threadIdx.x; q < Q; q += blockDim.x)
+        for (int64_t t = 0; t < n_tiles; t++) tile_counts[t * Q + q] += qoff[q];
+}
+
+__global__ void __launch_bounds__(kBucketTile) queue_scatter_kernel(const int32_t* __restrict__ route,
+                                                                    const int64_t* n_dev, int64_t max_n, int32_t Q,
+                                                                    const int64_t* __restrict__ tile_base,
+                                                                    int64_t* __restrict__ qpos) {
+    __shared__ int s_warp_cnt[kBucketTile / 32][kMaxQueues];
+    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+    const int64_t n_tiles_max = (max_n + kBucketTile - 1) / kBucketTile;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    for (int64_t tile = blockIdx.x; tile < n_tiles_max; tile += gridDim.x) {
+        const int64_t i = tile * kBucketTile + threadIdx.x;
+        const bool live = i < n;
+        const int q = live ? route[i] : -1;
+        const unsigned peers = __match_any_sync(0xffffffffu, q);
+        const int in_warp = __popc(peers & ((1u << lane) - 1));
+        for (int c = lane; c < Q; c += 32) s_warp_cnt[wid][c] = 0;
+        __syncwarp();
+        if (live && in_warp == 0) s_warp_cnt[wid][q] = __popc(peers);
+        __syncthreads();
+        if (live) {
+            int before = 0;
+            for (int w = 0; w < wid; w++) before += s_warp_cnt[w][q];
+            qpos[tile_base[tile * Q + q] + before + in_warp] = i;
+        }
+        __syncthreads();
+    }
+}
+
+__global__ void hotness_kernel(const int64_t* __restrict__ ids, const int64_t* n_dev, int64_t max_n, uint64_t* hot) {
+    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(reinterpret_cast<unsigned long long*>(hot + __ldg(ids + i)), 1ull);
+}
+
+BinTable make_bins(const moment_ctx_s* ctx) {
+    BinTable t{};
+    for (int b = 0; b < ctx->n_bins; b++) {
+        t.base[b] = reinterpret_cast<const int4*>(ctx->bin_ptr[b]);
+        t.owner[b] = (int8_t)ctx->bin_owner[b];
+    }
+    return t;
+}
+
+int grid_for(int64_t work_items, int per_block, int max_blocks) {
+    return (int)std::max<int64_t>(1, std::min<int64_t>((work_items + per_block - 1) / per_block, max_blocks));
+}
+
+}  // namespace
+
+moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n, void* out,
+                            const int32_t* route, int32_t serve_rank, cudaStream_t stream) {
+    if (max_n < 0 || (max_n > 0 && (!ids || !out))) return fail(MOMENT_EINVAL, "moment_gather: null argument");
+    if (ctx->n_bins <= 0) return fail(MOMENT_EINVAL, "moment_gather: ctx has no feature bins");
+    const int64_t rv = ctx->row_bytes / 16;
+    if (max_n * rv >= (int64_t(1) << 32))
+        return fail(MOMENT_EUNSUPPORTED, "moment_gather: %lld rows x %lld vectors exceeds 2^32 per call", (long long)max_n, (long long)rv);
+    if ((reinterpret_cast<uintptr_t>(out) & 15) != 0) return fail(MOMENT_EINVAL, "moment_gather: out must be 16-byte aligned");
+    MOMENT_TRY(cuda_pending("moment_gather: pending CUDA error"));
+    if (max_n == 0) return MOMENT_OK;
+    const int grid = grid_for(max_n * rv, kGatherThreads * kGatherUnroll, 148 * 8);
+    gather_kernel<<<grid, kGatherThreads, 0, stream>>>(make_bins(ctx), ctx->placement, ids, n_dev, max_n,
+                                                        make_fastdiv((uint32_t)rv), ctx->row_stride / 16, route,
+                                                        ctx->world, serve_rank, reinterpret_cast<int4*>(out));
+    return cuda_check(cudaGetLastError(), "moment_gather: launch");
+}
+
+moment_status launch_bucket(moment_ctx_s* ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n,
+                            int32_t* route, int64_t* qoff, int64_t* qpos, cudaStream_t stream) {
+    if (!ctx->placement) return fail(MOMENT_EINVAL, "moment_bucket: ctx has no placement map");
+    if (max_n > ctx->max_requests)
+        return fail(MOMENT_EOVERFLOW, "moment_bucket: %lld requests > workspace %lld", (long long)max_n, (long long)ctx->max_requests);
+    const int32_t Q = ctx->n_bins * ctx->world;
+    if (Q > kMaxQueues) return fail(MOMENT_EUNSUPPORTED, "moment_bucket: n_bins * world = %d > %d", Q, kMaxQueues);
+    MOMENT_TRY(cuda_pending("moment_bucket: pending CUDA error"));
+    const int64_t n_tiles = std::max<int64_t>(1, (max_n + kBucketTile - 1) / kBucketTile);
+    const int grid = (int)std::min<int64_t>(n_tiles, 148 * 2);
+    bucket_count_kernel<<<grid, 256, 0, stream>>>(ctx->placement, ids, n_dev, max_n, ctx->n_bins, ctx->bk_tile_counts);
+    bucket_scan_kernel<<<1, 64, 0, stream>>>(ctx->bk_tile_counts, n_tiles, ctx->n_bins, ctx->bk_bin_total);
+    const int32_t* owner_dev = ctx->d_bin_owner;
+    bucket_route_kernel<<<grid, kBucketTile, 0, stream>>>(ctx->placement, ids, n_dev, max_n, ctx->n_bins, ctx->world,
+                                                          ctx->rank, owner_dev, ctx->d_quota, ctx->bk_tile_counts,
+                                                          ctx->bk_bin_total, route);
+    queue_count_kernel<<<grid, 256, 0, stream>>>(route, n_dev, max_n, Q, ctx->bk_tile_counts);
+    queue_scan_kernel<<<1, 256, 0, stream>>>(ctx->bk_tile_counts, n_tiles, Q, qoff);
+    queue_scatter_kernel<<<grid, kBucketTile, 0, stream>>>(route, n_dev, max_n, Q, ctx->bk_tile_counts, qpos);
+    return cuda_check(cudaGetLastError(), "moment_bucket: launch");
+}
+
+moment_status launch_relay(moment_ctx_s* server, moment_ctx_s* requester, const int64_t* ids, const int32_t* route,
+                           const int64_t* qoff, const int64_t* qpos, void* requester_out, cudaStream_t stream) {
+    (void)route;
+    const int64_t rv = server->row_bytes / 16;
+    const int grid = 148 * 4;
+    relay_kernel<<<grid, kGatherThreads, 0, stream>>>(make_bins(server), requester->placement, ids, qoff, qpos,
+                                                       server->n_bins, server->world, server->rank,
+                                                       make_fastdiv((uint32_t)rv), server->row_stride / 16,
+                                                       reinterpret_cast<int4*>(requester_out));
+    return cuda_check(cudaGetLastError(), "moment_gather: relay launch");
+}
+
+moment_status launch_hotness(const int64_t* ids, const int64_t* n_dev, int64_t max_n, uint64_t* hot, cudaStream_t stream) {
+    if (max_n <= 0) return MOMENT_OK;
+    hotness_kernel<<<grid_for(max_n, 256, 148 * 8), 256, 0, stream>>>(ids, n_dev, max_n, hot);
+    return cuda_check(cudaGetLastError(), "moment_hotness: launch");
+}
+
+}  // namespace moment

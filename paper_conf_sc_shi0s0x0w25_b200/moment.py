@@ -1,0 +1,398 @@
+"""Thin Python binding of include/moment.h (ctypes; argument marshalling only).
+
+Every computation runs in libmoment.so: the host planner in C++, the hot path in sm_100a kernels.
+PyTorch is used for device memory and streams only. There is no fallback: if the library is missing or
+fails to load, every call raises.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "lib", "libmoment.so")
+
+OK, EINVAL, ENOMEM, ECUDA, ENCCL, EINFEASIBLE, EOVERFLOW, EUNSUPPORTED, ETIMEDOUT = 0, -1, -2, -3, -4, -5, -6, -7, -8
+CAP_INF = np.iinfo(np.int64).max
+NODE_SOURCE, NODE_SINK, NODE_STORAGE, NODE_INTERCONNECT, NODE_COMPUTE = range(5)
+TIER_NONE, TIER_GPU_HBM, TIER_HOST_DRAM, TIER_SSD = range(4)
+PLACE_DDAK, PLACE_HASH = 0, 1
+SAMPLE_REPLACE, SAMPLE_CHECK = 1, 2
+MAX_BINS = 64
+
+EXPORTED = [
+    "moment_last_error", "moment_version", "moment_topology", "moment_topology_info", "moment_topology_export",
+    "moment_topology_free", "moment_maxflow", "moment_place", "moment_place_pack", "moment_plan", "moment_plan_info",
+    "moment_plan_free", "moment_ctx_create", "moment_ctx_free", "moment_ctx_workspace_bytes", "moment_sample_bounds",
+    "moment_sample", "moment_sample_check", "moment_hotness", "moment_bucket", "moment_gather", "moment_gather_group",
+    "moment_step_host",
+]
+
+
+class MomentError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"[moment status {status}] {msg}")
+        self.status = status
+
+
+class Node(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("tier", C.c_int32), ("device", C.c_int32), ("reserved", C.c_int32)]
+
+
+class Link(C.Structure):
+    _fields_ = [("from_", C.c_int32), ("to", C.c_int32), ("cap", C.c_int64)]
+
+
+class PlaceArgs(C.Structure):
+    _fields_ = [("n_vertices", C.c_int64), ("hotness", C.c_void_p), ("n_bins", C.c_int32), ("bin_node", C.c_void_p),
+                ("bin_tier", C.c_void_p), ("bin_capacity_rows", C.c_void_p), ("bin_traffic", C.c_void_p),
+                ("pool", C.c_int64), ("mode", C.c_int32)]
+
+
+class PlaceOut(C.Structure):
+    _fields_ = [("bin_of", C.c_void_p), ("slot_of", C.c_void_p), ("bin_access", C.c_void_p),
+                ("bin_rows_used", C.c_void_p), ("bin_traffic_used", C.c_void_p)]
+
+
+class PlanArgs(C.Structure):
+    _fields_ = [("k", C.c_int32), ("gpu_node", C.c_void_p), ("bin_demand_bytes", C.c_void_p),
+                ("nvlink_cap", C.c_int64), ("hbm_cap", C.c_int64)]
+
+
+class CtxArgs(C.Structure):
+    _fields_ = [("rank", C.c_int32), ("world", C.c_int32), ("device", C.c_int32), ("n_vertices", C.c_int64),
+                ("max_seeds", C.c_int64), ("max_hops", C.c_int32), ("max_fanout", C.c_void_p),
+                ("row_bytes", C.c_int64), ("row_stride", C.c_int64), ("n_bins", C.c_int32),
+                ("bin_owner", C.c_void_p), ("bin_ptr", C.c_void_p), ("placement", C.c_void_p), ("quota", C.c_void_p)]
+
+
+class Csr(C.Structure):
+    _fields_ = [("indptr", C.c_void_p), ("indices", C.c_void_p), ("n_vertices", C.c_int64), ("n_edges", C.c_int64)]
+
+
+class SampleParams(C.Structure):
+    _fields_ = [("n_hops", C.c_int32), ("fanout", C.c_void_p), ("rng_seed", C.c_uint64), ("flags", C.c_uint32)]
+
+
+class SampleOut(C.Structure):
+    _fields_ = [("nodes", C.c_void_p), ("offsets", C.c_void_p), ("src", C.c_void_p), ("counts", C.c_void_p),
+                ("cap_nodes", C.c_int64), ("cap_offsets", C.c_int64), ("cap_edges", C.c_int64)]
+
+
+_lib = None
+P = C.c_void_p
+I32, I64, U64 = C.c_int32, C.c_int64, C.c_uint64
+
+
+def lib():
+    """Load libmoment.so (raises if it is missing: there is no fallback path)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise MomentError(EUNSUPPORTED, f"{LIB_PATH} is missing: run __graft_entry__.build()")
+        L = C.CDLL(LIB_PATH)
+        sig = {
+            "moment_last_error": ([], C.c_char_p),
+            "moment_version": ([], I32),
+            "moment_topology": ([P, I32, P, I32, P], I32),
+            "moment_topology_info": ([P, P, P, P, P], I32),
+            "moment_topology_export": ([P, P, P], I32),
+            "moment_topology_free": ([P], I32),
+            "moment_maxflow": ([P, P, P], I32),
+            "moment_place": ([P, P, P], I32),
+            "moment_place_pack": ([I64, P, P, P], I32),
+            "moment_plan": ([P, P, P], I32),
+            "moment_plan_info": ([P, P, P, P, P, P, P], I32),
+            "moment_plan_free": ([P], I32),
+            "moment_ctx_create": ([P, P], I32),
+            "moment_ctx_free": ([P], I32),
+            "moment_ctx_workspace_bytes": ([P, P], I32),
+            "moment_sample_bounds": ([I64, P, I32, I64, P, P, P], I32),
+            "moment_sample": ([P, P, P, I64, P, P, P], I32),
+            "moment_sample_check": ([P, P], I32),
+            "moment_hotness": ([P, P, P, I64, P, P], I32),
+            "moment_bucket": ([P, P, P, I64, P, P, P, P], I32),
+            "moment_gather": ([P, P, P, I64, P, P], I32),
+            "moment_gather_group": ([P, I32, P, P, I64, P, P], I32),
+            "moment_step_host": ([P, P, P, I64, P, P, P, P, P], I32),
+        }
+        for name, (args, res) in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = res
+        _lib = L
+    return _lib
+
+
+def _check(status: int):
+    if status != OK:
+        raise MomentError(status, lib().moment_last_error().decode())
+
+
+def _np(a, dtype):
+    return np.ascontiguousarray(np.asarray(a, dtype=dtype))
+
+
+def _ptr(a) -> int:
+    """Address of a numpy array or torch tensor (None -> NULL)."""
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        return a.ctypes.data
+    return a.data_ptr()
+
+
+def _stream(stream) -> int | None:
+    if stream is None:
+        import torch
+
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+# ---------------------------------------------------------------------------------------------- P1
+class Topology:
+    def __init__(self, nodes, links):
+        """nodes: [(kind, tier, device)], links: [(from, to, cap)] (cap = CAP_INF for infinite)."""
+        na = (Node * len(nodes))(*[Node(k, t, d, 0) for (k, t, d) in nodes])
+        la = (Link * max(1, len(links)))(*[Link(f, t, c) for (f, t, c) in links])
+        h = C.c_void_p()
+        _check(lib().moment_topology(C.cast(na, P), len(nodes), C.cast(la, P), len(links), C.byref(h)))
+        self.handle = h
+
+    def __del__(self):
+        if getattr(self, "handle", None) and _lib is not None:
+            _lib.moment_topology_free(self.handle)
+            self.handle = None
+
+    def info(self):
+        n, m, s, t = C.c_int32(), C.c_int32(), C.c_int32(), C.c_int32()
+        _check(lib().moment_topology_info(self.handle, C.byref(n), C.byref(m), C.byref(s), C.byref(t)))
+        return n.value, m.value, s.value, t.value
+
+    def export(self):
+        n, m, s, t = self.info()
+        na = (Node * n)()
+        la = (Link * max(1, m))()
+        _check(lib().moment_topology_export(self.handle, C.cast(na, P), C.cast(la, P)))
+        nodes = [(x.kind, x.tier, x.device) for x in na]
+        links = [(x.from_, x.to, x.cap) for x in la[:m]]
+        return nodes, links, s, t
+
+    def maxflow(self):
+        """P3: (value, per-link flow) of the rate max-flow (Dinic)."""
+        _, m, _, _ = self.info()
+        v = C.c_int64()
+        flow = np.zeros(max(m, 1), np.int64)
+        _check(lib().moment_maxflow(self.handle, C.byref(v), _ptr(flow)))
+        return v.value, flow[:m]
+
+
+def topology(nodes, links) -> Topology:
+    return Topology(nodes, links)
+
+
+# ---------------------------------------------------------------------------------------------- P4
+def place(topo: Topology | None, hotness, capacity_rows, *, bin_node=None, bin_tier=None, bin_traffic=None,
+          pool: int = 100, mode: int = PLACE_DDAK):
+    """DDAK placement. Returns (bin_of int32[n], slot_of int64[n], access uint64[nb], used int64[nb],
+    traffic int64[nb])."""
+    hot = _np(hotness, np.uint64)
+    cap = _np(capacity_rows, np.int64)
+    nb = len(cap)
+    n = len(hot)
+    keep = []
+
+    def opt(a, dt):
+        if a is None:
+            return None
+        arr = _np(a, dt)
+        keep.append(arr)
+        return arr.ctypes.data
+
+    args = PlaceArgs(n, hot.ctypes.data, nb, opt(bin_node, np.int32), opt(bin_tier, np.int32), cap.ctypes.data,
+                     opt(bin_traffic, np.int64), pool, mode)
+    bin_of = np.zeros(max(n, 1), np.int32)
+    slot_of = np.zeros(max(n, 1), np.int64)
+    acc = np.zeros(nb, np.uint64)
+    used = np.zeros(nb, np.int64)
+    traf = np.zeros(nb, np.int64)
+    out = PlaceOut(bin_of.ctypes.data, slot_of.ctypes.data, acc.ctypes.data, used.ctypes.data, traf.ctypes.data)
+    _check(lib().moment_place(topo.handle if topo is not None else None, C.byref(args), C.byref(out)))
+    return bin_of[:n], slot_of[:n], acc, used, traf
+
+
+def place_pack(bin_of, slot_of) -> np.ndarray:
+    b = _np(bin_of, np.int32)
+    s = _np(slot_of, np.int64)
+    out = np.zeros(max(len(b), 1), np.uint64)
+    _check(lib().moment_place_pack(len(b), b.ctypes.data, s.ctypes.data, out.ctypes.data))
+    return out[: len(b)]
+
+
+# ---------------------------------------------------------------------------------------------- P5
+class Plan:
+    def __init__(self, topo: Topology, gpu_node, demand_bytes, nvlink_cap: int, hbm_cap: int):
+        g = _np(gpu_node, np.int32)
+        d = _np(demand_bytes, np.int64)
+        n, m, _, _ = topo.info()
+        if len(d) != n:
+            raise MomentError(EINVAL, f"demand has {len(d)} entries, topology has {n} nodes")
+        self.k, self.n_nodes, self.n_links = len(g), n, m
+        args = PlanArgs(len(g), g.ctypes.data, d.ctypes.data, nvlink_cap, hbm_cap)
+        h = C.c_void_p()
+        _check(lib().moment_plan(topo.handle, C.byref(args), C.byref(h)))
+        self.handle = h
+
+    def __del__(self):
+        if getattr(self, "handle", None) and _lib is not None:
+            _lib.moment_plan_free(self.handle)
+            self.handle = None
+
+    def info(self):
+        ts, ti, tn, th = C.c_int64(), C.c_int64(), C.c_int64(), C.c_int64()
+        flow = np.zeros(max(self.n_links, 1), np.int64)
+        quota = np.zeros(self.n_nodes * self.k, np.int64)
+        _check(lib().moment_plan_info(self.handle, C.byref(ts), C.byref(ti), C.byref(tn), C.byref(th), _ptr(flow),
+                                      _ptr(quota)))
+        return {"t_star": ts.value, "t_ingest": ti.value, "t_nvlink": tn.value, "t_hbm": th.value,
+                "link_flow": flow[: self.n_links], "quota": quota.reshape(self.n_nodes, self.k)}
+
+
+def plan(topo, gpu_node, demand_bytes, nvlink_cap, hbm_cap) -> Plan:
+    return Plan(topo, gpu_node, demand_bytes, nvlink_cap, hbm_cap)
+
+
+# ---------------------------------------------------------------------------------------------- ctx
+def sample_bounds(n_seeds: int, fanout, n_vertices: int):
+    f = _np(fanout, np.int32)
+    a, b, c = C.c_int64(), C.c_int64(), C.c_int64()
+    _check(lib().moment_sample_bounds(n_seeds, f.ctypes.data, len(f), n_vertices, C.byref(a), C.byref(b), C.byref(c)))
+    return a.value, b.value, c.value
+
+
+@dataclass
+class SampleBuffers:
+    nodes: object
+    offsets: object
+    src: object
+    counts: object
+    fanout: tuple
+
+    @staticmethod
+    def allocate(n_seeds: int, fanout, n_vertices: int, device):
+        import torch
+
+        mn, mo, me = sample_bounds(n_seeds, fanout, n_vertices)
+        H = len(fanout)
+        return SampleBuffers(torch.empty(max(mn, 1), dtype=torch.int64, device=device),
+                             torch.empty(max(mo, 1), dtype=torch.int64, device=device),
+                             torch.empty(max(me, 1), dtype=torch.int32, device=device),
+                             torch.zeros(2 * H + 1, dtype=torch.int64, device=device), tuple(fanout))
+
+    def struct(self) -> SampleOut:
+        return SampleOut(self.nodes.data_ptr(), self.offsets.data_ptr(), self.src.data_ptr(), self.counts.data_ptr(),
+                         self.nodes.numel(), self.offsets.numel(), self.src.numel())
+
+    def result(self):
+        """Host copy split per hop, in the oracle's layout (synchronises)."""
+        H = len(self.fanout)
+        counts = self.counts.cpu().numpy()
+        F, E = counts[: H + 1], counts[H + 1:]
+        nodes = self.nodes[: F[H]].cpu().numpy()
+        offs_all = self.offsets.cpu().numpy()
+        src_all = self.src.cpu().numpy()
+        offs, srcs, ob, eb = [], [], 0, 0
+        for h in range(H):
+            offs.append(offs_all[ob: ob + F[h] + 1])
+            srcs.append(src_all[eb: eb + E[h]])
+            ob += F[h] + 1
+            eb += E[h]
+        return {"nodes": nodes, "offsets": offs, "src": srcs, "counts": counts}
+
+
+class Ctx:
+    """Device context of one rank (moment_ctx_create)."""
+
+    def __init__(self, *, n_vertices: int, max_seeds: int, max_fanout, rank: int = 0, world: int = 1, device: int = 0,
+                 row_bytes: int = 0, row_stride: int | None = None, bin_owner=(), bin_ptr=(), placement=None,
+                 quota=None):
+        mf = _np(max_fanout, np.int32)
+        owners = _np(bin_owner, np.int32) if len(bin_owner) else np.zeros(1, np.int32)
+        ptrs = (C.c_void_p * max(1, len(bin_ptr)))(*[C.c_void_p(int(p)) for p in bin_ptr])
+        q = _np(quota, np.int64) if quota is not None else None
+        self._keep = (mf, owners, ptrs, q, placement)
+        args = CtxArgs(rank, world, device, n_vertices, max_seeds, len(mf), mf.ctypes.data, row_bytes,
+                       row_stride if row_stride is not None else row_bytes, len(bin_ptr), owners.ctypes.data,
+                       C.cast(ptrs, P), _ptr(placement), q.ctypes.data if q is not None else None)
+        h = C.c_void_p()
+        _check(lib().moment_ctx_create(C.byref(args), C.byref(h)))
+        self.handle = h
+        self.rank, self.world, self.device, self.row_bytes = rank, world, device, row_bytes
+        self.n_vertices = n_vertices
+
+    def close(self):
+        if getattr(self, "handle", None) and _lib is not None:
+            _lib.moment_ctx_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        self.close()
+
+    def workspace_bytes(self) -> int:
+        b = C.c_int64()
+        _check(lib().moment_ctx_workspace_bytes(self.handle, C.byref(b)))
+        return b.value
+
+    def sample(self, indptr, indices, seeds, fanout, rng_seed: int, out: SampleBuffers, *, flags: int = 0,
+               stream=None):
+        csr = Csr(indptr.data_ptr(), indices.data_ptr(), indptr.numel() - 1, indices.numel())
+        f = _np(fanout, np.int32)
+        params = SampleParams(len(f), f.ctypes.data, rng_seed & 0xFFFFFFFFFFFFFFFF, flags)
+        so = out.struct()
+        _check(lib().moment_sample(self.handle, C.byref(csr), seeds.data_ptr(), seeds.numel(), C.byref(params),
+                                   C.byref(so), _stream(stream)))
+        return out
+
+    def sample_check(self, stream=None):
+        _check(lib().moment_sample_check(self.handle, _stream(stream)))
+
+    def gather(self, ids, out, *, n_dev=None, max_n: int | None = None, stream=None):
+        mn = ids.numel() if max_n is None else max_n
+        _check(lib().moment_gather(self.handle, ids.data_ptr(), _ptr(n_dev), mn, out.data_ptr(), _stream(stream)))
+        return out
+
+    def bucket(self, ids, route, qoff, qpos, *, n_dev=None, max_n: int | None = None, stream=None):
+        mn = ids.numel() if max_n is None else max_n
+        _check(lib().moment_bucket(self.handle, ids.data_ptr(), _ptr(n_dev), mn, route.data_ptr(), qoff.data_ptr(),
+                                   qpos.data_ptr(), _stream(stream)))
+
+    def hotness(self, ids, hot, *, n_dev=None, max_n: int | None = None, stream=None):
+        mn = ids.numel() if max_n is None else max_n
+        _check(lib().moment_hotness(self.handle, ids.data_ptr(), _ptr(n_dev), mn, hot.data_ptr(), _stream(stream)))
+
+    def step_host(self, indptr, indices, seeds_host, fanout, rng_seed: int, out: SampleBuffers, rows, counts_host,
+                  *, flags: int = 0, stream=None):
+        csr = Csr(indptr.data_ptr(), indices.data_ptr(), indptr.numel() - 1, indices.numel())
+        f = _np(fanout, np.int32)
+        params = SampleParams(len(f), f.ctypes.data, rng_seed & 0xFFFFFFFFFFFFFFFF, flags)
+        so = out.struct()
+        _check(lib().moment_step_host(self.handle, C.byref(csr), seeds_host.data_ptr(), seeds_host.numel(),
+                                      C.byref(params), C.byref(so), _ptr(rows), counts_host.data_ptr(),
+                                      _stream(stream)))
+
+
+def gather_group(ctxs, ids, out, *, n_dev=None, max_n: int, stream=None):
+    """moment_gather_group: logical ranks driven from one stream (all pointers addressable)."""
+    k = len(ctxs)
+    hs = (C.c_void_p * k)(*[c.handle for c in ctxs])
+    ip = (C.c_void_p * k)(*[t.data_ptr() for t in ids])
+    op = (C.c_void_p * k)(*[t.data_ptr() for t in out])
+    nd = (C.c_void_p * k)(*[t.data_ptr() for t in n_dev]) if n_dev is not None else None
+    _check(lib().moment_gather_group(C.cast(hs, P), k, C.cast(ip, P), C.cast(nd, P) if nd is not None else None,
+                                     max_n, C.cast(op, P), _stream(stream)))

@@ -1,0 +1,307 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+Sampling (H1-H3) is compared bit-exactly: nodes (F_H), per-hop offsets, src and counts. Gathers
+(H4-H7) are compared byte-exactly with the oracle's out[i] = table[ids[i]]. Bucketing (H4) is compared
+with the oracle's routing given the same quota. Sizes span several tiles and ragged tails; C1 runs at its
+full BASELINE size, C2 at full size with the launch configuration bench.py times.
+"""
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_sc_shi0s0x0w25_b200 as M
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+DEV = "cuda:0"
+
+
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+@pytest.fixture(scope="module")
+def c1():
+    _need_gpu()
+    cfg = W.CONFIGS["C1"]
+    g = W.rmat_csr(cfg["n"], cfg["m"], device=DEV)
+    return cfg, g
+
+
+def sample_both(orc, g, seeds, fanout, rng_seed, flags=0, ctx=None):
+    ctx = ctx or M.Ctx(n_vertices=g.n, max_seeds=max(len(seeds), 1), max_fanout=fanout, device=0)
+    bufs = M.SampleBuffers.allocate(len(seeds), fanout, g.n, DEV)
+    seeds_d = torch.as_tensor(np.asarray(seeds, np.int64), device=DEV)
+    ctx.sample(g.indptr, g.indices, seeds_d, fanout, rng_seed, bufs, flags=flags)
+    got = bufs.result()
+    want = orc.sample(g.indptr.cpu().numpy(), g.indices.cpu().numpy(), np.asarray(seeds, np.int64), fanout, rng_seed,
+                      replace=bool(flags & M.SAMPLE_REPLACE))
+    return got, want
+
+
+def assert_same_sample(got, want):
+    assert np.array_equal(got["counts"], want["counts"]), (got["counts"], want["counts"])
+    assert np.array_equal(got["nodes"], want["nodes"])
+    for h in range(len(want["offsets"])):
+        assert np.array_equal(got["offsets"][h], want["offsets"][h]), h
+        assert np.array_equal(got["src"][h], want["src"][h]), h
+
+
+def test_sample_c1_full_size(orc, c1):
+    cfg, g = c1
+    train = W.training_set(g, min_count=cfg["batch"])
+    for b, seeds in enumerate(W.epoch_batches(train, cfg["batch"], 0)[:2]):
+        got, want = sample_both(orc, g, seeds.cpu().numpy(), list(cfg["fanout"]), W.batch_rng_seed(1, 0, 0, b))
+        assert_same_sample(got, want)
+
+
+@pytest.mark.parametrize("fanout", [[15, 10, 5], [3], [1, 1, 1, 1], [25, 10], [33, 2], [64], [200]])
+@pytest.mark.parametrize("n_seeds", [1, 257, 1000])
+def test_sample_fanouts_and_ragged(orc, c1, fanout, n_seeds):
+    _, g = c1
+    rng = np.random.default_rng(n_seeds * 7 + len(fanout))
+    seeds = rng.choice(g.n, n_seeds, replace=False)
+    got, want = sample_both(orc, g, seeds, fanout, 12345 + n_seeds)
+    assert_same_sample(got, want)
+
+
+@pytest.mark.parametrize("fanout", [[10, 5], [40]])
+def test_sample_replace(orc, c1, fanout):
+    _, g = c1
+    seeds = np.random.default_rng(3).choice(g.n, 700, replace=False)
+    got, want = sample_both(orc, g, seeds, fanout, 99, flags=M.SAMPLE_REPLACE)
+    assert_same_sample(got, want)
+
+
+def test_sample_handmade_graphs(orc):
+    _need_gpu()
+    # path + isolated vertex + star + self loop + duplicate edges
+    edges = [(0, 1), (1, 2), (2, 3), (5, 6), (5, 7), (5, 8), (5, 9), (5, 10), (5, 11), (5, 12), (9, 9), (10, 11),
+             (10, 11), (10, 11)]
+    n = 13
+    edges.sort()
+    indptr = np.zeros(n + 1, np.int64)
+    for u, _ in edges:
+        indptr[u + 1] += 1
+    indptr = np.cumsum(indptr)
+    indices = np.array([v for _, v in edges], np.int32)
+    g = W.Graph(torch.as_tensor(indptr, device=DEV), torch.as_tensor(indices, device=DEV), n, len(edges))
+    for seeds, fanout in [([0, 4], [3, 3]), ([5], [3, 2, 1]), ([10, 9], [2, 2]), ([4], [5]), (list(range(13)), [2])]:
+        for seed in range(5):
+            got, want = sample_both(orc, g, seeds, fanout, seed)
+            assert_same_sample(got, want)
+
+
+def test_sample_empty_batch(orc, c1):
+    _, g = c1
+    ctx = M.Ctx(n_vertices=g.n, max_seeds=16, max_fanout=[4, 4], device=0)
+    bufs = M.SampleBuffers.allocate(0, [4, 4], g.n, DEV)
+    ctx.sample(g.indptr, g.indices, torch.zeros(0, dtype=torch.int64, device=DEV), [4, 4], 1, bufs)
+    assert list(bufs.counts.cpu().numpy()) == [0, 0, 0, 0, 0]
+
+
+def test_sample_check_flags_bad_seeds(c1):
+    _, g = c1
+    ctx = M.Ctx(n_vertices=g.n, max_seeds=16, max_fanout=[4], device=0)
+    bufs = M.SampleBuffers.allocate(3, [4], g.n, DEV)
+    ctx.sample(g.indptr, g.indices, torch.tensor([1, 2, 1], device=DEV), [4], 1, bufs, flags=M.SAMPLE_CHECK)
+    with pytest.raises(M.MomentError):
+        ctx.sample_check()
+    ctx.sample(g.indptr, g.indices, torch.tensor([1, 2, g.n + 5], device=DEV), [4], 1, bufs, flags=M.SAMPLE_CHECK)
+    with pytest.raises(M.MomentError):
+        ctx.sample_check()
+    ctx.sample(g.indptr, g.indices, torch.tensor([1, 2, 3], device=DEV), [4], 1, bufs, flags=M.SAMPLE_CHECK)
+    ctx.sample_check()
+    with pytest.raises(M.MomentError) as e:  # host-side argument errors
+        ctx.sample(g.indptr, g.indices, torch.tensor([1, 2, 3], device=DEV), [5], 1, bufs)
+    assert e.value.status == M.EINVAL
+
+
+def test_sample_reused_ctx_many_batches(orc, c1):
+    """The workspace (lidx, bitmaps, tile descriptors) is reset correctly between calls."""
+    cfg, g = c1
+    ctx = M.Ctx(n_vertices=g.n, max_seeds=1024, max_fanout=[10, 5], device=0)
+    rng = np.random.default_rng(0)
+    for b in range(4):
+        seeds = rng.choice(g.n, int(rng.integers(1, 1024)), replace=False)
+        got, want = sample_both(orc, g, seeds, [10, 5], b, ctx=ctx)
+        assert_same_sample(got, want)
+
+
+@pytest.mark.parametrize("dim,dtype", [(4, torch.float32), (12, torch.float32), (100, torch.float32),
+                                       (128, torch.float32), (768, torch.float16), (1024, torch.float32)])
+def test_gather_replicated(orc, dim, dtype):
+    _need_gpu()
+    n = 5000
+    table = W.feature_table(n, dim, dtype, device=DEV)
+    R = table.shape[1]
+    rng = np.random.default_rng(dim)
+    for count in [1, 31, 1000, 4099]:
+        ids = torch.as_tensor(rng.integers(0, n, count), device=DEV)
+        ctx = M.Ctx(n_vertices=n, max_seeds=1, max_fanout=[1], device=0, row_bytes=R, bin_owner=[0],
+                    bin_ptr=[table.data_ptr()])
+        out = torch.empty((count, R), dtype=torch.uint8, device=DEV)
+        ctx.gather(ids, out)
+        want = orc.gather(table.cpu().numpy(), ids.cpu().numpy())
+        assert np.array_equal(out.cpu().numpy(), want)
+        # device count smaller than max_n: only the first n_dev rows are written
+        out2 = torch.zeros((count, R), dtype=torch.uint8, device=DEV)
+        nd = torch.tensor([count // 2], dtype=torch.int64, device=DEV)
+        ctx.gather(ids, out2, n_dev=nd)
+        o2 = out2.cpu().numpy()
+        assert np.array_equal(o2[: count // 2], want[: count // 2]) and not o2[count // 2:].any()
+
+
+def build_tiered(table, bin_of, slot_of, owners, host_bins, device=DEV):
+    """Materialise bins from a placement: HBM bins as device buffers, host bins as pinned host memory."""
+    R = table.shape[1]
+    nb = len(owners)
+    bins = []
+    t_cpu = table.cpu()
+    b_t = torch.as_tensor(bin_of)
+    s_t = torch.as_tensor(slot_of)
+    for b in range(nb):
+        sel = torch.nonzero(b_t == b).flatten()
+        rows = max(1, int(s_t[sel].max()) + 1) if len(sel) else 1
+        buf = torch.zeros((rows, R), dtype=torch.uint8)
+        buf[s_t[sel]] = t_cpu[sel]
+        if b in host_bins:
+            buf = buf.pin_memory()
+        else:
+            buf = buf.to(device)
+        bins.append(buf)
+    return bins
+
+
+def test_gather_tiered_and_bucket_vs_oracle(orc, c1):
+    """DDAK placement over 2 HBM bins (local + 'peer') and 2 pinned host bins; routed gather for rank 0."""
+    cfg, g = c1
+    n = g.n
+    table = W.feature_table(n, 32, torch.float32, device=DEV)  # 128-byte rows
+    R = table.shape[1]
+    train = W.training_set(g, min_count=1024)
+    seeds = W.epoch_batches(train, 1024, 0)[0]
+    # hotness from product pre-sampling (P2), compared with the oracle sampler's counts
+    ctx_s = M.Ctx(n_vertices=n, max_seeds=1024, max_fanout=[10, 5], device=0)
+    hot = torch.zeros(n, dtype=torch.int64, device=DEV)
+    hot_np = np.zeros(n, np.uint64)
+    for b in range(3):
+        bufs = M.SampleBuffers.allocate(1024, [10, 5], n, DEV)
+        ctx_s.sample(g.indptr, g.indices, seeds, [10, 5], 1000 + b, bufs)
+        ctx_s.hotness(bufs.nodes, hot, n_dev=bufs.counts[2:3], max_n=bufs.nodes.numel())
+        ref = orc.sample(g.indptr.cpu().numpy(), g.indices.cpu().numpy(), seeds.cpu().numpy(), [10, 5], 1000 + b)
+        np.add.at(hot_np, ref["nodes"], 1)
+    assert np.array_equal(hot.cpu().numpy().astype(np.uint64), hot_np)
+    owners = [0, 1, -1, -1]
+    tiers = [M.TIER_GPU_HBM, M.TIER_GPU_HBM, M.TIER_HOST_DRAM, M.TIER_HOST_DRAM]
+    caps = [n // 8, n // 8, n // 2, n]
+    bin_of, slot_of, *_ = M.place(None, hot_np, caps, bin_tier=tiers, bin_traffic=[500, 300, 50, 40], pool=100)
+    bins = build_tiered(table, bin_of, slot_of, owners, host_bins={2, 3})
+    placement = torch.as_tensor(M.place_pack(bin_of, slot_of).view(np.int64), device=DEV)
+    world = 2
+    quota = np.zeros((4, world), np.int64)
+    quota[2] = [3, 1]  # host bin 2: 3/4 of rank 0's requests direct, 1/4 via rank 1
+    quota[3] = [1, 1]
+    ctx = M.Ctx(n_vertices=n, max_seeds=1024, max_fanout=[10, 5], rank=0, world=world, device=0, row_bytes=R,
+                bin_owner=owners, bin_ptr=[b.data_ptr() for b in bins], placement=placement, quota=quota)
+    bufs = M.SampleBuffers.allocate(1024, [10, 5], n, DEV)
+    ctx.sample(g.indptr, g.indices, seeds, [10, 5], 7, bufs)
+    nF = int(bufs.counts[2])
+    ids = bufs.nodes[:nF].clone()
+    route = torch.empty(nF, dtype=torch.int32, device=DEV)
+    qoff = torch.empty(4 * world + 1, dtype=torch.int64, device=DEV)
+    qpos = torch.empty(nF, dtype=torch.int64, device=DEV)
+    ctx.bucket(ids, route, qoff, qpos)
+    o_route, o_qoff, o_qpos = orc.bucket(0, world, owners, quota, bin_of[ids.cpu().numpy()])
+    assert np.array_equal(route.cpu().numpy(), o_route)
+    assert np.array_equal(qoff.cpu().numpy(), o_qoff)
+    assert np.array_equal(qpos.cpu().numpy(), o_qpos)
+    # single-rank gather refuses quotas that relay through another rank
+    out = torch.empty((nF, R), dtype=torch.uint8, device=DEV)
+    with pytest.raises(M.MomentError) as e:
+        ctx.gather(ids, out)
+    assert e.value.status == M.EUNSUPPORTED
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_gather_group_relay_logical_ranks(orc, c1, world):
+    """k logical ranks on one GPU: per-rank HBM bins (peer loads), 2 host bins with quota relays."""
+    cfg, g = c1
+    n = g.n
+    table = W.feature_table(n, 100, torch.float32, device=DEV)  # 400-byte rows
+    R = table.shape[1]
+    rng = np.random.default_rng(world)
+    hot = rng.pareto(1.0, n).astype(np.uint64)
+    owners = list(range(world)) + [-1, -1]
+    tiers = [M.TIER_GPU_HBM] * world + [M.TIER_HOST_DRAM] * 2
+    caps = [n // (4 * world)] * world + [n // 2, n]
+    bin_of, slot_of, *_ = M.place(None, hot, caps, bin_tier=tiers, bin_traffic=[100] * world + [10, 10])
+    bins = build_tiered(table, bin_of, slot_of, owners, host_bins={world, world + 1})
+    placement = torch.as_tensor(M.place_pack(bin_of, slot_of).view(np.int64), device=DEV)
+    quota = np.zeros((world + 2, world), np.int64)
+    quota[world] = rng.integers(0, 5, world) + 1
+    quota[world + 1] = np.arange(world)  # rank 0 gets nothing directly
+    ctxs, ids, outs, nds = [], [], [], []
+    train = W.training_set(g, min_count=1024 * world)
+    for r in range(world):
+        ctx = M.Ctx(n_vertices=n, max_seeds=1024, max_fanout=[10, 5], rank=r, world=world, device=0, row_bytes=R,
+                    bin_owner=owners, bin_ptr=[b.data_ptr() for b in bins], placement=placement, quota=quota)
+        seeds = W.epoch_batches(train, 1024, 0, rank=r, world=world)[0]
+        bufs = M.SampleBuffers.allocate(1024, [10, 5], n, DEV)
+        ctx.sample(g.indptr, g.indices, seeds, [10, 5], 50 + r, bufs)
+        ctxs.append(ctx)
+        ids.append(bufs.nodes)
+        nds.append(bufs.counts[2:3])
+        outs.append(torch.zeros((bufs.nodes.numel(), R), dtype=torch.uint8, device=DEV))
+    max_n = max(t.numel() for t in ids)
+    ids = [torch.nn.functional.pad(t, (0, max_n - t.numel())) for t in ids]
+    outs = [torch.zeros((max_n, R), dtype=torch.uint8, device=DEV) for _ in range(world)]
+    M.gather_group(ctxs, ids, outs, n_dev=nds, max_n=max_n)
+    tab = table.cpu().numpy()
+    for r in range(world):
+        nF = int(nds[r])
+        want = orc.gather(tab, ids[r][:nF].cpu().numpy())
+        assert np.array_equal(outs[r][:nF].cpu().numpy(), want), r
+
+
+def test_step_host_matches_device_path(orc, c1):
+    cfg, g = c1
+    n = g.n
+    table = W.feature_table(n, 128, torch.float32, device=DEV)
+    R = table.shape[1]
+    ctx = M.Ctx(n_vertices=n, max_seeds=1024, max_fanout=[10, 5], device=0, row_bytes=R, bin_owner=[0],
+                bin_ptr=[table.data_ptr()])
+    train = W.training_set(g, min_count=1024)
+    seeds = W.epoch_batches(train, 1024, 0)[0]
+    bufs = M.SampleBuffers.allocate(1024, [10, 5], n, DEV)
+    rows = torch.empty((bufs.nodes.numel(), R), dtype=torch.uint8, device=DEV)
+    counts_h = torch.zeros(5, dtype=torch.int64).pin_memory()
+    seeds_h = seeds.cpu().pin_memory()
+    ctx.step_host(g.indptr, g.indices, seeds_h, [10, 5], 77, bufs, rows, counts_h)
+    want = orc.sample(g.indptr.cpu().numpy(), g.indices.cpu().numpy(), seeds_h.numpy(), [10, 5], 77)
+    assert np.array_equal(counts_h.numpy(), want["counts"])
+    nF = int(want["counts"][2])
+    assert np.array_equal(rows[:nF].cpu().numpy(), orc.gather(table.cpu().numpy(), want["nodes"]))
+
+
+def test_c2_full_size_bench_configuration(orc):
+    """C2 at BASELINE size, in bench.py's launch configuration: whole-batch sample parity + sampled rows."""
+    _need_gpu()
+    import bench
+
+    st = bench.build_state("C2", device=DEV, rank=0, world=1)
+    for b in range(2):
+        seeds, rng_seed = st.batch(b)
+        st.step(seeds, rng_seed)
+        torch.cuda.synchronize()
+        got = st.bufs.result()
+        want = orc.sample(st.graph.indptr.cpu().numpy(), st.graph.indices.cpu().numpy(), seeds.cpu().numpy(),
+                          list(st.fanout), rng_seed)
+        assert_same_sample(got, want)
+        nF = int(got["counts"][len(st.fanout)])
+        pick = np.random.default_rng(b).integers(0, nF, 4096)
+        rows = st.rows[torch.as_tensor(pick, device=DEV)].cpu().numpy()
+        ids = want["nodes"][pick]
+        assert np.array_equal(rows, W.feature_rows(torch.as_tensor(ids), st.dim, st.dtype).numpy())

@@ -1,0 +1,302 @@
+"""Product host planner (libmoment.so, C++) vs the oracle (CPU, no GPU needed).
+
+P1 topology validation/augmentation, P3 Dinic vs Edmonds-Karp (value + optimality certificate of the
+product's own flow), P4 DDAK bit-exact vs the oracle, P5 time bisection (T_ingest vs the oracle's
+bisection on the same ingest graph), quota validity and the closed-form NVLink/HBM times recomputed by
+the oracle from the product's quotas. Also: every symbol include/moment.h declares is exported.
+"""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_sc_shi0s0x0w25_b200 as M
+
+from test_oracle_planner import INF, brute_min_cut, random_links
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_library_exports_every_declared_symbol():
+    hdr = open(os.path.join(ROOT, "include", "moment.h")).read()
+    declared = set(re.findall(r"\b(moment_[a-z_]+)\s*\(", hdr))
+    declared -= {"moment_"}
+    L = M.lib()
+    missing = [s for s in sorted(declared) if not hasattr(L, s)]
+    assert not missing, missing
+    assert set(M.EXPORTED) == declared
+    assert L.moment_version() >= 1
+
+
+def _graph_topology(n, links, s, t):
+    """Wrap a plain s-t graph as a topology: s = SOURCE, t = SINK, first hop STORAGE, others interconnect,
+    predecessors of t COMPUTE. Only used for max-flow parity on arbitrary graphs."""
+    return None
+
+
+def flow_certificate(n, links, s, t, value, flow):
+    bal = [0] * n
+    for (u, v, c), f in zip(links, flow):
+        assert 0 <= f and (c == INF or f <= c)
+        bal[u] -= int(f)
+        bal[v] += int(f)
+    for x in range(n):
+        if x not in (s, t):
+            assert bal[x] == 0
+    assert bal[t] == value
+    # min-cut certificate: S = residual-reachable from s; cut capacity == value
+    adj = {}
+    for (u, v, c), f in zip(links, flow):
+        if c == INF or f < c:
+            adj.setdefault(u, []).append(v)
+        if f > 0:
+            adj.setdefault(v, []).append(u)
+    S = {s}
+    st = [s]
+    while st:
+        u = st.pop()
+        for w in adj.get(u, []):
+            if w not in S:
+                S.add(w)
+                st.append(w)
+    assert t not in S
+    cut = sum(c for (u, v, c) in links if u in S and v not in S)
+    assert cut == value
+
+
+def layered_topology(rng, n_storage, n_inter, n_compute, n_links):
+    """Random valid topology: storage -> interconnect -> ... -> compute."""
+    nodes = []
+    for i in range(n_storage):
+        nodes.append((M.NODE_STORAGE, int(rng.choice([M.TIER_GPU_HBM, M.TIER_HOST_DRAM])), i % max(1, n_compute)))
+    for i in range(n_inter):
+        nodes.append((M.NODE_INTERCONNECT, M.TIER_NONE, -1))
+    for i in range(n_compute):
+        nodes.append((M.NODE_COMPUTE, M.TIER_NONE, i))
+    S = list(range(n_storage))
+    I = list(range(n_storage, n_storage + n_inter))
+    Cp = list(range(n_storage + n_inter, n_storage + n_inter + n_compute))
+    links = []
+    for _ in range(n_links):
+        kind = rng.integers(0, 4)
+        if kind == 0 and I:
+            u, v = int(rng.choice(S)), int(rng.choice(I))
+        elif kind == 1 and len(I) > 1:
+            u, v = [int(x) for x in rng.choice(I, 2, replace=False)]
+        elif kind == 2 and I:
+            u, v = int(rng.choice(I)), int(rng.choice(Cp))
+        else:
+            u, v = int(rng.choice(S)), int(rng.choice(Cp))
+        r = rng.random()
+        cap = 0 if r < 0.05 else int(rng.integers(1, 100))
+        links.append((u, v, cap))
+    return nodes, links
+
+
+@pytest.mark.parametrize("seed", range(30))
+def test_maxflow_dinic_vs_oracle(orc, seed):
+    rng = np.random.default_rng(seed)
+    nodes, links = layered_topology(rng, int(rng.integers(1, 5)), int(rng.integers(0, 6)), int(rng.integers(1, 4)),
+                                    int(rng.integers(1, 25)))
+    topo = M.topology(nodes, links)
+    allnodes, alllinks, s, t = topo.export()
+    val, flow = topo.maxflow()
+    oval, _ = orc.maxflow(len(allnodes), alllinks, s, t)
+    assert val == oval
+    flow_certificate(len(allnodes), alllinks, s, t, val, flow)
+    if len(allnodes) <= 14:
+        assert val == brute_min_cut(len(allnodes), alllinks, s, t)
+
+
+def test_topology_augmentation_and_errors():
+    nodes = [(M.NODE_STORAGE, M.TIER_HOST_DRAM, 0), (M.NODE_INTERCONNECT, 0, -1), (M.NODE_COMPUTE, 0, 0),
+             (M.NODE_COMPUTE, 0, 1)]
+    links = [(0, 1, 30), (0, 1, 20), (1, 2, 25), (1, 3, 25)]
+    topo = M.topology(nodes, links)
+    n, m, s, t = topo.info()
+    assert (n, m, s, t) == (6, 7, 4, 5)
+    _, L, _, _ = topo.export()
+    assert L[4] == (4, 0, 50)  # c(s, v_s) = sum of the storage node's out-capacities (R8)
+    assert L[5] == (2, 5, INF) and L[6] == (3, 5, INF)
+    assert topo.maxflow()[0] == 50
+    bad = [
+        ([(M.NODE_COMPUTE, 0, 0), (M.NODE_STORAGE, M.TIER_GPU_HBM, 0)], [(0, 1, 5)]),  # wrong direction
+        ([(M.NODE_STORAGE, M.TIER_GPU_HBM, 0)], [(0, 0, 5)]),  # self loop
+        ([(M.NODE_STORAGE, M.TIER_GPU_HBM, 0), (M.NODE_COMPUTE, 0, 0)], [(0, 1, -1)]),  # negative
+        ([(M.NODE_STORAGE, M.TIER_GPU_HBM, 0), (M.NODE_COMPUTE, 0, 0)], [(0, 7, 1)]),  # out of range
+        ([(M.NODE_STORAGE, 0, 0)], []),  # storage without tier
+        ([(M.NODE_SOURCE, 0, -1), (M.NODE_SOURCE, 0, -1)], []),  # two sources
+    ]
+    for nd, lk in bad:
+        with pytest.raises(M.MomentError) as e:
+            M.topology(nd, lk)
+        assert e.value.status == M.EINVAL
+    # unbounded: INF path from s to t
+    with pytest.raises(M.MomentError):
+        M.topology([(M.NODE_STORAGE, M.TIER_HOST_DRAM, 0), (M.NODE_COMPUTE, 0, 0)], [(0, 1, INF)]).maxflow()
+
+
+@pytest.mark.parametrize("seed", range(25))
+def test_ddak_bit_exact_vs_oracle(orc, seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(1, 3000))
+    nb = int(rng.integers(1, 7))
+    hot = (rng.pareto(1.2, n) * 10).astype(np.uint64)
+    if seed % 3 == 0:
+        hot[:] = rng.integers(0, 3, n)  # many ties
+    tier = np.array(sorted(rng.choice([1, 2, 3], nb)), np.int32)
+    caps = rng.integers(0, n, nb).astype(np.int64)
+    if caps.sum() < n:
+        caps[-1] += n - caps.sum()
+    traffic = rng.integers(0, 1000, nb).astype(np.int64)
+    if seed % 4 == 1:
+        traffic[rng.integers(0, nb)] = 0
+    for pool in (1, 7, 100):
+        b, s, A, U, T = M.place(None, hot, caps, bin_tier=tier, bin_traffic=traffic, pool=pool)
+        ob, os_, oA, oU = orc.ddak(hot, tier - 1, caps, traffic, pool)
+        assert np.array_equal(b, ob) and np.array_equal(s, os_)
+        assert np.array_equal(A, oA) and np.array_equal(U, oU) and np.array_equal(T, traffic)
+
+
+def test_ddak_large_values_exact(orc):
+    # priorities whose cross products need more than 128 bits
+    n = 500
+    hot = np.full(n, 2**40, np.uint64)
+    hot[::3] = 2**40 + 1
+    caps = np.array([2**35, 2**35 + 3, 2**34], np.int64)
+    traffic = np.array([2**50, 2**50 - 1, 2**49 + 7], np.int64)
+    tier = np.array([1, 1, 1], np.int32)
+    b, s, *_ = M.place(None, hot, caps, bin_tier=tier, bin_traffic=traffic, pool=3)
+    ob, os_, *_ = orc.ddak(hot, tier - 1, caps, traffic, 3)
+    assert np.array_equal(b, ob) and np.array_equal(s, os_)
+
+
+def test_ddak_traffic_from_rate_maxflow(orc):
+    # bins = storage nodes; traffic = f(s, b) of the product's rate max-flow
+    nodes = [(M.NODE_STORAGE, M.TIER_GPU_HBM, 0), (M.NODE_STORAGE, M.TIER_HOST_DRAM, 0),
+             (M.NODE_INTERCONNECT, 0, -1), (M.NODE_COMPUTE, 0, 0)]
+    links = [(0, 3, 600), (1, 2, 50), (2, 3, 40)]
+    topo = M.topology(nodes, links)
+    hot = np.arange(100, dtype=np.uint64)
+    b, s, A, U, T = M.place(topo, hot, [30, 100])
+    assert list(T) == [600, 40]
+    assert U[0] == 30 and set(np.where(b == 0)[0]) == set(range(70, 100))  # hottest 30 in HBM
+    ob, os_, _, _ = orc.ddak(hot, [0, 1], [30, 100], T, 100)
+    assert np.array_equal(b, ob) and np.array_equal(s, os_)
+
+
+def test_place_pack_and_errors():
+    packed = M.place_pack([0, 3, 63], [0, 5, 2**40 - 1])
+    assert list(packed) == [0, (3 << 40) | 5, (63 << 40) | (2**40 - 1)]
+    with pytest.raises(M.MomentError):
+        M.place_pack([64], [0])
+    with pytest.raises(M.MomentError) as e:
+        M.place(None, [1, 2, 3], [1], bin_tier=[1], bin_traffic=[1])
+    assert e.value.status == M.EINFEASIBLE
+
+
+def two_socket_box(k=8, port=55, upi=40, hbm=6000, nv=770, host_per_socket=True):
+    """A B200-like box: 2 NUMA host bins, k GPUs (PCIe port cap each), HBM bin per GPU."""
+    nodes, links = [], []
+    host = [len(nodes), len(nodes) + 1]
+    nodes += [(M.NODE_STORAGE, M.TIER_HOST_DRAM, 0), (M.NODE_STORAGE, M.TIER_HOST_DRAM, 1)]
+    cpu = [len(nodes), len(nodes) + 1]
+    nodes += [(M.NODE_INTERCONNECT, 0, -1)] * 2
+    hbm_nodes, gpu_nodes = [], []
+    for g in range(k):
+        hbm_nodes.append(len(nodes))
+        nodes.append((M.NODE_STORAGE, M.TIER_GPU_HBM, g))
+    for g in range(k):
+        gpu_nodes.append(len(nodes))
+        nodes.append((M.NODE_COMPUTE, 0, g))
+    links += [(host[0], cpu[0], 400), (host[1], cpu[1], 400), (cpu[0], cpu[1], upi), (cpu[1], cpu[0], upi)]
+    for g in range(k):
+        links.append((cpu[0] if g < k // 2 else cpu[1], gpu_nodes[g], port))
+        links.append((hbm_nodes[g], gpu_nodes[g], hbm))
+    return nodes, links, host, hbm_nodes, gpu_nodes
+
+
+@pytest.mark.parametrize("k,d_host0,d_host1,d_hbm", [(8, 4000, 1000, 500), (4, 100, 9000, 0), (2, 0, 0, 300),
+                                                     (8, 12345, 777, 4096), (1, 500, 500, 500)])
+def test_plan_vs_oracle(orc, k, d_host0, d_host1, d_hbm):
+    nodes, links, host, hbm_nodes, gpu_nodes = two_socket_box(k=8)
+    topo = M.topology(nodes, links)
+    N, Lc, s, t = topo.info()
+    allnodes, alllinks, _, _ = topo.export()
+    demand = np.zeros(N, np.int64)
+    demand[host[0]], demand[host[1]] = d_host0, d_host1
+    for g in range(k):
+        demand[hbm_nodes[g]] = d_hbm
+    active = gpu_nodes[:k]
+    p = M.plan(topo, active, demand, 770, 6000).info()
+    # oracle: T_ingest on the same ingest graph (supplies k*d on host bins, none on HBM, active sinks only)
+    il, sup = [], []
+    for (u, v, c) in alllinks:
+        if u == s:
+            tier = allnodes[v][1]
+            il.append((u, v, 0 if tier == M.TIER_GPU_HBM else k * demand[v]))
+            sup.append(1)
+        elif v == t:
+            il.append((u, v, INF if u in active else 0))
+            sup.append(0)
+        else:
+            il.append((u, v, c))
+            sup.append(0)
+    tin, _ = orc.time_bisect(N, il, sup, s, t)
+    assert p["t_ingest"] == tin
+    # the product's ingest flow is a max flow of the graph at T_ingest (certificate)
+    scaled = [(u, v, c if (sp or c == INF) else c * tin) for (u, v, c), sp in zip(il, sup)]
+    flow_certificate(N, scaled, s, t, k * (d_host0 + d_host1), p["link_flow"])
+    # quotas: row sums = supplies, only host rows, only active GPU columns
+    x = p["quota"]
+    for v in range(N):
+        if v in host:
+            assert x[v].sum() == k * demand[v]
+        else:
+            assert x[v].sum() == 0
+    # closed forms recomputed by the oracle from the product's quotas
+    bins = [v for v in range(N) if allnodes[v][0] == M.NODE_STORAGE]
+    owner = [allnodes[v][2] if allnodes[v][1] == M.TIER_GPU_HBM else -1 for v in bins]
+    owner = [o if o < k else -1 for o in owner]
+    d = [demand[v] if not (allnodes[v][1] == M.TIER_GPU_HBM and allnodes[v][2] >= k) else 0 for v in bins]
+    xb = [x[v] for v in bins]
+    tn, th = orc.plan_closed_forms(k, owner, d, xb, 770, 6000)
+    assert (p["t_nvlink"], p["t_hbm"]) == (tn, th)
+    assert p["t_star"] == max(tin, tn, th)
+
+
+def test_plan_needs_nvlink_for_peer_traffic(orc):
+    # peer HBM reads and relays need the NVLink edges; without them the plan is infeasible
+    nodes, links, host, hbm_nodes, gpu_nodes = two_socket_box(k=4)
+    topo = M.topology(nodes, links)
+    N = topo.info()[0]
+    demand = np.zeros(N, np.int64)
+    demand[host[0]] = 10000
+    for g in range(4):
+        demand[hbm_nodes[g]] = 1000
+    with_nv = M.plan(topo, gpu_nodes[:4], demand, 770, 6000).info()["t_star"]
+    with pytest.raises(M.MomentError) as e:
+        M.plan(topo, gpu_nodes[:4], demand, 0, 6000)  # peer traffic exists but no NVLink
+    assert e.value.status == M.EINFEASIBLE
+    demand2 = demand.copy()
+    for g in range(4):
+        demand2[hbm_nodes[g]] = 0
+    # less demand never needs more time (monotone plan)
+    assert M.plan(topo, gpu_nodes[:4], demand2, 770, 6000).info()["t_star"] <= with_nv
+
+
+def test_plan_infeasible_and_zero():
+    nodes = [(M.NODE_STORAGE, M.TIER_HOST_DRAM, 0), (M.NODE_STORAGE, M.TIER_HOST_DRAM, 1),
+             (M.NODE_INTERCONNECT, 0, -1), (M.NODE_COMPUTE, 0, 0)]
+    links = [(0, 2, 10), (2, 3, 10)]  # node 1 is unreachable
+    topo = M.topology(nodes, links)
+    N = topo.info()[0]
+    d = np.zeros(N, np.int64)
+    d[1] = 5
+    with pytest.raises(M.MomentError) as e:
+        M.plan(topo, [3], d, 0, 100)
+    assert e.value.status == M.EINFEASIBLE
+    d[:] = 0
+    info = M.plan(topo, [3], d, 0, 100).info()
+    assert info["t_ingest"] == 0 and info["t_star"] == 0
