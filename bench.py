@@ -87,7 +87,7 @@ class State:
             ev[1].record()
 
     def launches_per_step(self):
-        return 1 + 3 * len(self.fanout) + 1  # init, (sample, bitscan, relabel) per hop, gather
+        return 1 + 3 * len(self.fanout) + 1 + 1  # init, (offsets, sample, bitscan) per hop, finalize, gather
 
 
 def build_state(name, device="cuda:0", rank=0, world=1):
@@ -296,7 +296,7 @@ def main():
     peak, peak_kind = _peaks()
     achieved = alg_bytes / (gather_ms / 1000) / 1e9
     # e2e: the same step through the C ABI with host buffers (seeds H2D, counts D2H, synchronised)
-    seeds_h = [batches[i % len(batches)][0].cpu().pin_memory() for i in range(args.e2e_steps)]
+    seeds_h = [batches[i % len(batches)][0].cpu().pin_memory() for i in range(max(3, args.e2e_steps))]
     counts_h = torch.zeros(2 * H + 1, dtype=torch.int64).pin_memory()
     for i in range(3):
         st.ctx.step_host(st.graph.indptr, st.graph.indices, seeds_h[i], st.fanout, batches[i][1], st.bufs, st.rows,

@@ -60,9 +60,9 @@ inline moment_status cuda_check(cudaError_t e, const char* what) {
 inline moment_status cuda_pending(const char* what) { return cuda_check(cudaPeekAtLastError(), what); }
 
 constexpr int kSampleTile = 256;     // frontier nodes per sampler tile
-constexpr int kBitscanWordsPerThread = 8;
+constexpr int kBitscanWordsPerThread = 4;
 constexpr int kBitscanThreads = 256;
-constexpr int kBitscanTileWords = kBitscanWordsPerThread * kBitscanThreads;  // 2048 words = 65536 ids
+constexpr int kBitscanTileWords = kBitscanWordsPerThread * kBitscanThreads;  // 1024 words = 32768 ids
 constexpr int kBucketTile = 1024;    // requests per bucketing tile
 constexpr int kMaxFanout = 1024;
 

@@ -66,6 +66,88 @@ __device__ __forceinline__ int64_t block_exclusive_scan(int64_t x, int64_t* tota
 // in increasing order through an atomic ticket, so every predecessor tile is owned by a running block.
 constexpr uint64_t kFlagAgg = 1ull << 62, kFlagPrefix = 2ull << 62, kValMask = (1ull << 62) - 1;
 
+__device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p) {
+    return cuda::atomic_ref<unsigned long long, cuda::thread_scope_device>(
+               *reinterpret_cast<unsigned long long*>(const_cast<uint64_t*>(p)))
+        .load(cuda::memory_order_acquire);
+}
+__device__ __forceinline__ void st_release(uint64_t* p, uint64_t v) {
+    cuda::atomic_ref<unsigned long long, cuda::thread_scope_device>(*reinterpret_cast<unsigned long long*>(p))
+        .store(v, cuda::memory_order_release);
+}
+
+// Warp-parallel decoupled look-back: called by ALL 32 lanes of one warp; inspects 32 predecessors per
+// step (lane 0 = nearest), stops at the nearest inclusive prefix. Returns the exclusive prefix (all lanes).
+__device__ __forceinline__ int64_t lookback_warp(uint64_t* status, int64_t tile, int64_t aggregate) {
+    const int lane = threadIdx.x & 31;
+    if (tile == 0) {
+        if (lane == 0) st_release(&status[0], kFlagPrefix | (uint64_t)aggregate);
+        return 0;
+    }
+    if (lane == 0) st_release(&status[tile], kFlagAgg | (uint64_t)aggregate);
+    int64_t exclusive = 0;
+    for (int64_t end = tile - 1;; end -= 32) {
+        const int64_t j = end - lane;
+        uint64_t s = kFlagPrefix;  // "before tile 0" acts as a zero prefix (never reached: tile 0 is a prefix)
+        if (j >= 0) {
+            do {
+                s = ld_acquire(&status[j]);
+            } while ((s & ~kValMask) == 0);
+        }
+        const unsigned pre = __ballot_sync(0xffffffffu, (s & ~kValMask) == kFlagPrefix);
+        const int stop = pre ? __ffs(pre) - 1 : 32;
+        int64_t v = (lane <= stop && j >= 0) ? (int64_t)(s & kValMask) : 0;
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
+        exclusive += v;
+        if (pre) break;
+    }
+    if (lane == 0) st_release(&status[tile], kFlagPrefix | (uint64_t)(exclusive + aggregate));
+    return exclusive;
+}
+
+// Block-wide decoupled look-back: ALL NT threads call it; each step inspects NT predecessors at once
+// (thread 0 = nearest), waits until each has published, and stops at the nearest inclusive prefix.
+// Returns the exclusive prefix to every thread. `red` is NT/32 int64 of shared scratch, `flag` one int.
+template <int NT>
+__device__ __forceinline__ int64_t lookback_block(uint64_t* status, int64_t tile, int64_t aggregate, int64_t* red,
+                                                  int* nearest) {
+    if (tile == 0) {
+        if (threadIdx.x == 0) st_release(&status[0], kFlagPrefix | (uint64_t)aggregate);
+        return 0;
+    }
+    if (threadIdx.x == 0) st_release(&status[tile], kFlagAgg | (uint64_t)aggregate);
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    int64_t exclusive = 0;
+    for (int64_t end = tile - 1;; end -= NT) {
+        const int64_t j = end - threadIdx.x;
+        uint64_t s = 0;
+        if (j >= 0) {
+            do {
+                s = ld_acquire(&status[j]);
+            } while ((s & ~kValMask) == 0);
+        }
+        if (threadIdx.x == 0) *nearest = NT;
+        __syncthreads();
+        if (j >= 0 && (s & ~kValMask) == kFlagPrefix) atomicMin(nearest, (int)threadIdx.x);
+        __syncthreads();
+        const int stop = *nearest;
+        int64_t v = (j >= 0 && (int)threadIdx.x <= stop) ? (int64_t)(s & kValMask) : 0;
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
+        if (lane == 0) red[wid] = v;
+        __syncthreads();
+        int64_t sum = 0;
+#pragma unroll
+        for (int w = 0; w < NT / 32; w++) sum += red[w];
+        exclusive += sum;
+        __syncthreads();
+        if (stop < NT || end - NT < 0) break;
+    }
+    if (threadIdx.x == 0) st_release(&status[tile], kFlagPrefix | (uint64_t)(exclusive + aggregate));
+    return exclusive;
+}
+
 __device__ __forceinline__ int64_t lookback(uint64_t* status, int64_t tile, int64_t aggregate) {
     using ref = cuda::atomic_ref<unsigned long long, cuda::thread_scope_device>;
     if (tile == 0) {

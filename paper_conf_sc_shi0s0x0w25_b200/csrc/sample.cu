@@ -1,13 +1,15 @@
 // sample.cu — H1-H3: multi-hop neighbour sampling with dedup/relabel on sm_100a (R3-R6).
 //
-// Per hop h the path is three kernels, none of which needs the host to know |F_h| or E_h (every size is
-// read from device memory, so the whole sample call is CUDA-graph capturable):
-//   sample_hop  : tile of 256 frontier nodes -> degrees -> block scan + decoupled look-back = edge offsets;
-//                 then one G-lane group per node draws its Floyd / with-replacement positions from
-//                 Philox, writes the neighbour ids and marks them in the `newbits` bitmap.
-//   bitscan     : F_{h+1} = F_h ++ (newbits & ~visited) in ascending id order: a chained scan of bitmap
-//                 popcounts (2048 words per tile) gives each new id its position; lidx[id] = position.
-//   relabel     : src[e] = lidx[src[e]] (global id -> index in F_{h+1}).
+// One sample call is 3H + 2 kernels and no memsets; no kernel needs the host to know |F_h| or E_h (every
+// size is read from device memory), so the call is CUDA-graph capturable:
+//   init        : F_0 = seeds; lidx / visited of the seeds; zero the tile descriptors and tickets.
+//   offsets (h) : tile of 256 frontier nodes -> degrees -> block scan + block-wide decoupled look-back =
+//                 edge offsets. Blocks without a tile relabel hop h-1's edges (src = lidx[id]).
+//   sample (h)  : one G-lane group per frontier node draws its Floyd / with-replacement positions from
+//                 Philox (choices resolved in parallel), writes the neighbour ids, marks them in `newbits`.
+//   bitscan (h) : F_{h+1} = F_h ++ (newbits & ~visited) in ascending id order: chained scan of bitmap
+//                 popcounts (1024 words per tile) gives each new id its position; lidx[id] = position.
+//   finalize    : relabel the last hop's edges, then clear the `visited` words of F_H (next call starts clean).
 #include <cooperative_groups.h>
 
 #include <algorithm>
@@ -20,6 +22,10 @@ namespace cg = cooperative_groups;
 namespace moment {
 namespace {
 
+constexpr int kScanWords = kBitscanWordsPerThread;  // bitmap words per bitscan thread (4: one uint4)
+constexpr int kScanTileWords = kBitscanTileWords;   // 1024 words = 32768 ids per tile
+static_assert(kScanWords == 4, "bitscan loads one uint4 per thread");
+
 struct HopArgs {
     const int64_t* indptr;
     const int32_t* indices;
@@ -28,6 +34,7 @@ struct HopArgs {
     int32_t* src;
     int64_t* counts;
     uint32_t* newbits;
+    const int32_t* lidx;
     uint64_t* tile_status;
     uint32_t* ticket;
     uint64_t seed;
@@ -53,58 +60,50 @@ __device__ __forceinline__ void mark_new(uint32_t* newbits, int32_t u) {
     if ((__ldcg(w) & bit) == 0) atomicOr(w, bit);
 }
 
-// One node, one group of G lanes. Positions are distinct CSR offsets in [0, d).
+// src[e] = lidx[src[e]] for the E edges of hop `hr` (grid-stride over `nthreads` participants).
+__device__ __forceinline__ void relabel_hop(int32_t* src_all, const int64_t* counts, const int32_t* lidx, int hr, int H,
+                                            int64_t tid, int64_t nthreads) {
+    int64_t ob, eb;
+    hop_bases(counts, hr, H, &ob, &eb);
+    const int64_t E = counts[H + 1 + hr];
+    int32_t* src = src_all + eb;
+    for (int64_t e = tid; e < E; e += nthreads) src[e] = __ldg(lidx + src[e]);
+}
+
+// Floyd's k choices for node v at hop h, lane i < k owning choice i (k <= G): t_i = uniform(draw(i),
+// j_i + 1), j_i = d - k + i, and c_i = j_i if t_i is already in S_{i-1} = {c_0..c_{i-1}}, else t_i.
+// Resolved without the k-step sequential chain: t_i is in S_{i-1} iff (a) some earlier t_l equals t_i
+// (if t_l was itself a duplicate it was already in S) or (b) t_i = j_l for an earlier l whose choice was
+// j_l. (a) is one match_any; (b) refers only to earlier lanes, so a fixpoint over ballots converges.
 template <int G>
-__device__ __forceinline__ void sample_node(const cg::thread_block_tile<G>& grp, const HopArgs& a, int64_t v,
-                                            int64_t lo, int32_t d, int32_t* out) {
+__device__ __forceinline__ int32_t floyd_choice(const cg::thread_block_tile<G>& grp, uint64_t seed, int64_t v, int h,
+                                                int32_t d, int k) {
+    const int lane = grp.thread_rank();
+    const bool active = lane < k;
+    const int32_t jj = d - k + lane;
+    const int32_t t = active ? (int32_t)dev::uniform(dev::draw(seed, v, h, lane), (uint32_t)(jj + 1)) : -1 - lane;
+    const unsigned below = (1u << lane) - 1u;
+    const unsigned same = grp.match_any(t);
+    const bool dup_a = active && (same & below) != 0;
+    const int lstar = t - (d - k);  // the earlier lane whose j equals t, if any
+    const bool ref = active && !dup_a && t >= d - k && lstar < lane;
+    unsigned dup = grp.ballot(dup_a);
+    for (;;) {
+        const bool now = dup_a || (ref && ((dup >> lstar) & 1u));
+        const unsigned nd = grp.ballot(now);
+        if (nd == dup) break;
+        dup = nd;
+    }
+    return ((dup >> lane) & 1u) ? jj : t;
+}
+
+// Positions for k > G (G == 32 only): chunks of 32 choices resolved in draw order; earlier chunks are
+// final and kept (as positions) in `out`, then sorted and replaced by ids. Rare (fanout > 32).
+__device__ void sample_node_wide(const cg::thread_block_tile<32>& grp, const HopArgs& a, int64_t v, int64_t lo,
+                                 int32_t d, int32_t* out) {
     const int lane = grp.thread_rank();
     const int k = a.k;
-    if (d <= 0) return;
-    if (a.replace) {
-        // with replacement: k draws in draw order
-        for (int i = lane; i < k; i += G) {
-            const uint32_t p = dev::uniform(dev::draw(a.seed, v, a.h, i), (uint32_t)d);
-            const int32_t u = __ldg(a.indices + lo + p);
-            out[i] = u;
-            mark_new(a.newbits, u);
-        }
-        return;
-    }
-    if (d <= k) {
-        // take all neighbours, CSR order, no draws
-        for (int p = lane; p < d; p += G) {
-            const int32_t u = __ldg(a.indices + lo + p);
-            out[p] = u;
-            mark_new(a.newbits, u);
-        }
-        return;
-    }
-    if (k <= G) {
-        // Floyd F2 with the k choices resolved in draw order by group ballots; lane i owns choice i.
-        int32_t j = 0, t = 0, c = -1;
-        if (lane < k) {
-            j = d - k + lane;
-            t = (int32_t)dev::uniform(dev::draw(a.seed, v, a.h, lane), (uint32_t)(j + 1));
-        }
-        for (int m = 0; m < k; m++) {
-            const int32_t tm = grp.shfl(t, m);
-            const bool hit = lane < m && c == tm;
-            const unsigned any = grp.ballot(hit);
-            if (lane == m) c = any ? j : t;
-        }
-        // rank of c among the k distinct choices = its position in sorted order
-        int r = 0;
-        for (int l = 0; l < k; l++) r += grp.shfl(c, l) < c;
-        if (lane < k) {
-            const int32_t u = __ldg(a.indices + lo + c);
-            out[r] = u;
-            mark_new(a.newbits, u);
-        }
-        return;
-    }
-    // k > G (only G == 32 reaches here): chunks of 32 choices; earlier chunks are final and kept in
-    // `out` as positions, then replaced by ids after the sort.
-    for (int c0 = 0; c0 < k; c0 += G) {
+    for (int c0 = 0; c0 < k; c0 += 32) {
         const int i = c0 + lane;
         int32_t j = 0, t = 0, c = -1;
         bool prev_hit = false;
@@ -113,23 +112,21 @@ __device__ __forceinline__ void sample_node(const cg::thread_block_tile<G>& grp,
             t = (int32_t)dev::uniform(dev::draw(a.seed, v, a.h, i), (uint32_t)(j + 1));
             for (int q = 0; q < c0; q++) prev_hit |= out[q] == t;
         }
-        const int nm = min(G, k - c0);
+        const int nm = min(32, k - c0);
         for (int m = 0; m < nm; m++) {
             const int32_t tm = grp.shfl(t, m);
-            const bool hit = lane < m && c == tm;
-            const unsigned any = grp.ballot(hit);
+            const unsigned any = grp.ballot(lane < m && c == tm);
             if (lane == m) c = (any || prev_hit) ? j : t;
         }
         grp.sync();
         if (i < k) out[i] = c;
         grp.sync();
     }
-    // sort positions: rank by counting (distinct), then write ids
     int32_t mine[kMaxFanout / 32];
     int rk[kMaxFanout / 32];
-    const int per = (k + G - 1) / G;
+    const int per = (k + 31) / 32;
     for (int q = 0; q < per; q++) {
-        const int i = q * G + lane;
+        const int i = q * 32 + lane;
         mine[q] = i < k ? out[i] : 0;
         int r = 0;
         if (i < k)
@@ -138,7 +135,7 @@ __device__ __forceinline__ void sample_node(const cg::thread_block_tile<G>& grp,
     }
     grp.sync();
     for (int q = 0; q < per; q++) {
-        const int i = q * G + lane;
+        const int i = q * 32 + lane;
         if (i < k) {
             const int32_t u = __ldg(a.indices + lo + mine[q]);
             out[rk[q]] = u;
@@ -147,47 +144,37 @@ __device__ __forceinline__ void sample_node(const cg::thread_block_tile<G>& grp,
     }
 }
 
-template <int G>
-__global__ void __launch_bounds__(kSampleTile) sample_hop_kernel(HopArgs a) {
-    __shared__ int64_t s_v[kSampleTile], s_lo[kSampleTile], s_off[kSampleTile];
-    __shared__ int32_t s_deg[kSampleTile];
-    __shared__ int64_t s_warp[kSampleTile / 32];
-    __shared__ int64_t s_prefix;
+// Pass A of hop h: edge offsets. count(v) = min(deg v, k) (k if REPLACE and deg > 0); tile of 256 nodes
+// -> block scan -> block-wide decoupled look-back. Writes offsets[F] and E_h = counts[H+1+h]. Blocks
+// without (further) tiles relabel hop h-1's edges (its lidx is final once bitscan h-1 has run).
+__global__ void __launch_bounds__(kSampleTile) hop_offsets_kernel(HopArgs a) {
+    __shared__ int64_t s_red[kSampleTile / 32];
     __shared__ uint32_t s_tile;
+    __shared__ int s_nearest;
     const int64_t F = a.counts[a.h];
     int64_t off_base, edge_base;
     hop_bases(a.counts, a.h, a.H, &off_base, &edge_base);
     int64_t* offsets = a.offsets + off_base;
-    int32_t* src = a.src + edge_base;
-    const int64_t n_tiles = (F + kSampleTile - 1) / kSampleTile;
-    if (F == 0) {
-        if (blockIdx.x == 0 && threadIdx.x == 0) {
-            offsets[0] = 0;
-            a.counts[a.H + 1 + a.h] = 0;
-        }
-        return;
+    if (F == 0 && blockIdx.x == 0 && threadIdx.x == 0) {
+        offsets[0] = 0;
+        a.counts[a.H + 1 + a.h] = 0;
     }
-    auto grp = cg::tiled_partition<G>(cg::this_thread_block());
-    const int group = threadIdx.x / G, n_groups = kSampleTile / G;
+    const int64_t n_tiles = (F + kSampleTile - 1) / kSampleTile;
     for (;;) {
         if (threadIdx.x == 0) s_tile = atomicAdd(a.ticket, 1u);
         __syncthreads();
         const int64_t tile = s_tile;
         if (tile >= n_tiles) break;
         const int64_t idx = tile * kSampleTile + threadIdx.x;
-        int64_t v = 0, lo = 0;
-        int32_t d = 0, c = 0;
+        int32_t c = 0;
         if (idx < F) {
-            v = a.nodes[idx];
-            lo = __ldg(a.indptr + v);
-            d = (int32_t)(__ldg(a.indptr + v + 1) - lo);
-            c = a.replace ? (d > 0 ? a.k : 0) : min(d, a.k);
+            const int64_t v = a.nodes[idx];
+            const int64_t d = __ldg(a.indptr + v + 1) - __ldg(a.indptr + v);
+            c = a.replace ? (d > 0 ? a.k : 0) : (int32_t)min(d, (int64_t)a.k);
         }
         int64_t agg;
-        const int64_t excl = dev::block_exclusive_scan<kSampleTile>(c, &agg, s_warp);
-        if (threadIdx.x == 0) s_prefix = dev::lookback(a.tile_status, tile, agg);
-        __syncthreads();
-        const int64_t off = s_prefix + excl;
+        const int64_t excl = dev::block_exclusive_scan<kSampleTile>(c, &agg, s_red);
+        const int64_t off = dev::lookback_block<kSampleTile>(a.tile_status, tile, agg, s_red, &s_nearest) + excl;
         if (idx < F) {
             offsets[idx] = off;
             if (idx == F - 1) {
@@ -195,14 +182,59 @@ __global__ void __launch_bounds__(kSampleTile) sample_hop_kernel(HopArgs a) {
                 a.counts[a.H + 1 + a.h] = off + c;
             }
         }
-        s_v[threadIdx.x] = v;
-        s_lo[threadIdx.x] = lo;
-        s_deg[threadIdx.x] = d;
-        s_off[threadIdx.x] = off;
         __syncthreads();
-        const int live = (int)min((int64_t)kSampleTile, F - tile * kSampleTile);
-        for (int j = group; j < live; j += n_groups) sample_node<G>(grp, a, s_v[j], s_lo[j], s_deg[j], src + s_off[j]);
-        __syncthreads();
+    }
+    if (a.h > 0)
+        relabel_hop(a.src, a.counts, a.lidx, a.h - 1, a.H, (int64_t)blockIdx.x * kSampleTile + threadIdx.x,
+                    (int64_t)gridDim.x * kSampleTile);
+}
+
+// Pass B of hop h: one G-lane group per frontier node (grid-stride), every node in flight at once.
+template <int G>
+__global__ void __launch_bounds__(256) hop_sample_kernel(HopArgs a) {
+    const int64_t F = a.counts[a.h];
+    int64_t off_base, edge_base;
+    hop_bases(a.counts, a.h, a.H, &off_base, &edge_base);
+    const int64_t* offsets = a.offsets + off_base;
+    int32_t* src = a.src + edge_base;
+    auto grp = cg::tiled_partition<G>(cg::this_thread_block());
+    const int lane = grp.thread_rank();
+    const int k = a.k;
+    const int64_t groups = (int64_t)gridDim.x * (256 / G);
+    for (int64_t idx = (int64_t)blockIdx.x * (256 / G) + threadIdx.x / G; idx < F; idx += groups) {
+        const int64_t v = a.nodes[idx];
+        const int64_t lo = __ldg(a.indptr + v);
+        const int32_t d = (int32_t)(__ldg(a.indptr + v + 1) - lo);
+        int32_t* out = src + offsets[idx];
+        if (d <= 0) continue;
+        if (a.replace) {  // k draws, draw order
+            for (int i = lane; i < k; i += G) {
+                const int32_t u = __ldg(a.indices + lo + dev::uniform(dev::draw(a.seed, v, a.h, i), (uint32_t)d));
+                out[i] = u;
+                mark_new(a.newbits, u);
+            }
+        } else if (d <= k) {  // all neighbours, CSR order, no draws
+            for (int p = lane; p < d; p += G) {
+                const int32_t u = __ldg(a.indices + lo + p);
+                out[p] = u;
+                mark_new(a.newbits, u);
+            }
+        } else if (k <= G) {  // Floyd, one choice per lane, then rank = position in sorted order
+            const int32_t c = floyd_choice<G>(grp, a.seed, v, a.h, d, k);
+            int r = 0;
+#pragma unroll
+            for (int l = 0; l < G; l++) {
+                const int32_t cl = grp.shfl(c, l);
+                r += (l < k) && cl < c;
+            }
+            if (lane < k) {
+                const int32_t u = __ldg(a.indices + lo + c);
+                out[r] = u;
+                mark_new(a.newbits, u);
+            }
+        } else {
+            if constexpr (G == 32) sample_node_wide(grp, a, v, lo, d, out);
+        }
     }
 }
 
@@ -220,47 +252,41 @@ struct ScanArgs {
 
 // F_{h+1} = F_h ++ ascending ids set in (newbits & ~visited).
 __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
-    __shared__ int64_t s_warp[kBitscanThreads / 32];
-    __shared__ int64_t s_prefix;
+    __shared__ int64_t s_red[kBitscanThreads / 32];
     __shared__ uint32_t s_tile;
+    __shared__ int s_nearest;
     const int64_t F = a.counts[a.h];
-    const int64_t n_tiles = (a.n_words + kBitscanTileWords - 1) / kBitscanTileWords;
+    const int64_t n_tiles = (a.n_words + kScanTileWords - 1) / kScanTileWords;
     for (;;) {
         if (threadIdx.x == 0) s_tile = atomicAdd(a.ticket, 1u);
         __syncthreads();
         const int64_t tile = s_tile;
         if (tile >= n_tiles) break;
-        const int64_t w0 = tile * kBitscanTileWords + (int64_t)threadIdx.x * kBitscanWordsPerThread;
-        uint32_t nb[kBitscanWordsPerThread], nw[kBitscanWordsPerThread];
+        const int64_t w0 = tile * kScanTileWords + (int64_t)threadIdx.x * kScanWords;
+        uint32_t nb[kScanWords], nw[kScanWords];
         int cnt = 0;
-        if (w0 + kBitscanWordsPerThread <= a.n_words) {
-            const uint4* pn = reinterpret_cast<const uint4*>(a.newbits + w0);
-            const uint4* pv = reinterpret_cast<const uint4*>(a.visited + w0);
-            uint4 n0 = __ldcg(pn), n1 = __ldcg(pn + 1), v0 = __ldcg(pv), v1 = __ldcg(pv + 1);
-            nb[0] = n0.x; nb[1] = n0.y; nb[2] = n0.z; nb[3] = n0.w; nb[4] = n1.x; nb[5] = n1.y; nb[6] = n1.z; nb[7] = n1.w;
-            uint32_t vv[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
-#pragma unroll
-            for (int q = 0; q < 8; q++) {
-                nw[q] = nb[q] & ~vv[q];
-                cnt += __popc(nw[q]);
-            }
+        if (w0 + kScanWords <= a.n_words) {
+            const uint4 n4 = __ldcg(reinterpret_cast<const uint4*>(a.newbits + w0));
+            const uint4 v4 = __ldcg(reinterpret_cast<const uint4*>(a.visited + w0));
+            nb[0] = n4.x; nb[1] = n4.y; nb[2] = n4.z; nb[3] = n4.w;
+            nw[0] = n4.x & ~v4.x; nw[1] = n4.y & ~v4.y; nw[2] = n4.z & ~v4.z; nw[3] = n4.w & ~v4.w;
         } else {
 #pragma unroll
-            for (int q = 0; q < 8; q++) {
+            for (int q = 0; q < kScanWords; q++) {
                 const int64_t w = w0 + q;
                 nb[q] = w < a.n_words ? __ldcg(a.newbits + w) : 0u;
                 nw[q] = w < a.n_words ? nb[q] & ~__ldcg(a.visited + w) : 0u;
-                cnt += __popc(nw[q]);
             }
         }
-        int64_t agg;
-        const int64_t excl = dev::block_exclusive_scan<kBitscanThreads>(cnt, &agg, s_warp);
-        if (threadIdx.x == 0) s_prefix = dev::lookback(a.tile_status, tile, agg);
-        __syncthreads();
-        int64_t pos = F + s_prefix + excl;
-        if (tile == n_tiles - 1 && threadIdx.x == 0) a.counts[a.h + 1] = F + s_prefix + agg;
 #pragma unroll
-        for (int q = 0; q < 8; q++) {
+        for (int q = 0; q < kScanWords; q++) cnt += __popc(nw[q]);
+        int64_t agg;
+        const int64_t excl = dev::block_exclusive_scan<kBitscanThreads>(cnt, &agg, s_red);
+        const int64_t prefix = dev::lookback_block<kBitscanThreads>(a.tile_status, tile, agg, s_red, &s_nearest);
+        int64_t pos = F + prefix + excl;
+        if (tile == n_tiles - 1 && threadIdx.x == 0) a.counts[a.h + 1] = F + prefix + agg;
+#pragma unroll
+        for (int q = 0; q < kScanWords; q++) {
             const int64_t w = w0 + q;
             uint32_t bits = nw[q];
             while (bits) {
@@ -280,19 +306,22 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
     }
 }
 
-__global__ void relabel_kernel(int32_t* src_all, const int64_t* counts, const int32_t* lidx, int h, int H) {
-    int64_t off_base, edge_base;
-    hop_bases(counts, h, H, &off_base, &edge_base);
-    const int64_t E = counts[H + 1 + h];
-    int32_t* src = src_all + edge_base;
-    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < E; e += (int64_t)gridDim.x * blockDim.x)
-        src[e] = __ldg(lidx + src[e]);
+// Relabel the last hop's edges; clear the visited words of every node of F_H.
+__global__ void finalize_kernel(int32_t* src_all, const int64_t* counts, const int32_t* lidx, const int64_t* nodes,
+                                uint32_t* visited, int H) {
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (int64_t)gridDim.x * blockDim.x;
+    if (H > 0) relabel_hop(src_all, counts, lidx, H - 1, H, tid, nth);
+    const int64_t FH = counts[H];
+    for (int64_t i = tid; i < FH; i += nth) visited[nodes[i] >> 5] = 0u;
 }
 
-__global__ void init_seeds_kernel(const int64_t* seeds, int64_t n_seeds, int64_t n_vertices, int64_t* nodes,
-                                  int32_t* lidx, uint32_t* visited, int64_t* counts, uint32_t* error_flag,
-                                  int check) {
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_seeds; i += (int64_t)gridDim.x * blockDim.x) {
+__global__ void init_kernel(const int64_t* seeds, int64_t n_seeds, int64_t n_vertices, int64_t* nodes, int32_t* lidx,
+                            uint32_t* visited, int64_t* counts, uint32_t* error_flag, int check, uint64_t* tile_status,
+                            int64_t n_tile_status, uint32_t* tickets, int n_tickets) {
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = tid; i < n_tile_status; i += nth) tile_status[i] = 0;
+    for (int64_t i = tid; i < n_tickets; i += nth) tickets[i] = 0;
+    for (int64_t i = tid; i < n_seeds; i += nth) {
         const int64_t v = seeds[i];
         if (v < 0 || v >= n_vertices) {  // never write out of range, checked or not
             atomicOr(error_flag, 1u);
@@ -305,14 +334,16 @@ __global__ void init_seeds_kernel(const int64_t* seeds, int64_t n_seeds, int64_t
         const uint32_t old = atomicOr(visited + (v >> 5), bit);
         if (check && (old & bit)) atomicOr(error_flag, 2u);
     }
-    if (blockIdx.x == 0 && threadIdx.x == 0) counts[0] = n_seeds;
+    if (tid == 0) counts[0] = n_seeds;
 }
 
 template <int G>
-void launch_hop(const HopArgs& a, int64_t max_F, cudaStream_t stream) {
+void launch_hop(const HopArgs& a, int64_t max_F, int64_t prev_E, cudaStream_t stream) {
     const int64_t tiles = std::max<int64_t>(1, (max_F + kSampleTile - 1) / kSampleTile);
-    const int grid = (int)std::min<int64_t>(tiles, 148 * 8);
-    sample_hop_kernel<G><<<grid, kSampleTile, 0, stream>>>(a);
+    const int64_t relabel_blocks = (prev_E + kSampleTile * 4 - 1) / (kSampleTile * 4);
+    hop_offsets_kernel<<<(int)std::min<int64_t>(std::max(tiles, relabel_blocks), 148 * 4), kSampleTile, 0, stream>>>(a);
+    const int64_t blocks = std::max<int64_t>(1, (max_F * G + 255) / 256);
+    hop_sample_kernel<G><<<(int)std::min<int64_t>(blocks, 148 * 16), 256, 0, stream>>>(a);
 }
 
 }  // namespace
@@ -342,32 +373,33 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const int6
     MOMENT_TRY(cuda_pending("moment_sample: pending CUDA error"));
     const int check = (p->flags & MOMENT_SAMPLE_CHECK) ? 1 : 0;
     const int replace = (p->flags & MOMENT_SAMPLE_REPLACE) ? 1 : 0;
-    MOMENT_TRY(cuda_check(cudaMemsetAsync(ctx->visited, 0, ctx->n_words * sizeof(uint32_t), stream), "memset visited"));
-    MOMENT_TRY(cuda_check(cudaMemsetAsync(ctx->tile_status, 0, ctx->n_tile_status * sizeof(uint64_t), stream), "memset tiles"));
-    MOMENT_TRY(cuda_check(cudaMemsetAsync(ctx->tickets, 0, 2 * std::max(1, ctx->max_hops) * sizeof(uint32_t), stream), "memset tickets"));
     {
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n_seeds + 255) / 256, 148 * 4));
-        init_seeds_kernel<<<grid, 256, 0, stream>>>(seeds, n_seeds, ctx->n_vertices, out->nodes, ctx->lidx, ctx->visited,
-                                                    out->counts, ctx->error_flag, check);
+        init_kernel<<<grid, 256, 0, stream>>>(seeds, n_seeds, ctx->n_vertices, out->nodes, ctx->lidx, ctx->visited,
+                                              out->counts, ctx->error_flag, check, ctx->tile_status, ctx->n_tile_status,
+                                              ctx->tickets, 2 * std::max(1, ctx->max_hops));
     }
     // per-call bounds on |F_h| for launch sizing (the kernels read the true sizes from counts)
-    int64_t F_bound = n_seeds;
+    int64_t F_bound = n_seeds, E_prev = 0;
+    const int64_t n_scan_tiles = (ctx->n_words + kScanTileWords - 1) / kScanTileWords;
     for (int h = 0; h < H; h++) {
-        HopArgs a{csr->indptr, csr->indices, out->nodes, out->offsets, out->src, out->counts, ctx->newbits,
-                  ctx->tile_status + ctx->sample_tiles_off[h], ctx->tickets + 2 * h, p->rng_seed, h, H, p->fanout[h], replace};
         const int k = p->fanout[h];
-        if (k <= 4) launch_hop<4>(a, F_bound, stream);
-        else if (k <= 8) launch_hop<8>(a, F_bound, stream);
-        else if (k <= 16) launch_hop<16>(a, F_bound, stream);
-        else launch_hop<32>(a, F_bound, stream);
+        HopArgs a{csr->indptr, csr->indices, out->nodes, out->offsets, out->src, out->counts, ctx->newbits, ctx->lidx,
+                  ctx->tile_status + ctx->sample_tiles_off[h], ctx->tickets + 2 * h, p->rng_seed, h, H, k, replace};
+        if (k <= 4) launch_hop<4>(a, F_bound, E_prev, stream);
+        else if (k <= 8) launch_hop<8>(a, F_bound, E_prev, stream);
+        else if (k <= 16) launch_hop<16>(a, F_bound, E_prev, stream);
+        else launch_hop<32>(a, F_bound, E_prev, stream);
         ScanArgs s{out->nodes, out->counts, ctx->lidx, ctx->newbits, ctx->visited,
                    ctx->tile_status + ctx->bitscan_tiles_off[h], ctx->tickets + 2 * h + 1, ctx->n_words, h};
-        const int64_t tiles = (ctx->n_words + kBitscanTileWords - 1) / kBitscanTileWords;
-        bitscan_kernel<<<(int)std::min<int64_t>(tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
-        const int64_t E_bound = F_bound * (int64_t)k;
-        const int rgrid = (int)std::max<int64_t>(1, std::min<int64_t>((E_bound + 255) / 256, 148 * 8));
-        relabel_kernel<<<rgrid, 256, 0, stream>>>(out->src, out->counts, ctx->lidx, h, H);
+        bitscan_kernel<<<(int)std::min<int64_t>(n_scan_tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
+        E_prev = F_bound * (int64_t)k;
         F_bound = std::min(F_bound + F_bound * (int64_t)k, ctx->n_vertices);
+    }
+    {
+        const int64_t work = std::max(E_prev, F_bound);
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((work + 1023) / 1024, 148 * 8));
+        finalize_kernel<<<grid, 256, 0, stream>>>(out->src, out->counts, ctx->lidx, out->nodes, ctx->visited, H);
     }
     return cuda_check(cudaGetLastError(), "moment_sample: launch");
 }

@@ -1,7 +1,7 @@
 #!/bin/bash
 # Launch list of a short bench run (cold-cache, serialised per-launch times; compare SHARES only).
-set -e
 OUT=${1:-gpurun_out/launches.csv}
-ncu --metrics gpu__time_duration.sum --clock-control none -c 200 --csv --log-file "$OUT" \
-    python bench.py --steps 6 --warmup 3 --no-cpu-baseline --e2e-steps 1 > /dev/null 2>&1 || true
+CFG=${2:-C2}
+ncu --metrics gpu__time_duration.sum --clock-control none -k "regex:hop_|bitscan|finalize|init_kernel|gather_kernel|bucket_|queue_|relay_|hotness" -c 300 --csv --log-file "$OUT" \
+    python bench.py --config "$CFG" --steps 10 --warmup 3 --no-cpu-baseline --e2e-steps 1 > /dev/null 2>&1 || true
 python tools/summarize_launches.py "$OUT"
