@@ -42,10 +42,23 @@ def _peaks():
         return 6650.0, "fallback"
 
 
-class State:
-    """Resident inputs and buffers of one rank for one config (the bench and the full-size parity test)."""
+class Lane:
+    """One batch in flight: its own device context (workspace), sample buffers, row buffer and stream."""
 
-    def __init__(self, name, device, rank, world):
+    def __init__(self, M, cfg, fanout, B, R, rank, world, device, table, stream):
+        self.ctx = M.Ctx(n_vertices=cfg["n"], max_seeds=B, max_fanout=fanout, rank=rank, world=world,
+                         device=torch.device(device).index or 0, row_bytes=R, bin_owner=[rank],
+                         bin_ptr=[table.data_ptr()])
+        self.bufs = M.SampleBuffers.allocate(B, fanout, cfg["n"], device)
+        self.rows = torch.empty((self.bufs.nodes.numel(), R), dtype=torch.uint8, device=device)
+        self.stream = stream
+
+
+class State:
+    """Resident inputs of one rank for one config and `inflight` lanes (the bench and the full-size parity
+    test). Every lane shares the replicated graph and feature table (C2: all features in HBM)."""
+
+    def __init__(self, name, device, rank, world, inflight=1):
         import paper_conf_sc_shi0s0x0w25_b200 as M
 
         self.M = M
@@ -59,11 +72,9 @@ class State:
         self.table = W.feature_table(cfg["n"], self.dim, self.dtype, device=device)  # replicated, all in HBM
         self.R = self.table.shape[1]
         self.train = W.training_set(self.graph, min_count=self.B * world)
-        self.ctx = M.Ctx(n_vertices=cfg["n"], max_seeds=self.B, max_fanout=self.fanout, rank=rank, world=world,
-                         device=torch.device(device).index or 0, row_bytes=self.R, bin_owner=[rank],
-                         bin_ptr=[self.table.data_ptr()])
-        self.bufs = M.SampleBuffers.allocate(self.B, self.fanout, cfg["n"], device)
-        self.rows = torch.empty((self.bufs.nodes.numel(), self.R), dtype=torch.uint8, device=device)
+        streams = [torch.cuda.current_stream(device)] + [torch.cuda.Stream(device) for _ in range(inflight - 1)]
+        self.lanes = [Lane(M, cfg, self.fanout, self.B, self.R, rank, world, device, self.table, s) for s in streams]
+        self.ctx, self.bufs, self.rows = self.lanes[0].ctx, self.lanes[0].bufs, self.lanes[0].rows
         self._batches = []
         self._epoch = 0
 
@@ -76,22 +87,30 @@ class State:
         seeds, ep, j = self._batches[i]
         return seeds, W.batch_rng_seed(RUN_SEED, ep, self.rank, j)
 
-    def step(self, seeds, rng_seed, stream=None, ev=None):
+    def step(self, seeds, rng_seed, stream=None, ev=None, lane=0):
+        """Sample + gather one batch on `lane` (its stream unless `stream` is given)."""
         H = len(self.fanout)
-        self.ctx.sample(self.graph.indptr, self.graph.indices, seeds, self.fanout, rng_seed, self.bufs, stream=stream)
+        L = self.lanes[lane]
+        s = stream if stream is not None else L.stream
+        L.ctx.sample(self.graph.indptr, self.graph.indices, seeds, self.fanout, rng_seed, L.bufs, stream=s)
         if ev is not None:
-            ev[0].record()
-        self.ctx.gather(self.bufs.nodes, self.rows, n_dev=self.bufs.counts[H:H + 1], max_n=self.bufs.nodes.numel(),
-                        stream=stream)
+            ev[0].record(s)
+        L.ctx.gather(L.bufs.nodes, L.rows, n_dev=L.bufs.counts[H:H + 1], max_n=L.bufs.nodes.numel(), stream=s)
         if ev is not None:
-            ev[1].record()
+            ev[1].record(s)
+
+    def step_host(self, seeds_host, rng_seed, counts_host, lane=0):
+        """The same step through moment_step_host: host seeds in, host counts out (asynchronous)."""
+        L = self.lanes[lane]
+        L.ctx.step_host(self.graph.indptr, self.graph.indices, seeds_host, self.fanout, rng_seed, L.bufs, L.rows,
+                        counts_host, stream=L.stream)
 
     def launches_per_step(self):
-        return 1 + 3 * len(self.fanout) + 1 + 1  # init, (offsets, sample, bitscan) per hop, finalize, gather
+        return 1 + 2 * len(self.fanout) + 1 + 1  # init, (sample, bitscan) per hop, compact, gather
 
 
-def build_state(name, device="cuda:0", rank=0, world=1):
-    return State(name, device, rank, world)
+def build_state(name, device="cuda:0", rank=0, world=1, inflight=1):
+    return State(name, device, rank, world, inflight)
 
 
 class Clocks:
@@ -236,6 +255,7 @@ def main():
     ap.add_argument("--impl", default="moment", choices=["moment", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=100)
+    ap.add_argument("--inflight", type=int, default=4, help="batches in flight per GPU (one stream each)")
     args = ap.parse_args()
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -251,11 +271,23 @@ def main():
         import torch.distributed as dist
 
         dist.init_process_group("nccl", device_id=torch.device(dev))
-    st = build_state(args.config, dev, rank, world)
+    st = build_state(args.config, dev, rank, world, args.inflight)
     H = len(st.fanout)
-    stream = torch.cuda.current_stream()
+    P = len(st.lanes)
+    main_stream = torch.cuda.current_stream()
+
+    def fork(ev):
+        for L in st.lanes[1:]:
+            L.stream.wait_event(ev)
+
+    def join():
+        for L in st.lanes[1:]:
+            e = torch.cuda.Event()
+            e.record(L.stream)
+            main_stream.wait_event(e)
+
     for i in range(args.warmup):
-        st.step(*st.batch(i))
+        st.step(*st.batch(i), lane=i % P)
     torch.cuda.synchronize()
     batches = [st.batch(args.warmup + i) for i in range(args.steps)]
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
@@ -265,10 +297,12 @@ def main():
         dist.barrier()
     torch.cuda.synchronize()
     t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    t_start.record()
+    t_start.record(main_stream)
+    fork(t_start)
     for i in range(args.steps):
-        st.step(*batches[i], ev=evs[i])
-    t_end.record()
+        st.step(*batches[i], ev=evs[i], lane=i % P)
+    join()
+    t_end.record(main_stream)
     torch.cuda.synchronize()
     if dist:
         dist.barrier()
@@ -278,8 +312,8 @@ def main():
     # |F_H| per timed step (deterministic: recomputed untimed from the same batches)
     nF = []
     for i in range(args.steps):
-        st.step(*batches[i])
-        nF.append(int(st.bufs.counts[H]))
+        st.step(*batches[i], lane=0)
+        nF.append(int(st.lanes[0].bufs.counts[H]))
     if dist:
         t = torch.tensor([ms], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -295,22 +329,26 @@ def main():
     alg_bytes = (sum(nF) / args.steps) * (2 * st.R + 8)
     peak, peak_kind = _peaks()
     achieved = alg_bytes / (gather_ms / 1000) / 1e9
-    # e2e: the same step through the C ABI with host buffers (seeds H2D, counts D2H, synchronised)
-    seeds_h = [batches[i % len(batches)][0].cpu().pin_memory() for i in range(max(3, args.e2e_steps))]
-    counts_h = torch.zeros(2 * H + 1, dtype=torch.int64).pin_memory()
+    # e2e: the same steps through the C ABI with host buffers: pinned seeds H2D and counts D2H every step,
+    # P steps in flight (one per lane), all copies inside the timed region
+    n_e2e = max(3, args.e2e_steps)
+    seeds_h = [batches[i % len(batches)][0].cpu().pin_memory() for i in range(n_e2e)]
+    counts_h = [torch.zeros(2 * H + 1, dtype=torch.int64).pin_memory() for _ in range(n_e2e)]
     for i in range(3):
-        st.ctx.step_host(st.graph.indptr, st.graph.indices, seeds_h[i], st.fanout, batches[i][1], st.bufs, st.rows,
-                         counts_h)
+        st.step_host(seeds_h[i], batches[i][1], counts_h[i], lane=i % P)
+    torch.cuda.synchronize()
     if dist:
         dist.barrier()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
+    e0.record(main_stream)
+    fork(e0)
     for i in range(args.e2e_steps):
-        st.ctx.step_host(st.graph.indptr, st.graph.indices, seeds_h[i], st.fanout, batches[i][1], st.bufs, st.rows,
-                         counts_h)
-    e1.record()
+        st.step_host(seeds_h[i], batches[i][1], counts_h[i], lane=i % P)
+    join()
+    e1.record(main_stream)
     torch.cuda.synchronize()
     e2e_ms = e0.elapsed_time(e1)
+    assert all(int(c[H]) > 0 for c in counts_h[: args.e2e_steps])
     if dist:
         t = torch.tensor([e2e_ms], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -325,7 +363,8 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u8", "data": "synthetic",
             "config": {"workload": args.config, "desc": st.cfg["desc"], "global_batch": st.B * world,
-                       "fanout": list(st.fanout), "row_bytes": st.R, "parallelism": f"dp{world} (replicated graph+features)",
+                       "fanout": list(st.fanout), "row_bytes": st.R, "inflight_batches_per_gpu": P,
+                       "parallelism": f"dp{world} (replicated graph+features)",
                        "l2": "inputs larger than L2 (features %.2f GB, CSR %.2f GB)" % (
                            st.table.numel() / 1e9, (st.graph.indptr.numel() * 8 + st.graph.indices.numel() * 4) / 1e9),
                        "mean_F_H": sum(nF) / args.steps},

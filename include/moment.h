@@ -275,8 +275,10 @@ moment_status moment_gather_group(moment_ctx_t const* ctxs, int32_t world, const
 
 /* ================================================================================================
  * End-to-end step with HOST buffers (the e2e leg of the benchmark): copies seeds host->device, samples,
- * gathers F_H into d_out, copies the 2H+1 counts device->host (into counts_host), and synchronises.
- * seeds_host / counts_host should be pinned for asynchronous copies.
+ * gathers F_H into d_rows (NULL: sample only), copies the 2H+1 counts device->host into counts_host. All of
+ * it is enqueued on `stream`; counts_host is valid once the stream has reached the copy (synchronise the
+ * stream or an event). seeds_host / counts_host should be pinned; seeds_host must stay unchanged until the
+ * H2D copy has executed. Several steps may be in flight on different ctxs / streams.
  * ================================================================================================ */
 moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds_host,
                                int64_t n_seeds, const moment_sample_params* params,

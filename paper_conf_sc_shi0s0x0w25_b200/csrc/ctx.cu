@@ -2,6 +2,8 @@
 // points of include/moment.h: moment_sample, moment_gather, moment_gather_group, moment_bucket,
 // moment_hotness, moment_step_host.
 #include <algorithm>
+#include <cstdlib>
+#include <string>
 #include <new>
 
 #include "ctx.h"
@@ -89,6 +91,10 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     c->bin_owner.assign(a->bin_owner, a->bin_owner + a->n_bins);
     c->bin_ptr.assign(a->bin_ptr, a->bin_ptr + a->n_bins);
     c->placement = a->placement;
+    if (const char* gp = std::getenv("MOMENT_GATHER_PATH")) {
+        const std::string v(gp);
+        c->gather_path = v == "ldg" ? 1 : (v == "bulk" ? 2 : 0);
+    }
     if (a->quota) c->quota.assign(a->quota, a->quota + (size_t)a->n_bins * a->world);
     // bounds per hop
     c->max_F.resize(a->max_hops + 1);
@@ -112,18 +118,22 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     const int64_t o_newbits = cv.take<uint32_t>(n_words_pad);
     const int64_t o_visited = cv.take<uint32_t>(n_words_pad);
     const int64_t scan_tiles = n_words_pad / kBitscanTileWords;
-    c->sample_tiles_off.resize(a->max_hops);
     c->bitscan_tiles_off.resize(a->max_hops);
-    int64_t nts = 0;
+    int64_t nts = 0, cnt_total = 0;
+    for (int h = 0; h < a->max_hops; h++) {  // compact chain: hop-aligned tiles of all hops
+        nts += (c->max_F[h] + kSampleTile - 1) / kSampleTile;
+        cnt_total += c->max_F[h];
+    }
     for (int h = 0; h < a->max_hops; h++) {
-        c->sample_tiles_off[h] = nts;
-        nts += std::max<int64_t>(1, (c->max_F[h] + kSampleTile - 1) / kSampleTile);
         c->bitscan_tiles_off[h] = nts;
         nts += scan_tiles;
     }
     c->n_tile_status = std::max<int64_t>(nts, 1);
     const int64_t o_tiles = cv.take<uint64_t>(c->n_tile_status);
-    const int64_t o_tickets = cv.take<uint32_t>(2 * std::max(1, a->max_hops));
+    const int64_t o_tickets = cv.take<uint32_t>(1 + std::max(1, a->max_hops));
+    const int64_t o_ebase = cv.take<uint64_t>(std::max(1, a->max_hops));
+    const int64_t o_pad = cv.take<int32_t>(c->max_edges);
+    const int64_t o_cnt = cv.take<int32_t>(cnt_total);
     const int64_t o_err = cv.take<uint32_t>(1);
     const int32_t Q = std::max(1, a->n_bins * a->world);
     const int64_t bk_tiles = (c->max_requests + kBucketTile - 1) / kBucketTile + 1;
@@ -150,6 +160,9 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     c->visited = reinterpret_cast<uint32_t*>(w + o_visited);
     c->tile_status = reinterpret_cast<uint64_t*>(w + o_tiles);
     c->tickets = reinterpret_cast<uint32_t*>(w + o_tickets);
+    c->ebase = reinterpret_cast<uint64_t*>(w + o_ebase);
+    c->pad = reinterpret_cast<int32_t*>(w + o_pad);
+    c->cnt = reinterpret_cast<int32_t*>(w + o_cnt);
     c->error_flag = reinterpret_cast<uint32_t*>(w + o_err);
     if (a->n_bins > 0) {
         c->bk_tile_counts = reinterpret_cast<int64_t*>(w + o_bk_tc);
@@ -283,6 +296,6 @@ extern "C" moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* cs
     MOMENT_TRY(launch_sample(ctx, csr, ctx->d_seed_stage, n_seeds, params, out, s));
     const int H = params->n_hops;
     if (d_rows) MOMENT_TRY(launch_gather(ctx, out->nodes, out->counts + H, out->cap_nodes, d_rows, nullptr, ctx->rank, s));
-    MOMENT_TRY(cuda_check(cudaMemcpyAsync(counts_host, out->counts, (2 * H + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "moment_step_host: D2H"));
-    return cuda_check(cudaStreamSynchronize(s), "moment_step_host: sync");
+    return cuda_check(cudaMemcpyAsync(counts_host, out->counts, (2 * H + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s),
+                      "moment_step_host: D2H");
 }

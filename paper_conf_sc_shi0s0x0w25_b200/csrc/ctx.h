@@ -19,6 +19,7 @@ struct moment_ctx_s {
     int64_t max_nodes = 0, max_edges = 0, max_offsets = 0;
     int64_t row_bytes = 0, row_stride = 0;
     int32_t n_bins = 0;
+    int32_t gather_path = 0;  // 0 auto (TMA bulk copies for local rows), 1 LDG.128 only, 2 bulk (MOMENT_GATHER_PATH)
     std::vector<int32_t> bin_owner;
     std::vector<void*> bin_ptr;
     const uint64_t* placement = nullptr;
@@ -31,10 +32,13 @@ struct moment_ctx_s {
     uint32_t* newbits = nullptr;    // [n_words]: ids emitted at the current hop
     uint32_t* visited = nullptr;    // [n_words]: F_h membership
     int64_t n_words = 0;
-    uint64_t* tile_status = nullptr;  // decoupled look-back descriptors, all hops, both scans
+    uint64_t* tile_status = nullptr;  // decoupled look-back descriptors: compact chain, then bitscan per hop
     int64_t n_tile_status = 0;
-    std::vector<int64_t> sample_tiles_off, bitscan_tiles_off;  // per hop offsets into tile_status
-    uint32_t* tickets = nullptr;      // [2 * max_hops] tile tickets
+    std::vector<int64_t> bitscan_tiles_off;  // per hop offsets into tile_status
+    uint32_t* tickets = nullptr;      // [1 + max_hops] tile tickets (compact, bitscan per hop)
+    uint64_t* ebase = nullptr;        // [max_hops] first global edge position of each hop (compact)
+    int32_t* pad = nullptr;           // [max_edges] padded samples (node idx * k + r), all hops
+    int32_t* cnt = nullptr;           // [sum_h max_F[h]] samples per node, all hops
     uint32_t* error_flag = nullptr;   // device error bits (seed check)
     // bucketing workspace
     int64_t max_requests = 0;

@@ -82,6 +82,110 @@ __global__ void __launch_bounds__(kGatherThreads) gather_kernel(BinTable bins, c
     }
 }
 
+// ---- TMA bulk-copy gather (H6, local rows) ---------------------------------------------------------
+// One warp per block. A tile is 32 consecutive output rows: lane l issues one cp.async.bulk global->smem
+// copy of row l (completion counted in bytes on the stage's mbarrier); once the tile has landed, lane 0
+// stores the whole tile (contiguous in the output) with ONE cp.async.bulk smem->global copy. kStages
+// tiles are in flight per block, so an SM keeps kStages x blocks x 32 rows of reads outstanding with a
+// handful of instructions per row.
+constexpr int kBulkMaxRows = 32;
+constexpr int kBulkStageBudget = 14 * 1024;  // bytes per stage: 4 stages x 4 blocks per SM fit in smem
+constexpr int kBulkStages = 4;
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void bulk_load(void* dst_smem, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst_smem)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_store(void* dst, const void* src_smem, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src_smem)),
+                 "r"(bytes)
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// Source address of output row i (a row of bin b at slot s, or of the replicated table at slot id).
+__device__ __forceinline__ const char* row_src(const BinTable& bins, const uint64_t* placement, int64_t id,
+                                               int64_t stride) {
+    if (placement) {
+        const uint64_t p = __ldg(placement + id);
+        return reinterpret_cast<const char*>(bins.base[(int)(p >> 40)]) + (int64_t)(p & kSlotMask) * stride;
+    }
+    return reinterpret_cast<const char*>(bins.base[0]) + id * stride;
+}
+
+__global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const uint64_t* __restrict__ placement,
+                                                         const int64_t* __restrict__ ids, const int64_t* n_dev,
+                                                         int64_t max_n, uint32_t R, int64_t stride,
+                                                         int rows_per_tile, char* __restrict__ out) {
+    extern __shared__ __align__(128) char stage[];  // kBulkStages * rows_per_tile * R
+    __shared__ __align__(8) uint64_t full[kBulkStages];
+    const int lane = threadIdx.x;
+    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+    const int64_t n_tiles = (n + rows_per_tile - 1) / rows_per_tile;
+    if (lane == 0)
+        for (int s = 0; s < kBulkStages; s++) mbar_init(&full[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    __syncwarp();
+    const int64_t t0 = blockIdx.x, dt = gridDim.x;
+    auto issue = [&](int64_t tile, int s) {
+        const int64_t row0 = tile * rows_per_tile;
+        const int rows = (int)min((int64_t)rows_per_tile, n - row0);
+        if (lane == 0) mbar_expect_tx(&full[s], (uint32_t)rows * R);
+        __syncwarp();
+        if (lane < rows) {
+            const char* src = row_src(bins, placement, __ldg(ids + row0 + lane), stride);
+            bulk_load(stage + ((size_t)s * rows_per_tile + lane) * R, src, R, &full[s]);
+        }
+    };
+    // prologue: fill the pipeline
+    int64_t next = t0;
+    for (int s = 0; s < kBulkStages && next < n_tiles; s++, next += dt) issue(next, s);
+    int it = 0;
+    for (int64_t tile = t0; tile < n_tiles; tile += dt, it++) {
+        const int s = it % kBulkStages;
+        mbar_wait(&full[s], (uint32_t)((it / kBulkStages) & 1));
+        const int64_t row0 = tile * rows_per_tile;
+        const int rows = (int)min((int64_t)rows_per_tile, n - row0);
+        if (lane == 0) {
+            bulk_store(out + row0 * (int64_t)R, stage + (size_t)s * rows_per_tile * R, (uint32_t)rows * R);
+            bulk_wait_read<0>();  // stage s may be refilled once the store has read it
+        }
+        __syncwarp();
+        if (next < n_tiles) {
+            issue(next, s);
+            next += dt;
+        }
+    }
+    if (lane == 0) bulk_wait_all();
+}
+
 // Relay service (H7): this rank (server) reads the host rows that `requester` routed through it and
 // stores them into the requester's output (an NVLink store when the requester is another GPU).
 // Requests are the queue segments q = j * world + server of every host bin j.
@@ -297,10 +401,29 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
     if ((reinterpret_cast<uintptr_t>(out) & 15) != 0) return fail(MOMENT_EINVAL, "moment_gather: out must be 16-byte aligned");
     MOMENT_TRY(cuda_pending("moment_gather: pending CUDA error"));
     if (max_n == 0) return MOMENT_OK;
-    const int grid = grid_for(max_n * rv, kGatherThreads * kGatherUnroll, 148 * 8);
-    gather_kernel<<<grid, kGatherThreads, 0, stream>>>(make_bins(ctx), ctx->placement, ids, n_dev, max_n,
-                                                        make_fastdiv((uint32_t)rv), ctx->row_stride / 16, route,
-                                                        ctx->world, serve_rank, reinterpret_cast<int4*>(out));
+    bool all_local = true;
+    for (int b = 0; b < ctx->n_bins; b++) all_local &= ctx->bin_owner[b] == ctx->rank;
+    const bool bulk = ctx->gather_path == 2 || (ctx->gather_path == 0 && route == nullptr && all_local);
+    if (bulk && route == nullptr) {
+        const int rows = (int)std::max<int64_t>(1, std::min<int64_t>(kBulkMaxRows, kBulkStageBudget / ctx->row_bytes));
+        const size_t smem = (size_t)kBulkStages * rows * ctx->row_bytes;
+        static thread_local size_t configured = 0;
+        if (smem > 48 * 1024 && configured < smem) {
+            MOMENT_TRY(cuda_check(cudaFuncSetAttribute(gather_bulk_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                       (int)smem), "moment_gather: smem attribute"));
+            configured = smem;
+        }
+        const int64_t tiles = (max_n + rows - 1) / rows;
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, 148 * 4));
+        gather_bulk_kernel<<<grid, 32, smem, stream>>>(make_bins(ctx), ctx->placement, ids, n_dev, max_n,
+                                                       (uint32_t)ctx->row_bytes, ctx->row_stride, rows,
+                                                       reinterpret_cast<char*>(out));
+    } else {
+        const int grid = grid_for(max_n * rv, kGatherThreads * kGatherUnroll, 148 * 8);
+        gather_kernel<<<grid, kGatherThreads, 0, stream>>>(make_bins(ctx), ctx->placement, ids, n_dev, max_n,
+                                                            make_fastdiv((uint32_t)rv), ctx->row_stride / 16, route,
+                                                            ctx->world, serve_rank, reinterpret_cast<int4*>(out));
+    }
     return cuda_check(cudaGetLastError(), "moment_gather: launch");
 }
 

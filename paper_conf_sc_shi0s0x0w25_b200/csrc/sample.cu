@@ -1,15 +1,17 @@
 // sample.cu — H1-H3: multi-hop neighbour sampling with dedup/relabel on sm_100a (R3-R6).
 //
-// One sample call is 3H + 2 kernels and no memsets; no kernel needs the host to know |F_h| or E_h (every
-// size is read from device memory), so the call is CUDA-graph capturable:
+// One sample call is 2H + 2 kernels and no memsets. No kernel needs the host to know |F_h| or E_h (every
+// size is read from device memory), so the call is CUDA-graph capturable. The critical path per hop is
+// two kernels; offsets, compaction and relabelling of every hop happen once, after the last hop:
 //   init        : F_0 = seeds; lidx / visited of the seeds; zero the tile descriptors and tickets.
-//   offsets (h) : tile of 256 frontier nodes -> degrees -> block scan + block-wide decoupled look-back =
-//                 edge offsets. Blocks without a tile relabel hop h-1's edges (src = lidx[id]).
-//   sample (h)  : one G-lane group per frontier node draws its Floyd / with-replacement positions from
-//                 Philox (choices resolved in parallel), writes the neighbour ids, marks them in `newbits`.
+//   sample (h)  : one G-lane group per frontier node v draws min(deg v, k) Floyd (or with-replacement)
+//                 positions from Philox (choices resolved in parallel), writes the neighbour ids to the
+//                 node's k-slot row of a padded buffer, its count to cnt_h, and marks them in `newbits`.
 //   bitscan (h) : F_{h+1} = F_h ++ (newbits & ~visited) in ascending id order: chained scan of bitmap
 //                 popcounts (1024 words per tile) gives each new id its position; lidx[id] = position.
-//   finalize    : relabel the last hop's edges, then clear the `visited` words of F_H (next call starts clean).
+//   compact     : one chained scan over the counts of all hops (hop-aligned tiles of 256 nodes, block-wide
+//                 decoupled look-back) = global edge positions -> per-hop offsets, E_h, and
+//                 src = lidx[padded id] copied into the packed output; then clears `visited` for F_H.
 #include <cooperative_groups.h>
 
 #include <algorithm>
@@ -25,49 +27,26 @@ namespace {
 constexpr int kScanWords = kBitscanWordsPerThread;  // bitmap words per bitscan thread (4: one uint4)
 constexpr int kScanTileWords = kBitscanTileWords;   // 1024 words = 32768 ids per tile
 static_assert(kScanWords == 4, "bitscan loads one uint4 per thread");
+constexpr int kMaxHops = 16;
+constexpr uint64_t kBaseReady = 1ull << 63;
 
 struct HopArgs {
     const int64_t* indptr;
     const int32_t* indices;
-    int64_t* nodes;
-    int64_t* offsets;
-    int32_t* src;
-    int64_t* counts;
+    const int64_t* nodes;
+    const int64_t* counts;
+    int32_t* pad;      // [F_bound_h * k]: node idx's samples at pad[idx * k + r]
+    int32_t* cnt;      // [F_bound_h]: samples of node idx
     uint32_t* newbits;
-    const int32_t* lidx;
-    uint64_t* tile_status;
-    uint32_t* ticket;
     uint64_t seed;
-    int32_t h, H, k;
+    int32_t h, k;
     int32_t replace;
 };
-
-// Sizes of earlier hops live in counts: offsets block h starts at sum_{h'<h} (|F_h'| + 1) and the
-// edges of hop h at sum_{h'<h} E_h'.
-__device__ __forceinline__ void hop_bases(const int64_t* counts, int h, int H, int64_t* off_base, int64_t* edge_base) {
-    int64_t ob = 0, eb = 0;
-    for (int q = 0; q < h; q++) {
-        ob += counts[q] + 1;
-        eb += counts[H + 1 + q];
-    }
-    *off_base = ob;
-    *edge_base = eb;
-}
 
 __device__ __forceinline__ void mark_new(uint32_t* newbits, int32_t u) {
     const uint32_t bit = 1u << (u & 31);
     uint32_t* w = newbits + (u >> 5);
     if ((__ldcg(w) & bit) == 0) atomicOr(w, bit);
-}
-
-// src[e] = lidx[src[e]] for the E edges of hop `hr` (grid-stride over `nthreads` participants).
-__device__ __forceinline__ void relabel_hop(int32_t* src_all, const int64_t* counts, const int32_t* lidx, int hr, int H,
-                                            int64_t tid, int64_t nthreads) {
-    int64_t ob, eb;
-    hop_bases(counts, hr, H, &ob, &eb);
-    const int64_t E = counts[H + 1 + hr];
-    int32_t* src = src_all + eb;
-    for (int64_t e = tid; e < E; e += nthreads) src[e] = __ldg(lidx + src[e]);
 }
 
 // Floyd's k choices for node v at hop h, lane i < k owning choice i (k <= G): t_i = uniform(draw(i),
@@ -97,8 +76,8 @@ __device__ __forceinline__ int32_t floyd_choice(const cg::thread_block_tile<G>& 
     return ((dup >> lane) & 1u) ? jj : t;
 }
 
-// Positions for k > G (G == 32 only): chunks of 32 choices resolved in draw order; earlier chunks are
-// final and kept (as positions) in `out`, then sorted and replaced by ids. Rare (fanout > 32).
+// Positions for k > 32 (G == 32): chunks of 32 choices resolved in draw order; earlier chunks are final
+// and kept (as positions) in `out`, then sorted and replaced by ids. Rare (fanout > 32).
 __device__ void sample_node_wide(const cg::thread_block_tile<32>& grp, const HopArgs& a, int64_t v, int64_t lo,
                                  int32_t d, int32_t* out) {
     const int lane = grp.thread_rank();
@@ -144,59 +123,10 @@ __device__ void sample_node_wide(const cg::thread_block_tile<32>& grp, const Hop
     }
 }
 
-// Pass A of hop h: edge offsets. count(v) = min(deg v, k) (k if REPLACE and deg > 0); tile of 256 nodes
-// -> block scan -> block-wide decoupled look-back. Writes offsets[F] and E_h = counts[H+1+h]. Blocks
-// without (further) tiles relabel hop h-1's edges (its lidx is final once bitscan h-1 has run).
-__global__ void __launch_bounds__(kSampleTile) hop_offsets_kernel(HopArgs a) {
-    __shared__ int64_t s_red[kSampleTile / 32];
-    __shared__ uint32_t s_tile;
-    __shared__ int s_nearest;
-    const int64_t F = a.counts[a.h];
-    int64_t off_base, edge_base;
-    hop_bases(a.counts, a.h, a.H, &off_base, &edge_base);
-    int64_t* offsets = a.offsets + off_base;
-    if (F == 0 && blockIdx.x == 0 && threadIdx.x == 0) {
-        offsets[0] = 0;
-        a.counts[a.H + 1 + a.h] = 0;
-    }
-    const int64_t n_tiles = (F + kSampleTile - 1) / kSampleTile;
-    for (;;) {
-        if (threadIdx.x == 0) s_tile = atomicAdd(a.ticket, 1u);
-        __syncthreads();
-        const int64_t tile = s_tile;
-        if (tile >= n_tiles) break;
-        const int64_t idx = tile * kSampleTile + threadIdx.x;
-        int32_t c = 0;
-        if (idx < F) {
-            const int64_t v = a.nodes[idx];
-            const int64_t d = __ldg(a.indptr + v + 1) - __ldg(a.indptr + v);
-            c = a.replace ? (d > 0 ? a.k : 0) : (int32_t)min(d, (int64_t)a.k);
-        }
-        int64_t agg;
-        const int64_t excl = dev::block_exclusive_scan<kSampleTile>(c, &agg, s_red);
-        const int64_t off = dev::lookback_block<kSampleTile>(a.tile_status, tile, agg, s_red, &s_nearest) + excl;
-        if (idx < F) {
-            offsets[idx] = off;
-            if (idx == F - 1) {
-                offsets[F] = off + c;
-                a.counts[a.H + 1 + a.h] = off + c;
-            }
-        }
-        __syncthreads();
-    }
-    if (a.h > 0)
-        relabel_hop(a.src, a.counts, a.lidx, a.h - 1, a.H, (int64_t)blockIdx.x * kSampleTile + threadIdx.x,
-                    (int64_t)gridDim.x * kSampleTile);
-}
-
-// Pass B of hop h: one G-lane group per frontier node (grid-stride), every node in flight at once.
+// One G-lane group per frontier node (grid-stride): every node of F_h in flight at once.
 template <int G>
 __global__ void __launch_bounds__(256) hop_sample_kernel(HopArgs a) {
     const int64_t F = a.counts[a.h];
-    int64_t off_base, edge_base;
-    hop_bases(a.counts, a.h, a.H, &off_base, &edge_base);
-    const int64_t* offsets = a.offsets + off_base;
-    int32_t* src = a.src + edge_base;
     auto grp = cg::tiled_partition<G>(cg::this_thread_block());
     const int lane = grp.thread_rank();
     const int k = a.k;
@@ -205,7 +135,9 @@ __global__ void __launch_bounds__(256) hop_sample_kernel(HopArgs a) {
         const int64_t v = a.nodes[idx];
         const int64_t lo = __ldg(a.indptr + v);
         const int32_t d = (int32_t)(__ldg(a.indptr + v + 1) - lo);
-        int32_t* out = src + offsets[idx];
+        int32_t* out = a.pad + idx * k;
+        const int32_t c = a.replace ? (d > 0 ? k : 0) : min(d, k);
+        if (lane == 0) a.cnt[idx] = c;
         if (d <= 0) continue;
         if (a.replace) {  // k draws, draw order
             for (int i = lane; i < k; i += G) {
@@ -219,16 +151,16 @@ __global__ void __launch_bounds__(256) hop_sample_kernel(HopArgs a) {
                 out[p] = u;
                 mark_new(a.newbits, u);
             }
-        } else if (k <= G) {  // Floyd, one choice per lane, then rank = position in sorted order
-            const int32_t c = floyd_choice<G>(grp, a.seed, v, a.h, d, k);
+        } else if (k <= G) {  // Floyd, one choice per lane; rank = position in sorted order
+            const int32_t ch = floyd_choice<G>(grp, a.seed, v, a.h, d, k);
             int r = 0;
 #pragma unroll
             for (int l = 0; l < G; l++) {
-                const int32_t cl = grp.shfl(c, l);
-                r += (l < k) && cl < c;
+                const int32_t cl = grp.shfl(ch, l);
+                r += (l < k) && cl < ch;
             }
             if (lane < k) {
-                const int32_t u = __ldg(a.indices + lo + c);
+                const int32_t u = __ldg(a.indices + lo + ch);
                 out[r] = u;
                 mark_new(a.newbits, u);
             }
@@ -306,21 +238,96 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
     }
 }
 
-// Relabel the last hop's edges; clear the visited words of every node of F_H.
-__global__ void finalize_kernel(int32_t* src_all, const int64_t* counts, const int32_t* lidx, const int64_t* nodes,
-                                uint32_t* visited, int H) {
-    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (int64_t)gridDim.x * blockDim.x;
-    if (H > 0) relabel_hop(src_all, counts, lidx, H - 1, H, tid, nth);
-    const int64_t FH = counts[H];
-    for (int64_t i = tid; i < FH; i += nth) visited[nodes[i] >> 5] = 0u;
+struct CompactArgs {
+    int64_t* offsets;
+    int32_t* src;
+    int64_t* counts;
+    const int64_t* nodes;
+    const int32_t* lidx;
+    uint32_t* visited;
+    uint64_t* tile_status;  // one chain over the tiles of all hops
+    uint64_t* ebase;        // [H]: global edge position of hop h's first edge, kBaseReady-flagged
+    uint32_t* ticket;
+    int32_t H;
+    int32_t k[kMaxHops];
+    const int32_t* pad[kMaxHops];
+    const int32_t* cnt[kMaxHops];
+};
+
+__global__ void __launch_bounds__(kSampleTile) compact_kernel(CompactArgs a) {
+    __shared__ int64_t s_red[kSampleTile / 32];
+    __shared__ uint32_t s_tile;
+    __shared__ int s_nearest;
+    __shared__ int64_t s_base;
+    int64_t tiles_before[kMaxHops + 1];
+    tiles_before[0] = 0;
+    for (int h = 0; h < a.H; h++) tiles_before[h + 1] = tiles_before[h] + (a.counts[h] + kSampleTile - 1) / kSampleTile;
+    const int64_t n_tiles = tiles_before[a.H];
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        // hops with an empty frontier have no tile: write their (empty) offsets and E_h here
+        int64_t ob = 0;
+        for (int h = 0; h < a.H; h++) {
+            if (a.counts[h] == 0) {
+                a.offsets[ob] = 0;
+                a.counts[a.H + 1 + h] = 0;
+            }
+            ob += a.counts[h] + 1;
+        }
+    }
+    for (;;) {
+        if (threadIdx.x == 0) s_tile = atomicAdd(a.ticket, 1u);
+        __syncthreads();
+        const int64_t tile = s_tile;
+        if (tile >= n_tiles) break;
+        int h = 0;
+        while (tile >= tiles_before[h + 1]) h++;
+        const int64_t F = a.counts[h];
+        int64_t ob = 0;
+        for (int q = 0; q < h; q++) ob += a.counts[q] + 1;
+        const int64_t lt = tile - tiles_before[h];
+        const int64_t idx = lt * kSampleTile + threadIdx.x;
+        const int32_t c = idx < F ? a.cnt[h][idx] : 0;
+        int64_t agg;
+        const int64_t excl = dev::block_exclusive_scan<kSampleTile>(c, &agg, s_red);
+        const int64_t prefix = dev::lookback_block<kSampleTile>(a.tile_status, tile, agg, s_red, &s_nearest);
+        if (threadIdx.x == 0) {
+            if (lt == 0) {
+                dev::st_release(&a.ebase[h], kBaseReady | (uint64_t)prefix);
+                s_base = prefix;
+            } else {
+                uint64_t b;
+                do {
+                    b = dev::ld_acquire(&a.ebase[h]);
+                } while (!(b & kBaseReady));
+                s_base = (int64_t)(b & ~kBaseReady);
+            }
+        }
+        __syncthreads();
+        const int64_t gpos = prefix + excl;  // global position of this node's first edge
+        const int64_t rel = gpos - s_base;
+        if (idx < F) {
+            a.offsets[ob + idx] = rel;
+            if (idx == F - 1) {
+                a.offsets[ob + F] = rel + c;
+                a.counts[a.H + 1 + h] = rel + c;
+            }
+            const int32_t* p = a.pad[h] + idx * a.k[h];
+            for (int r = 0; r < c; r++) a.src[gpos + r] = __ldg(a.lidx + __ldg(p + r));
+        }
+        __syncthreads();
+    }
+    const int64_t FH = a.counts[a.H];
+    for (int64_t i = (int64_t)blockIdx.x * kSampleTile + threadIdx.x; i < FH; i += (int64_t)gridDim.x * kSampleTile)
+        a.visited[a.nodes[i] >> 5] = 0u;
 }
 
 __global__ void init_kernel(const int64_t* seeds, int64_t n_seeds, int64_t n_vertices, int64_t* nodes, int32_t* lidx,
                             uint32_t* visited, int64_t* counts, uint32_t* error_flag, int check, uint64_t* tile_status,
-                            int64_t n_tile_status, uint32_t* tickets, int n_tickets) {
+                            int64_t n_tile_status, uint32_t* tickets, int n_tickets, uint64_t* ebase, int n_ebase) {
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (int64_t)gridDim.x * blockDim.x;
     for (int64_t i = tid; i < n_tile_status; i += nth) tile_status[i] = 0;
     for (int64_t i = tid; i < n_tickets; i += nth) tickets[i] = 0;
+    for (int64_t i = tid; i < n_ebase; i += nth) ebase[i] = 0;
     for (int64_t i = tid; i < n_seeds; i += nth) {
         const int64_t v = seeds[i];
         if (v < 0 || v >= n_vertices) {  // never write out of range, checked or not
@@ -338,10 +345,7 @@ __global__ void init_kernel(const int64_t* seeds, int64_t n_seeds, int64_t n_ver
 }
 
 template <int G>
-void launch_hop(const HopArgs& a, int64_t max_F, int64_t prev_E, cudaStream_t stream) {
-    const int64_t tiles = std::max<int64_t>(1, (max_F + kSampleTile - 1) / kSampleTile);
-    const int64_t relabel_blocks = (prev_E + kSampleTile * 4 - 1) / (kSampleTile * 4);
-    hop_offsets_kernel<<<(int)std::min<int64_t>(std::max(tiles, relabel_blocks), 148 * 4), kSampleTile, 0, stream>>>(a);
+void launch_sample_hop(const HopArgs& a, int64_t max_F, cudaStream_t stream) {
     const int64_t blocks = std::max<int64_t>(1, (max_F * G + 255) / 256);
     hop_sample_kernel<G><<<(int)std::min<int64_t>(blocks, 148 * 16), 256, 0, stream>>>(a);
 }
@@ -355,7 +359,8 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const int6
         return fail(MOMENT_EINVAL, "moment_sample: csr has %lld vertices, ctx was created for %lld",
                     (long long)csr->n_vertices, (long long)ctx->n_vertices);
     const int H = p->n_hops;
-    if (H < 0 || H > ctx->max_hops) return fail(MOMENT_EINVAL, "moment_sample: n_hops %d > max_hops %d", H, ctx->max_hops);
+    if (H < 0 || H > ctx->max_hops || H > kMaxHops)
+        return fail(MOMENT_EINVAL, "moment_sample: n_hops %d > max_hops %d", H, ctx->max_hops);
     if (n_seeds < 0 || n_seeds > ctx->max_seeds)
         return fail(MOMENT_EINVAL, "moment_sample: n_seeds %lld > max_seeds %lld", (long long)n_seeds, (long long)ctx->max_seeds);
     if (H > 0 && !p->fanout) return fail(MOMENT_EINVAL, "moment_sample: fanout is null");
@@ -377,30 +382,44 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const int6
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n_seeds + 255) / 256, 148 * 4));
         init_kernel<<<grid, 256, 0, stream>>>(seeds, n_seeds, ctx->n_vertices, out->nodes, ctx->lidx, ctx->visited,
                                               out->counts, ctx->error_flag, check, ctx->tile_status, ctx->n_tile_status,
-                                              ctx->tickets, 2 * std::max(1, ctx->max_hops));
+                                              ctx->tickets, 1 + std::max(1, ctx->max_hops), ctx->ebase,
+                                              std::max(1, ctx->max_hops));
     }
-    // per-call bounds on |F_h| for launch sizing (the kernels read the true sizes from counts)
-    int64_t F_bound = n_seeds, E_prev = 0;
+    // per-call bounds on |F_h| for launch sizing and padded-buffer carving (true sizes live in counts)
+    CompactArgs ca{};
+    int64_t F_bound = n_seeds, pad_off = 0, cnt_off = 0, comp_tiles = 0;
     const int64_t n_scan_tiles = (ctx->n_words + kScanTileWords - 1) / kScanTileWords;
     for (int h = 0; h < H; h++) {
         const int k = p->fanout[h];
-        HopArgs a{csr->indptr, csr->indices, out->nodes, out->offsets, out->src, out->counts, ctx->newbits, ctx->lidx,
-                  ctx->tile_status + ctx->sample_tiles_off[h], ctx->tickets + 2 * h, p->rng_seed, h, H, k, replace};
-        if (k <= 4) launch_hop<4>(a, F_bound, E_prev, stream);
-        else if (k <= 8) launch_hop<8>(a, F_bound, E_prev, stream);
-        else if (k <= 16) launch_hop<16>(a, F_bound, E_prev, stream);
-        else launch_hop<32>(a, F_bound, E_prev, stream);
+        HopArgs a{csr->indptr, csr->indices, out->nodes, out->counts, ctx->pad + pad_off, ctx->cnt + cnt_off,
+                  ctx->newbits, p->rng_seed, h, k, replace};
+        if (k <= 4) launch_sample_hop<4>(a, F_bound, stream);
+        else if (k <= 8) launch_sample_hop<8>(a, F_bound, stream);
+        else if (k <= 16) launch_sample_hop<16>(a, F_bound, stream);
+        else launch_sample_hop<32>(a, F_bound, stream);
         ScanArgs s{out->nodes, out->counts, ctx->lidx, ctx->newbits, ctx->visited,
-                   ctx->tile_status + ctx->bitscan_tiles_off[h], ctx->tickets + 2 * h + 1, ctx->n_words, h};
+                   ctx->tile_status + ctx->bitscan_tiles_off[h], ctx->tickets + 1 + h, ctx->n_words, h};
         bitscan_kernel<<<(int)std::min<int64_t>(n_scan_tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
-        E_prev = F_bound * (int64_t)k;
+        ca.k[h] = k;
+        ca.pad[h] = ctx->pad + pad_off;
+        ca.cnt[h] = ctx->cnt + cnt_off;
+        pad_off += F_bound * k;
+        cnt_off += F_bound;
+        comp_tiles += (F_bound + kSampleTile - 1) / kSampleTile;
         F_bound = std::min(F_bound + F_bound * (int64_t)k, ctx->n_vertices);
     }
-    {
-        const int64_t work = std::max(E_prev, F_bound);
-        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((work + 1023) / 1024, 148 * 8));
-        finalize_kernel<<<grid, 256, 0, stream>>>(out->src, out->counts, ctx->lidx, out->nodes, ctx->visited, H);
-    }
+    ca.offsets = out->offsets;
+    ca.src = out->src;
+    ca.counts = out->counts;
+    ca.nodes = out->nodes;
+    ca.lidx = ctx->lidx;
+    ca.visited = ctx->visited;
+    ca.tile_status = ctx->tile_status;  // the compact chain occupies the first entries
+    ca.ebase = ctx->ebase;
+    ca.ticket = ctx->tickets;
+    ca.H = H;
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(std::max(comp_tiles, (F_bound + 1023) / 1024), 148 * 4));
+    compact_kernel<<<grid, kSampleTile, 0, stream>>>(ca);
     return cuda_check(cudaGetLastError(), "moment_sample: launch");
 }
 

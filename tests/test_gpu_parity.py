@@ -130,10 +130,12 @@ def test_sample_reused_ctx_many_batches(orc, c1):
         assert_same_sample(got, want)
 
 
+@pytest.mark.parametrize("path", ["auto", "ldg", "bulk"])
 @pytest.mark.parametrize("dim,dtype", [(4, torch.float32), (12, torch.float32), (100, torch.float32),
                                        (128, torch.float32), (768, torch.float16), (1024, torch.float32)])
-def test_gather_replicated(orc, dim, dtype):
+def test_gather_replicated(orc, dim, dtype, path, monkeypatch):
     _need_gpu()
+    monkeypatch.setenv("MOMENT_GATHER_PATH", path)
     n = 5000
     table = W.feature_table(n, dim, dtype, device=DEV)
     R = table.shape[1]
@@ -280,6 +282,7 @@ def test_step_host_matches_device_path(orc, c1):
     counts_h = torch.zeros(5, dtype=torch.int64).pin_memory()
     seeds_h = seeds.cpu().pin_memory()
     ctx.step_host(g.indptr, g.indices, seeds_h, [10, 5], 77, bufs, rows, counts_h)
+    torch.cuda.synchronize()
     want = orc.sample(g.indptr.cpu().numpy(), g.indices.cpu().numpy(), seeds_h.numpy(), [10, 5], 77)
     assert np.array_equal(counts_h.numpy(), want["counts"])
     nF = int(want["counts"][2])

@@ -64,8 +64,8 @@ def main():
     from torch.profiler import ProfilerActivity, profile
 
     with profile(activities=[ProfilerActivity.CUDA]) as prof:
-        for _ in range(args.steps):
-            g.replay()
+        for i in range(args.steps):
+            st.step(*batches[5 + i])
         torch.cuda.synchronize()
     evs = [e for e in prof.events() if e.device_type.name == "CUDA"]
     evs.sort(key=lambda e: e.time_range.start)
@@ -73,8 +73,8 @@ def main():
     gap = defaultdict(list)
     prev_end = None
     for e in evs:
-        name = e.name.split("(")[0].replace("moment::", "").replace("(anonymous namespace)::", "")
-        name = name.replace("void ", "")[:48]
+        name = e.name.replace("(anonymous namespace)::", "").replace("moment::", "").replace("void ", "")
+        name = name.split("(")[0][:48]
         dur[name].append(e.time_range.elapsed_us())
         if prev_end is not None:
             gap[name].append(max(0.0, e.time_range.start - prev_end))
