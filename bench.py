@@ -88,16 +88,19 @@ class State:
         return seeds, W.batch_rng_seed(RUN_SEED, ep, self.rank, j)
 
     def step(self, seeds, rng_seed, stream=None, ev=None, lane=0):
-        """Sample + gather one batch on `lane` (its stream unless `stream` is given)."""
+        """Sample + gather one batch on `lane` (its stream unless `stream` is given): one moment_step call,
+        replayed from the lane ctx's cached CUDA graph. With `ev` (a pair of timing events) the step runs as
+        moment_sample + moment_gather with the events around the gather kernel instead."""
         H = len(self.fanout)
         L = self.lanes[lane]
         s = stream if stream is not None else L.stream
+        if ev is None:
+            L.ctx.step(self.graph.indptr, self.graph.indices, seeds, self.fanout, rng_seed, L.bufs, L.rows, stream=s)
+            return
         L.ctx.sample(self.graph.indptr, self.graph.indices, seeds, self.fanout, rng_seed, L.bufs, stream=s)
-        if ev is not None:
-            ev[0].record(s)
+        ev[0].record(s)
         L.ctx.gather(L.bufs.nodes, L.rows, n_dev=L.bufs.counts[H:H + 1], max_n=L.bufs.nodes.numel(), stream=s)
-        if ev is not None:
-            ev[1].record(s)
+        ev[1].record(s)
 
     def step_host(self, seeds_host, rng_seed, counts_host, lane=0):
         """The same step through moment_step_host: host seeds in, host counts out (asynchronous)."""
@@ -300,7 +303,7 @@ def main():
     t_start.record(main_stream)
     fork(t_start)
     for i in range(args.steps):
-        st.step(*batches[i], ev=evs[i], lane=i % P)
+        st.step(*batches[i], lane=i % P)
     join()
     t_end.record(main_stream)
     torch.cuda.synchronize()
@@ -308,9 +311,13 @@ def main():
         dist.barrier()
     ck = clocks.stop()
     ms = t_start.elapsed_time(t_end)
-    gather_ms = sum(a.elapsed_time(b) for a, b in evs) / args.steps
-    # |F_H| per timed step (deterministic: recomputed untimed from the same batches)
+    # roofline pass over the same batches: CUDA events around the dominant kernel (the gather) on its
+    # stream, one lane; also |F_H| of every timed step (deterministic, so identical to the timed run)
     nF = []
+    for i in range(args.steps):
+        st.step(*batches[i], ev=evs[i], lane=0)
+    torch.cuda.synchronize()
+    gather_ms = sum(a.elapsed_time(b) for a, b in evs) / args.steps
     for i in range(args.steps):
         st.step(*batches[i], lane=0)
         nF.append(int(st.lanes[0].bufs.counts[H]))

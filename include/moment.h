@@ -274,6 +274,19 @@ moment_status moment_gather_group(moment_ctx_t const* ctxs, int32_t world, const
                                   const int64_t* const* n_dev, int64_t max_n, void* const* out, void* stream);
 
 /* ================================================================================================
+ * One whole hot-path step on device buffers: moment_sample of `seeds` followed by moment_gather of F_H
+ * into d_rows (NULL: sample only; rows relayed through other ranks are not supported here). The 2H + 3
+ * kernels are replayed from a CUDA graph cached in the ctx (captured on the first call of a given shape:
+ * csr, n_seeds, fanout, flags, out and d_rows pointers; re-captured when any of them changes), so the host
+ * cost per step is two API calls. The per-batch rng_seed and seeds pointer reach the kernels through a
+ * device call block written by an async copy from a pinned ring. If `stream` is being captured by the
+ * caller, the kernels are launched directly instead. Same outputs as moment_sample + moment_gather.
+ * ================================================================================================ */
+moment_status moment_step(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
+                          const moment_sample_params* params, const moment_sample_out* out, void* d_rows,
+                          void* stream);
+
+/* ================================================================================================
  * End-to-end step with HOST buffers (the e2e leg of the benchmark): copies seeds host->device, samples,
  * gathers F_H into d_rows (NULL: sample only), copies the 2H+1 counts device->host into counts_host. All of
  * it is enqueued on `stream`; counts_host is valid once the stream has reached the copy (synchronise the

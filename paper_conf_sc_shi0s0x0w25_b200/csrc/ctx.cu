@@ -4,6 +4,7 @@
 #include <algorithm>
 #include <cstdlib>
 #include <string>
+#include <cstring>
 #include <new>
 
 #include "ctx.h"
@@ -148,6 +149,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
         o_owner = cv.take<int32_t>(a->n_bins);
     }
     const int64_t o_seed = cv.take<int64_t>(a->max_seeds);
+    const int64_t o_call = cv.take<uint64_t>(2);
     c->ws_bytes = cv.off;
     cudaError_t e = cudaMalloc(&c->ws, c->ws_bytes);
     if (e != cudaSuccess) {
@@ -174,8 +176,15 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
         c->d_bin_owner = reinterpret_cast<int32_t*>(w + o_owner);
     }
     c->d_seed_stage = reinterpret_cast<int64_t*>(w + o_seed);
+    c->d_call = reinterpret_cast<uint64_t*>(w + o_call);
     moment_status st = MOMENT_OK;
     do {
+        if ((st = cuda_check(cudaHostAlloc(reinterpret_cast<void**>(&c->h_ring), sizeof(uint64_t) * 2 * moment_ctx_s::kRing,
+                                           cudaHostAllocDefault), "moment_ctx_create: pinned call ring")) != MOMENT_OK) break;
+        for (int i = 0; i < moment_ctx_s::kRing && st == MOMENT_OK; i++)
+            st = cuda_check(cudaEventCreateWithFlags(&c->ring_ev[i], cudaEventDisableTiming), "moment_ctx_create: event");
+        if (st != MOMENT_OK) break;
+        if ((st = cuda_check(cudaStreamCreateWithFlags(&c->cap_stream, cudaStreamNonBlocking), "moment_ctx_create: stream")) != MOMENT_OK) break;
         if ((st = cuda_check(cudaMemset(c->ws, 0, c->ws_bytes), "moment_ctx_create: memset")) != MOMENT_OK) break;
         if ((st = cuda_check(cudaMemset(c->lidx, 0xFF, a->n_vertices * sizeof(int32_t)), "moment_ctx_create: memset")) != MOMENT_OK) break;
         if (a->n_bins > 0) {
@@ -188,8 +197,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     } while (0);
     if (cur != a->device) cudaSetDevice(cur);
     if (st != MOMENT_OK) {
-        cudaFree(c->ws);
-        delete c;
+        moment_ctx_free(c);
         return st;
     }
     *out = c;
@@ -201,7 +209,12 @@ extern "C" moment_status moment_ctx_free(moment_ctx_t ctx) {
     int cur = -1;
     cudaGetDevice(&cur);
     cudaSetDevice(ctx->device);
-    cudaError_t e = cudaFree(ctx->ws);
+    if (ctx->step_exec) cudaGraphExecDestroy(ctx->step_exec);
+    if (ctx->cap_stream) cudaStreamDestroy(ctx->cap_stream);
+    for (auto& ev : ctx->ring_ev)
+        if (ev) cudaEventDestroy(ev);
+    if (ctx->h_ring) cudaFreeHost(ctx->h_ring);
+    cudaError_t e = ctx->ws ? cudaFree(ctx->ws) : cudaSuccess;
     cudaSetDevice(cur);
     delete ctx;
     return cuda_check(e, "moment_ctx_free");
@@ -213,10 +226,104 @@ extern "C" moment_status moment_ctx_workspace_bytes(moment_ctx_t ctx, int64_t* b
     return MOMENT_OK;
 }
 
+namespace {
+
+// Stage the per-call arguments (rng_seed, seeds pointer) into the device call block: a pinned ring slot
+// plus one 16-byte async copy, ordered before the call's kernels on `s`.
+moment_status write_call(moment_ctx_s* c, uint64_t rng_seed, const int64_t* seeds, cudaStream_t s) {
+    const int slot = c->ring_pos++ % moment_ctx_s::kRing;
+    MOMENT_TRY(cuda_check(cudaEventSynchronize(c->ring_ev[slot]), "call ring"));  // slot's previous copy done
+    c->h_ring[2 * slot] = rng_seed;
+    c->h_ring[2 * slot + 1] = reinterpret_cast<uint64_t>(seeds);
+    MOMENT_TRY(cuda_check(cudaMemcpyAsync(c->d_call, c->h_ring + 2 * slot, 2 * sizeof(uint64_t), cudaMemcpyHostToDevice, s),
+                          "call block H2D"));
+    return cuda_check(cudaEventRecord(c->ring_ev[slot], s), "call ring event");
+}
+
+bool same_key(const moment_ctx_s::StepKey& k, const moment_csr* csr, int64_t n_seeds, const moment_sample_params* p,
+              const moment_sample_out* out, void* rows) {
+    if (k.indptr != csr->indptr || k.indices != csr->indices || k.n_seeds != n_seeds || k.flags != p->flags ||
+        k.rows != rows || (int)k.fanout.size() != p->n_hops)
+        return false;
+    for (int h = 0; h < p->n_hops; h++)
+        if (k.fanout[h] != p->fanout[h]) return false;
+    return std::memcmp(&k.out, out, sizeof(moment_sample_out)) == 0;
+}
+
+// One sample + gather, replayed from a cached CUDA graph (captured on first use of a shape); falls back to
+// direct launches while the caller's stream is itself being captured.
+moment_status run_step(moment_ctx_s* c, const moment_csr* csr, int64_t n_seeds, const moment_sample_params* p,
+                       const moment_sample_out* out, void* rows, cudaStream_t s) {
+    const int H = p->n_hops;
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    MOMENT_TRY(cuda_check(cudaStreamIsCapturing(s, &cs), "moment_step"));
+    if (cs != cudaStreamCaptureStatusNone || std::getenv("MOMENT_NO_GRAPH")) {
+        MOMENT_TRY(launch_sample(c, csr, c->d_call, n_seeds, p, out, s));
+        if (rows) MOMENT_TRY(launch_gather(c, out->nodes, out->counts + H, out->cap_nodes, rows, nullptr, c->rank, s));
+        return MOMENT_OK;
+    }
+    if (!c->step_exec || !same_key(c->step_key, csr, n_seeds, p, out, rows)) {
+        if (c->step_exec) {
+            MOMENT_TRY(cuda_check(cudaStreamSynchronize(s), "moment_step: drain before re-capture"));
+            cudaGraphExecDestroy(c->step_exec);
+            c->step_exec = nullptr;
+        }
+        MOMENT_TRY(cuda_check(cudaStreamBeginCapture(c->cap_stream, cudaStreamCaptureModeThreadLocal), "capture"));
+        moment_status st = launch_sample(c, csr, c->d_call, n_seeds, p, out, c->cap_stream);
+        if (st == MOMENT_OK && rows)
+            st = launch_gather(c, out->nodes, out->counts + H, out->cap_nodes, rows, nullptr, c->rank, c->cap_stream);
+        cudaGraph_t g = nullptr;
+        cudaError_t e = cudaStreamEndCapture(c->cap_stream, &g);
+        if (st != MOMENT_OK) {
+            if (g) cudaGraphDestroy(g);
+            return st;
+        }
+        MOMENT_TRY(cuda_check(e, "moment_step: end capture"));
+        e = cudaGraphInstantiate(&c->step_exec, g, 0);
+        cudaGraphDestroy(g);
+        MOMENT_TRY(cuda_check(e, "moment_step: instantiate"));
+        c->step_key.indptr = csr->indptr;
+        c->step_key.indices = csr->indices;
+        c->step_key.n_seeds = n_seeds;
+        c->step_key.fanout.assign(p->fanout, p->fanout + H);
+        c->step_key.flags = p->flags;
+        c->step_key.out = *out;
+        c->step_key.rows = rows;
+    }
+    return cuda_check(cudaGraphLaunch(c->step_exec, s), "moment_step: graph launch");
+}
+
+moment_status check_rows(const moment_ctx_s* c, void* rows, const moment_sample_out* out) {
+    if (!rows) return MOMENT_OK;
+    if (c->n_bins <= 0) return fail(MOMENT_EINVAL, "moment_step: ctx has no feature bins");
+    if (c->world > 1 && has_remote_relay(c))
+        return fail(MOMENT_EUNSUPPORTED, "moment_step: the quota relays host rows through other ranks; use moment_gather_group");
+    if ((reinterpret_cast<uintptr_t>(rows) & 15) != 0) return fail(MOMENT_EINVAL, "moment_step: rows must be 16-byte aligned");
+    if (out->cap_nodes * (c->row_bytes / 16) >= (int64_t(1) << 32))
+        return fail(MOMENT_EUNSUPPORTED, "moment_step: %lld rows exceed 2^32 vectors per call", (long long)out->cap_nodes);
+    return MOMENT_OK;
+}
+
+}  // namespace
+
 extern "C" moment_status moment_sample(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
                                        const moment_sample_params* params, const moment_sample_out* out, void* stream) {
     MOMENT_TRY(check_ctx(ctx, "moment_sample"));
-    return launch_sample(ctx, csr, seeds, n_seeds, params, out, static_cast<cudaStream_t>(stream));
+    MOMENT_TRY(check_sample(ctx, csr, seeds, n_seeds, params, out));
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    MOMENT_TRY(write_call(ctx, params->rng_seed, seeds, s));
+    return launch_sample(ctx, csr, ctx->d_call, n_seeds, params, out, s);
+}
+
+extern "C" moment_status moment_step(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
+                                     const moment_sample_params* params, const moment_sample_out* out, void* d_rows,
+                                     void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_step"));
+    MOMENT_TRY(check_sample(ctx, csr, seeds, n_seeds, params, out));
+    MOMENT_TRY(check_rows(ctx, d_rows, out));
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    MOMENT_TRY(write_call(ctx, params->rng_seed, seeds, s));
+    return run_step(ctx, csr, n_seeds, params, out, d_rows, s);
 }
 
 extern "C" moment_status moment_sample_check(moment_ctx_t ctx, void* stream) {
@@ -290,12 +397,13 @@ extern "C" moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* cs
                                           int64_t* counts_host, void* stream) {
     MOMENT_TRY(check_ctx(ctx, "moment_step_host"));
     if (!params || !out || !counts_host || (n_seeds > 0 && !seeds_host)) return fail(MOMENT_EINVAL, "moment_step_host: null argument");
-    if (n_seeds > ctx->max_seeds) return fail(MOMENT_EINVAL, "moment_step_host: n_seeds > max_seeds");
+    MOMENT_TRY(check_sample(ctx, csr, ctx->d_seed_stage, n_seeds, params, out));
+    MOMENT_TRY(check_rows(ctx, d_rows, out));
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     MOMENT_TRY(cuda_check(cudaMemcpyAsync(ctx->d_seed_stage, seeds_host, n_seeds * sizeof(int64_t), cudaMemcpyHostToDevice, s), "moment_step_host: H2D"));
-    MOMENT_TRY(launch_sample(ctx, csr, ctx->d_seed_stage, n_seeds, params, out, s));
+    MOMENT_TRY(write_call(ctx, params->rng_seed, ctx->d_seed_stage, s));
+    MOMENT_TRY(run_step(ctx, csr, n_seeds, params, out, d_rows, s));
     const int H = params->n_hops;
-    if (d_rows) MOMENT_TRY(launch_gather(ctx, out->nodes, out->counts + H, out->cap_nodes, d_rows, nullptr, ctx->rank, s));
     return cuda_check(cudaMemcpyAsync(counts_host, out->counts, (2 * H + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s),
                       "moment_step_host: D2H");
 }

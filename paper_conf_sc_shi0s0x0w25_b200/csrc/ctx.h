@@ -50,7 +50,24 @@ struct moment_ctx_s {
     int64_t* d_quota = nullptr;         // [n_bins * world]
     int32_t* d_bin_owner = nullptr;     // [n_bins]
     int64_t* d_seed_stage = nullptr;    // [max_seeds] for moment_step_host
-    int64_t* d_counts_stage = nullptr;  // unused placeholder
+    // per-call arguments the kernels read from device memory (so one captured graph serves every batch)
+    uint64_t* d_call = nullptr;         // [2]: rng_seed, seeds pointer
+    static constexpr int kRing = 64;
+    uint64_t* h_ring = nullptr;         // pinned [kRing][2] staging of the call block
+    cudaEvent_t ring_ev[kRing] = {};
+    int ring_pos = 0;
+    // cached CUDA graph of one moment_step (sample + gather), re-captured when its shape changes
+    cudaStream_t cap_stream = nullptr;
+    cudaGraphExec_t step_exec = nullptr;
+    struct StepKey {
+        const void* indptr = nullptr;
+        const void* indices = nullptr;
+        int64_t n_seeds = -1;
+        std::vector<int32_t> fanout;
+        uint32_t flags = 0;
+        moment_sample_out out{};
+        void* rows = nullptr;
+    } step_key;
 };
 
 namespace moment {
@@ -71,7 +88,9 @@ constexpr int kBucketTile = 1024;    // requests per bucketing tile
 constexpr int kMaxFanout = 1024;
 
 // Launchers (defined in sample.cu / gather.cu).
-moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
+moment_status check_sample(const moment_ctx_s* ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
+                           const moment_sample_params* p, const moment_sample_out* out);
+moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint64_t* call, int64_t n_seeds,
                             const moment_sample_params* p, const moment_sample_out* out, cudaStream_t stream);
 moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n, void* out,
                             const int32_t* route, int32_t serve_rank, cudaStream_t stream);

@@ -38,7 +38,7 @@ struct HopArgs {
     int32_t* pad;      // [F_bound_h * k]: node idx's samples at pad[idx * k + r]
     int32_t* cnt;      // [F_bound_h]: samples of node idx
     uint32_t* newbits;
-    uint64_t seed;
+    const uint64_t* call;  // device call block: [0] = rng_seed, [1] = seeds pointer (written per call)
     int32_t h, k;
     int32_t replace;
 };
@@ -78,8 +78,8 @@ __device__ __forceinline__ int32_t floyd_choice(const cg::thread_block_tile<G>& 
 
 // Positions for k > 32 (G == 32): chunks of 32 choices resolved in draw order; earlier chunks are final
 // and kept (as positions) in `out`, then sorted and replaced by ids. Rare (fanout > 32).
-__device__ void sample_node_wide(const cg::thread_block_tile<32>& grp, const HopArgs& a, int64_t v, int64_t lo,
-                                 int32_t d, int32_t* out) {
+__device__ void sample_node_wide(const cg::thread_block_tile<32>& grp, const HopArgs& a, uint64_t seed, int64_t v,
+                                 int64_t lo, int32_t d, int32_t* out) {
     const int lane = grp.thread_rank();
     const int k = a.k;
     for (int c0 = 0; c0 < k; c0 += 32) {
@@ -88,7 +88,7 @@ __device__ void sample_node_wide(const cg::thread_block_tile<32>& grp, const Hop
         bool prev_hit = false;
         if (i < k) {
             j = d - k + i;
-            t = (int32_t)dev::uniform(dev::draw(a.seed, v, a.h, i), (uint32_t)(j + 1));
+            t = (int32_t)dev::uniform(dev::draw(seed, v, a.h, i), (uint32_t)(j + 1));
             for (int q = 0; q < c0; q++) prev_hit |= out[q] == t;
         }
         const int nm = min(32, k - c0);
@@ -127,6 +127,7 @@ __device__ void sample_node_wide(const cg::thread_block_tile<32>& grp, const Hop
 template <int G>
 __global__ void __launch_bounds__(256) hop_sample_kernel(HopArgs a) {
     const int64_t F = a.counts[a.h];
+    const uint64_t seed = a.call[0];
     auto grp = cg::tiled_partition<G>(cg::this_thread_block());
     const int lane = grp.thread_rank();
     const int k = a.k;
@@ -141,7 +142,7 @@ __global__ void __launch_bounds__(256) hop_sample_kernel(HopArgs a) {
         if (d <= 0) continue;
         if (a.replace) {  // k draws, draw order
             for (int i = lane; i < k; i += G) {
-                const int32_t u = __ldg(a.indices + lo + dev::uniform(dev::draw(a.seed, v, a.h, i), (uint32_t)d));
+                const int32_t u = __ldg(a.indices + lo + dev::uniform(dev::draw(seed, v, a.h, i), (uint32_t)d));
                 out[i] = u;
                 mark_new(a.newbits, u);
             }
@@ -152,7 +153,7 @@ __global__ void __launch_bounds__(256) hop_sample_kernel(HopArgs a) {
                 mark_new(a.newbits, u);
             }
         } else if (k <= G) {  // Floyd, one choice per lane; rank = position in sorted order
-            const int32_t ch = floyd_choice<G>(grp, a.seed, v, a.h, d, k);
+            const int32_t ch = floyd_choice<G>(grp, seed, v, a.h, d, k);
             int r = 0;
 #pragma unroll
             for (int l = 0; l < G; l++) {
@@ -165,7 +166,7 @@ __global__ void __launch_bounds__(256) hop_sample_kernel(HopArgs a) {
                 mark_new(a.newbits, u);
             }
         } else {
-            if constexpr (G == 32) sample_node_wide(grp, a, v, lo, d, out);
+            if constexpr (G == 32) sample_node_wide(grp, a, seed, v, lo, d, out);
         }
     }
 }
@@ -321,10 +322,11 @@ __global__ void __launch_bounds__(kSampleTile) compact_kernel(CompactArgs a) {
         a.visited[a.nodes[i] >> 5] = 0u;
 }
 
-__global__ void init_kernel(const int64_t* seeds, int64_t n_seeds, int64_t n_vertices, int64_t* nodes, int32_t* lidx,
+__global__ void init_kernel(const uint64_t* call, int64_t n_seeds, int64_t n_vertices, int64_t* nodes, int32_t* lidx,
                             uint32_t* visited, int64_t* counts, uint32_t* error_flag, int check, uint64_t* tile_status,
                             int64_t n_tile_status, uint32_t* tickets, int n_tickets, uint64_t* ebase, int n_ebase) {
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (int64_t)gridDim.x * blockDim.x;
+    const int64_t* seeds = reinterpret_cast<const int64_t*>(call[1]);
     for (int64_t i = tid; i < n_tile_status; i += nth) tile_status[i] = 0;
     for (int64_t i = tid; i < n_tickets; i += nth) tickets[i] = 0;
     for (int64_t i = tid; i < n_ebase; i += nth) ebase[i] = 0;
@@ -352,8 +354,11 @@ void launch_sample_hop(const HopArgs& a, int64_t max_F, cudaStream_t stream) {
 
 }  // namespace
 
-moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
-                            const moment_sample_params* p, const moment_sample_out* out, cudaStream_t stream) {
+// Validates the call on the host; enqueues nothing on error. The seeds pointer and rng_seed are read by
+// the kernels from the device call block `call` ([0] rng_seed, [1] seeds), written beforehand by the
+// caller (ctx.cu) so that a captured graph of these launches serves every batch.
+moment_status check_sample(const moment_ctx_s* ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
+                           const moment_sample_params* p, const moment_sample_out* out) {
     if (!csr || !p || !out || (!seeds && n_seeds > 0)) return fail(MOMENT_EINVAL, "moment_sample: null argument");
     if (csr->n_vertices != ctx->n_vertices || !csr->indptr || !csr->indices)
         return fail(MOMENT_EINVAL, "moment_sample: csr has %lld vertices, ctx was created for %lld",
@@ -375,12 +380,18 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const int6
     if (out->cap_nodes < need_nodes || out->cap_offsets < need_offsets || out->cap_edges < need_edges)
         return fail(MOMENT_EOVERFLOW, "moment_sample: output capacity too small: need nodes %lld offsets %lld edges %lld",
                     (long long)need_nodes, (long long)need_offsets, (long long)need_edges);
-    MOMENT_TRY(cuda_pending("moment_sample: pending CUDA error"));
+    return cuda_pending("moment_sample: pending CUDA error");
+}
+
+// Enqueues the 2H + 2 kernels of one sample call (arguments already validated by check_sample).
+moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint64_t* call, int64_t n_seeds,
+                            const moment_sample_params* p, const moment_sample_out* out, cudaStream_t stream) {
+    const int H = p->n_hops;
     const int check = (p->flags & MOMENT_SAMPLE_CHECK) ? 1 : 0;
     const int replace = (p->flags & MOMENT_SAMPLE_REPLACE) ? 1 : 0;
     {
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n_seeds + 255) / 256, 148 * 4));
-        init_kernel<<<grid, 256, 0, stream>>>(seeds, n_seeds, ctx->n_vertices, out->nodes, ctx->lidx, ctx->visited,
+        init_kernel<<<grid, 256, 0, stream>>>(call, n_seeds, ctx->n_vertices, out->nodes, ctx->lidx, ctx->visited,
                                               out->counts, ctx->error_flag, check, ctx->tile_status, ctx->n_tile_status,
                                               ctx->tickets, 1 + std::max(1, ctx->max_hops), ctx->ebase,
                                               std::max(1, ctx->max_hops));
@@ -392,7 +403,7 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const int6
     for (int h = 0; h < H; h++) {
         const int k = p->fanout[h];
         HopArgs a{csr->indptr, csr->indices, out->nodes, out->counts, ctx->pad + pad_off, ctx->cnt + cnt_off,
-                  ctx->newbits, p->rng_seed, h, k, replace};
+                  ctx->newbits, call, h, k, replace};
         if (k <= 4) launch_sample_hop<4>(a, F_bound, stream);
         else if (k <= 8) launch_sample_hop<8>(a, F_bound, stream);
         else if (k <= 16) launch_sample_hop<16>(a, F_bound, stream);

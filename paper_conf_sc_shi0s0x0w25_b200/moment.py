@@ -28,7 +28,7 @@ EXPORTED = [
     "moment_topology_free", "moment_maxflow", "moment_place", "moment_place_pack", "moment_plan", "moment_plan_info",
     "moment_plan_free", "moment_ctx_create", "moment_ctx_free", "moment_ctx_workspace_bytes", "moment_sample_bounds",
     "moment_sample", "moment_sample_check", "moment_hotness", "moment_bucket", "moment_gather", "moment_gather_group",
-    "moment_step_host",
+    "moment_step", "moment_step_host",
 ]
 
 
@@ -117,6 +117,7 @@ def lib():
             "moment_bucket": ([P, P, P, I64, P, P, P, P], I32),
             "moment_gather": ([P, P, P, I64, P, P], I32),
             "moment_gather_group": ([P, I32, P, P, I64, P, P], I32),
+            "moment_step": ([P, P, P, I64, P, P, P, P], I32),
             "moment_step_host": ([P, P, P, I64, P, P, P, P, P], I32),
         }
         for name, (args, res) in sig.items():
@@ -376,15 +377,37 @@ class Ctx:
         mn = ids.numel() if max_n is None else max_n
         _check(lib().moment_hotness(self.handle, ids.data_ptr(), _ptr(n_dev), mn, hot.data_ptr(), _stream(stream)))
 
+    def _args(self, indptr, indices, fanout, flags, out):
+        """ctypes argument structs for one (graph, fanout, flags, buffers) shape, built once and reused."""
+        key = (indptr.data_ptr(), indptr.numel(), indices.data_ptr(), tuple(int(x) for x in fanout), flags, id(out),
+               out.nodes.data_ptr())
+        cache = self.__dict__.setdefault("_arg_cache", {})
+        hit = cache.get(key)
+        if hit is None:
+            f = _np(fanout, np.int32)
+            csr = Csr(indptr.data_ptr(), indices.data_ptr(), indptr.numel() - 1, indices.numel())
+            params = SampleParams(len(f), f.ctypes.data, 0, flags)
+            so = out.struct()
+            hit = (csr, params, so, f, C.byref(csr), C.byref(params), C.byref(so))
+            cache[key] = hit
+        return hit
+
+    def step(self, indptr, indices, seeds, fanout, rng_seed: int, out: SampleBuffers, rows, *, flags: int = 0,
+             stream=None):
+        """moment_step: sample + gather of one batch, replayed from the ctx's cached CUDA graph."""
+        a = self._args(indptr, indices, fanout, flags, out)
+        a[1].rng_seed = rng_seed & 0xFFFFFFFFFFFFFFFF
+        _check(lib().moment_step(self.handle, a[4], seeds.data_ptr(), seeds.numel(), a[5], a[6], _ptr(rows),
+                                 _stream(stream)))
+        return out
+
     def step_host(self, indptr, indices, seeds_host, fanout, rng_seed: int, out: SampleBuffers, rows, counts_host,
                   *, flags: int = 0, stream=None):
-        csr = Csr(indptr.data_ptr(), indices.data_ptr(), indptr.numel() - 1, indices.numel())
-        f = _np(fanout, np.int32)
-        params = SampleParams(len(f), f.ctypes.data, rng_seed & 0xFFFFFFFFFFFFFFFF, flags)
-        so = out.struct()
-        _check(lib().moment_step_host(self.handle, C.byref(csr), seeds_host.data_ptr(), seeds_host.numel(),
-                                      C.byref(params), C.byref(so), _ptr(rows), counts_host.data_ptr(),
-                                      _stream(stream)))
+        """moment_step_host: host seeds in, host counts out, all asynchronous on `stream`."""
+        a = self._args(indptr, indices, fanout, flags, out)
+        a[1].rng_seed = rng_seed & 0xFFFFFFFFFFFFFFFF
+        _check(lib().moment_step_host(self.handle, a[4], seeds_host.data_ptr(), seeds_host.numel(), a[5], a[6],
+                                      _ptr(rows), counts_host.data_ptr(), _stream(stream)))
 
 
 def gather_group(ctxs, ids, out, *, n_dev=None, max_n: int, stream=None):

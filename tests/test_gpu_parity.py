@@ -308,3 +308,48 @@ def test_c2_full_size_bench_configuration(orc):
         rows = st.rows[torch.as_tensor(pick, device=DEV)].cpu().numpy()
         ids = want["nodes"][pick]
         assert np.array_equal(rows, W.feature_rows(torch.as_tensor(ids), st.dim, st.dtype).numpy())
+
+
+def test_moment_step_graph_matches_oracle_across_batches_and_shapes(orc, c1):
+    """moment_step replays a cached CUDA graph: per-call seeds / rng_seed must reach the kernels, and a
+    new shape (batch size, fanout, buffers) must re-capture."""
+    cfg, g = c1
+    n = g.n
+    table = W.feature_table(n, 32, torch.float32, device=DEV)
+    R = table.shape[1]
+    ctx = M.Ctx(n_vertices=n, max_seeds=1024, max_fanout=[10, 5], device=0, row_bytes=R, bin_owner=[0],
+                bin_ptr=[table.data_ptr()])
+    train = W.training_set(g, min_count=4096)
+    batches = W.epoch_batches(train, 1024, 0)
+    tab = table.cpu().numpy()
+    ip, ix = g.indptr.cpu().numpy(), g.indices.cpu().numpy()
+    for fanout, bsz in [([10, 5], 1024), ([10, 5], 1024), ([4, 3], 500), ([10, 5], 1024)]:
+        bufs = M.SampleBuffers.allocate(bsz, fanout, n, DEV)
+        rows = torch.empty((bufs.nodes.numel(), R), dtype=torch.uint8, device=DEV)
+        for b in range(3):
+            seeds = batches[b][:bsz]
+            rng = W.batch_rng_seed(5, 0, 0, b * 7 + bsz)
+            ctx.step(g.indptr, g.indices, seeds, fanout, rng, bufs, rows)
+            torch.cuda.synchronize()
+            got = bufs.result()
+            want = orc.sample(ip, ix, seeds.cpu().numpy(), fanout, rng)
+            assert_same_sample(got, want)
+            nF = int(want["counts"][len(fanout)])
+            assert np.array_equal(rows[:nF].cpu().numpy(), orc.gather(tab, want["nodes"]))
+
+
+def test_moment_step_many_in_flight(orc, c1):
+    """Several steps enqueued back to back on one ctx/stream (call-block ring in use) stay exact."""
+    cfg, g = c1
+    n = g.n
+    ctx = M.Ctx(n_vertices=n, max_seeds=256, max_fanout=[6, 3], device=0)
+    train = W.training_set(g, min_count=256 * 80)
+    batches = W.epoch_batches(train, 256, 0)[:80]
+    bufs = [M.SampleBuffers.allocate(256, [6, 3], n, DEV) for _ in batches]
+    for b, seeds in enumerate(batches):  # 80 > ring size: exercises slot reuse
+        ctx.step(g.indptr, g.indices, seeds, [6, 3], 1000 + b, bufs[b], None)
+    torch.cuda.synchronize()
+    ip, ix = g.indptr.cpu().numpy(), g.indices.cpu().numpy()
+    for b in [0, 1, 40, 63, 64, 65, 79]:
+        want = orc.sample(ip, ix, batches[b].cpu().numpy(), [6, 3], 1000 + b)
+        assert_same_sample(bufs[b].result(), want)
