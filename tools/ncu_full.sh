@@ -2,7 +2,7 @@
 # One `ncu --set full` capture of every product kernel of one warm bench step (1 lane, C2 by default).
 OUT=${1:-gpurun_out/prof_full}
 CFG=${2:-C2}
-KRE="regex:hop_|bitscan|compact|init_kernel|gather_kernel"
+KRE="regex:hop_|bitscan|compact|init_kernel|gather_"
 ncu --set full --clock-control none --import-source on -k "$KRE" -s 27 -c 9 -o "$OUT" \
     python bench.py --config "$CFG" --steps 2 --warmup 3 --inflight 1 --no-cpu-baseline --e2e-steps 0 > /dev/null 2>&1
 ncu -i "$OUT.ncu-rep" --page raw --csv \
