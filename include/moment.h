@@ -278,9 +278,10 @@ moment_status moment_gather_group(moment_ctx_t const* ctxs, int32_t world, const
  * into d_rows (NULL: sample only; rows relayed through other ranks are not supported here). The 2H + 3
  * kernels are replayed from a CUDA graph cached in the ctx (captured on the first call of a given shape:
  * csr, n_seeds, fanout, flags, out and d_rows pointers; re-captured when any of them changes), so the host
- * cost per step is two API calls. The per-batch rng_seed and seeds pointer reach the kernels through a
- * device call block written by an async copy from a pinned ring. If `stream` is being captured by the
- * caller, the kernels are launched directly instead. Same outputs as moment_sample + moment_gather.
+ * cost per step is two launches. The per-batch rng_seed and seeds pointer reach the kernels through a
+ * 16-byte device call block written by a one-thread kernel launched just before the graph. If `stream` is
+ * being captured by the caller, the kernels are launched directly instead (capture-safe). Same outputs as
+ * moment_sample + moment_gather.
  * ================================================================================================ */
 moment_status moment_step(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
                           const moment_sample_params* params, const moment_sample_out* out, void* d_rows,

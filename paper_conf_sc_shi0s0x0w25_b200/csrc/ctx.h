@@ -51,11 +51,7 @@ struct moment_ctx_s {
     int32_t* d_bin_owner = nullptr;     // [n_bins]
     int64_t* d_seed_stage = nullptr;    // [max_seeds] for moment_step_host
     // per-call arguments the kernels read from device memory (so one captured graph serves every batch)
-    uint64_t* d_call = nullptr;         // [2]: rng_seed, seeds pointer
-    static constexpr int kRing = 64;
-    uint64_t* h_ring = nullptr;         // pinned [kRing][2] staging of the call block
-    cudaEvent_t ring_ev[kRing] = {};
-    int ring_pos = 0;
+    uint64_t* d_call = nullptr;         // [2]: rng_seed, seeds pointer (written by set_call_kernel per call)
     // cached CUDA graph of one moment_step (sample + gather), re-captured when its shape changes
     cudaStream_t cap_stream = nullptr;
     cudaGraphExec_t step_exec = nullptr;
@@ -100,5 +96,7 @@ moment_status launch_relay(moment_ctx_s* server, moment_ctx_s* requester, const 
                            const int64_t* qoff, const int64_t* qpos, void* requester_out, cudaStream_t stream);
 moment_status launch_hotness(const int64_t* ids, const int64_t* n_dev, int64_t max_n, uint64_t* hot,
                              cudaStream_t stream);
+moment_status configure_sample_kernels(int carveout);
+moment_status configure_gather_kernels(int carveout);
 
 }  // namespace moment

@@ -66,14 +66,16 @@ __device__ __forceinline__ int64_t block_exclusive_scan(int64_t x, int64_t* tota
 // in increasing order through an atomic ticket, so every predecessor tile is owned by a running block.
 constexpr uint64_t kFlagAgg = 1ull << 62, kFlagPrefix = 2ull << 62, kValMask = (1ull << 62) - 1;
 
-__device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p) {
+// A descriptor carries its flag and its value in ONE 64-bit word written by one store, so readers need
+// only coherence on that word: relaxed device-scope atomics (no fence, no L1 invalidate per poll).
+__device__ __forceinline__ uint64_t ld_flag(const uint64_t* p) {
     return cuda::atomic_ref<unsigned long long, cuda::thread_scope_device>(
                *reinterpret_cast<unsigned long long*>(const_cast<uint64_t*>(p)))
-        .load(cuda::memory_order_acquire);
+        .load(cuda::memory_order_relaxed);
 }
-__device__ __forceinline__ void st_release(uint64_t* p, uint64_t v) {
+__device__ __forceinline__ void st_flag(uint64_t* p, uint64_t v) {
     cuda::atomic_ref<unsigned long long, cuda::thread_scope_device>(*reinterpret_cast<unsigned long long*>(p))
-        .store(v, cuda::memory_order_release);
+        .store(v, cuda::memory_order_relaxed);
 }
 
 // Warp-parallel decoupled look-back: called by ALL 32 lanes of one warp; inspects 32 predecessors per
@@ -81,17 +83,17 @@ __device__ __forceinline__ void st_release(uint64_t* p, uint64_t v) {
 __device__ __forceinline__ int64_t lookback_warp(uint64_t* status, int64_t tile, int64_t aggregate) {
     const int lane = threadIdx.x & 31;
     if (tile == 0) {
-        if (lane == 0) st_release(&status[0], kFlagPrefix | (uint64_t)aggregate);
+        if (lane == 0) st_flag(&status[0], kFlagPrefix | (uint64_t)aggregate);
         return 0;
     }
-    if (lane == 0) st_release(&status[tile], kFlagAgg | (uint64_t)aggregate);
+    if (lane == 0) st_flag(&status[tile], kFlagAgg | (uint64_t)aggregate);
     int64_t exclusive = 0;
     for (int64_t end = tile - 1;; end -= 32) {
         const int64_t j = end - lane;
         uint64_t s = kFlagPrefix;  // "before tile 0" acts as a zero prefix (never reached: tile 0 is a prefix)
         if (j >= 0) {
             do {
-                s = ld_acquire(&status[j]);
+                s = ld_flag(&status[j]);
             } while ((s & ~kValMask) == 0);
         }
         const unsigned pre = __ballot_sync(0xffffffffu, (s & ~kValMask) == kFlagPrefix);
@@ -102,7 +104,7 @@ __device__ __forceinline__ int64_t lookback_warp(uint64_t* status, int64_t tile,
         exclusive += v;
         if (pre) break;
     }
-    if (lane == 0) st_release(&status[tile], kFlagPrefix | (uint64_t)(exclusive + aggregate));
+    if (lane == 0) st_flag(&status[tile], kFlagPrefix | (uint64_t)(exclusive + aggregate));
     return exclusive;
 }
 
@@ -113,10 +115,10 @@ template <int NT>
 __device__ __forceinline__ int64_t lookback_block(uint64_t* status, int64_t tile, int64_t aggregate, int64_t* red,
                                                   int* nearest) {
     if (tile == 0) {
-        if (threadIdx.x == 0) st_release(&status[0], kFlagPrefix | (uint64_t)aggregate);
+        if (threadIdx.x == 0) st_flag(&status[0], kFlagPrefix | (uint64_t)aggregate);
         return 0;
     }
-    if (threadIdx.x == 0) st_release(&status[tile], kFlagAgg | (uint64_t)aggregate);
+    if (threadIdx.x == 0) st_flag(&status[tile], kFlagAgg | (uint64_t)aggregate);
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     int64_t exclusive = 0;
     for (int64_t end = tile - 1;; end -= NT) {
@@ -124,7 +126,7 @@ __device__ __forceinline__ int64_t lookback_block(uint64_t* status, int64_t tile
         uint64_t s = 0;
         if (j >= 0) {
             do {
-                s = ld_acquire(&status[j]);
+                s = ld_flag(&status[j]);
             } while ((s & ~kValMask) == 0);
         }
         if (threadIdx.x == 0) *nearest = NT;
@@ -144,7 +146,7 @@ __device__ __forceinline__ int64_t lookback_block(uint64_t* status, int64_t tile
         __syncthreads();
         if (stop < NT || end - NT < 0) break;
     }
-    if (threadIdx.x == 0) st_release(&status[tile], kFlagPrefix | (uint64_t)(exclusive + aggregate));
+    if (threadIdx.x == 0) st_flag(&status[tile], kFlagPrefix | (uint64_t)(exclusive + aggregate));
     return exclusive;
 }
 

@@ -91,6 +91,7 @@ __global__ void __launch_bounds__(kGatherThreads) gather_kernel(BinTable bins, c
 constexpr int kBulkMaxRows = 32;
 constexpr int kBulkStageBudget = 14 * 1024;  // bytes per stage: 4 stages x 4 blocks per SM fit in smem
 constexpr int kBulkStages = 4;
+constexpr int kBulkBlocksPerSM = 4;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -167,6 +168,8 @@ __global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const ui
     // prologue: fill the pipeline
     int64_t next = t0;
     for (int s = 0; s < kBulkStages && next < n_tiles; s++, next += dt) issue(next, s);
+    // steady state: store the tile that landed, then refill the stage of the PREVIOUS tile, whose store
+    // was issued one iteration ago (wait_group.read 1: every store but the newest has read its stage).
     int it = 0;
     for (int64_t tile = t0; tile < n_tiles; tile += dt, it++) {
         const int s = it % kBulkStages;
@@ -175,11 +178,11 @@ __global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const ui
         const int rows = (int)min((int64_t)rows_per_tile, n - row0);
         if (lane == 0) {
             bulk_store(out + row0 * (int64_t)R, stage + (size_t)s * rows_per_tile * R, (uint32_t)rows * R);
-            bulk_wait_read<0>();  // stage s may be refilled once the store has read it
+            if (it > 0) bulk_wait_read<1>();
         }
         __syncwarp();
-        if (next < n_tiles) {
-            issue(next, s);
+        if (it > 0 && next < n_tiles) {
+            issue(next, (it - 1) % kBulkStages);
             next += dt;
         }
     }
@@ -407,14 +410,8 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
     if (bulk && route == nullptr) {
         const int rows = (int)std::max<int64_t>(1, std::min<int64_t>(kBulkMaxRows, kBulkStageBudget / ctx->row_bytes));
         const size_t smem = (size_t)kBulkStages * rows * ctx->row_bytes;
-        static thread_local size_t configured = 0;
-        if (smem > 48 * 1024 && configured < smem) {
-            MOMENT_TRY(cuda_check(cudaFuncSetAttribute(gather_bulk_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                                       (int)smem), "moment_gather: smem attribute"));
-            configured = smem;
-        }
         const int64_t tiles = (max_n + rows - 1) / rows;
-        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, 148 * 4));
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, 148 * kBulkBlocksPerSM));
         gather_bulk_kernel<<<grid, 32, smem, stream>>>(make_bins(ctx), ctx->placement, ids, n_dev, max_n,
                                                        (uint32_t)ctx->row_bytes, ctx->row_stride, rows,
                                                        reinterpret_cast<char*>(out));
@@ -459,6 +456,23 @@ moment_status launch_relay(moment_ctx_s* server, moment_ctx_s* requester, const 
                                                        make_fastdiv((uint32_t)rv), server->row_stride / 16,
                                                        reinterpret_cast<int4*>(requester_out));
     return cuda_check(cudaGetLastError(), "moment_gather: relay launch");
+}
+
+// Kernel attributes, set once per device: every kernel of the library asks for the same shared-memory
+// carveout (so consecutive kernels never force an L1/shared reconfiguration bubble on the SMs), and the
+// bulk gather may use up to kBulkStages x kBulkStageBudget bytes of dynamic shared memory.
+moment_status configure_gather_kernels(int carveout) {
+    const void* fns[] = {(const void*)gather_kernel, (const void*)gather_bulk_kernel, (const void*)relay_kernel,
+                         (const void*)bucket_count_kernel, (const void*)bucket_scan_kernel,
+                         (const void*)bucket_route_kernel, (const void*)queue_count_kernel,
+                         (const void*)queue_scan_kernel, (const void*)queue_scatter_kernel, (const void*)hotness_kernel};
+    for (const void* f : fns)
+        if (carveout >= 0)
+            MOMENT_TRY(cuda_check(cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, carveout),
+                                  "carveout attribute"));
+    return cuda_check(cudaFuncSetAttribute((const void*)gather_bulk_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           kBulkStages * kBulkStageBudget),
+                      "bulk gather smem attribute");
 }
 
 moment_status launch_hotness(const int64_t* ids, const int64_t* n_dev, int64_t max_n, uint64_t* hot, cudaStream_t stream) {

@@ -43,10 +43,9 @@ struct HopArgs {
     int32_t replace;
 };
 
+// Fire-and-forget: the result is unused, so this is a RED.OR the issuing warp never waits on.
 __device__ __forceinline__ void mark_new(uint32_t* newbits, int32_t u) {
-    const uint32_t bit = 1u << (u & 31);
-    uint32_t* w = newbits + (u >> 5);
-    if ((__ldcg(w) & bit) == 0) atomicOr(w, bit);
+    atomicOr(newbits + (u >> 5), 1u << (u & 31));
 }
 
 // Floyd's k choices for node v at hop h, lane i < k owning choice i (k <= G): t_i = uniform(draw(i),
@@ -123,8 +122,33 @@ __device__ void sample_node_wide(const cg::thread_block_tile<32>& grp, const Hop
     }
 }
 
-// One G-lane group per frontier node (grid-stride): every node of F_h in flight at once.
+// Nodes with fanout > G (G == 32 only, fanout > 32): per-node paths without the register batching.
 template <int G>
+__device__ __forceinline__ void sample_node_slow(const cg::thread_block_tile<G>& grp, const HopArgs& a, uint64_t seed,
+                                                 int64_t v, int64_t lo, int32_t d, int32_t* out) {
+    const int lane = grp.thread_rank();
+    const int k = a.k;
+    if (a.replace) {
+        for (int i = lane; i < k; i += G) {
+            const int32_t u = __ldg(a.indices + lo + dev::uniform(dev::draw(seed, v, a.h, i), (uint32_t)d));
+            out[i] = u;
+            mark_new(a.newbits, u);
+        }
+    } else if (d <= k) {
+        for (int p = lane; p < d; p += G) {
+            const int32_t u = __ldg(a.indices + lo + p);
+            out[p] = u;
+            mark_new(a.newbits, u);
+        }
+    } else {
+        if constexpr (G == 32) sample_node_wide(grp, a, seed, v, lo, d, out);
+    }
+}
+
+// One G-lane group handles Q consecutive frontier nodes per step (grid-stride): their node ids, degrees,
+// choices (lane i owns choice i: Floyd / all / with replacement) and neighbour loads are issued as Q
+// independent batches, so each thread keeps Q dependent chains in flight instead of one.
+template <int G, int Q>
 __global__ void __launch_bounds__(256) hop_sample_kernel(HopArgs a) {
     const int64_t F = a.counts[a.h];
     const uint64_t seed = a.call[0];
@@ -132,41 +156,68 @@ __global__ void __launch_bounds__(256) hop_sample_kernel(HopArgs a) {
     const int lane = grp.thread_rank();
     const int k = a.k;
     const int64_t groups = (int64_t)gridDim.x * (256 / G);
-    for (int64_t idx = (int64_t)blockIdx.x * (256 / G) + threadIdx.x / G; idx < F; idx += groups) {
-        const int64_t v = a.nodes[idx];
-        const int64_t lo = __ldg(a.indptr + v);
-        const int32_t d = (int32_t)(__ldg(a.indptr + v + 1) - lo);
-        int32_t* out = a.pad + idx * k;
-        const int32_t c = a.replace ? (d > 0 ? k : 0) : min(d, k);
-        if (lane == 0) a.cnt[idx] = c;
-        if (d <= 0) continue;
-        if (a.replace) {  // k draws, draw order
-            for (int i = lane; i < k; i += G) {
-                const int32_t u = __ldg(a.indices + lo + dev::uniform(dev::draw(seed, v, a.h, i), (uint32_t)d));
-                out[i] = u;
-                mark_new(a.newbits, u);
-            }
-        } else if (d <= k) {  // all neighbours, CSR order, no draws
-            for (int p = lane; p < d; p += G) {
-                const int32_t u = __ldg(a.indices + lo + p);
-                out[p] = u;
-                mark_new(a.newbits, u);
-            }
-        } else if (k <= G) {  // Floyd, one choice per lane; rank = position in sorted order
-            const int32_t ch = floyd_choice<G>(grp, seed, v, a.h, d, k);
-            int r = 0;
+    for (int64_t base = ((int64_t)blockIdx.x * (256 / G) + threadIdx.x / G) * Q; base < F; base += groups * Q) {
+        int64_t v[Q], lo[Q];
+        int32_t d[Q], pos[Q], rnk[Q], u[Q];
 #pragma unroll
-            for (int l = 0; l < G; l++) {
-                const int32_t cl = grp.shfl(ch, l);
-                r += (l < k) && cl < ch;
+        for (int q = 0; q < Q; q++) v[q] = base + q < F ? a.nodes[base + q] : -1;
+#pragma unroll
+        for (int q = 0; q < Q; q++) {
+            lo[q] = 0;
+            d[q] = 0;
+            if (v[q] >= 0) {
+                lo[q] = __ldg(a.indptr + v[q]);
+                d[q] = (int32_t)(__ldg(a.indptr + v[q] + 1) - lo[q]);
             }
-            if (lane < k) {
-                const int32_t u = __ldg(a.indices + lo + ch);
-                out[r] = u;
-                mark_new(a.newbits, u);
+        }
+#pragma unroll
+        for (int q = 0; q < Q; q++) {
+            pos[q] = -1;
+            rnk[q] = 0;
+            const int32_t dq = d[q];
+            if (dq <= 0 || k > G) continue;  // uniform per group
+            if (a.replace) {
+                if (lane < k) {
+                    pos[q] = (int32_t)dev::uniform(dev::draw(seed, v[q], a.h, lane), (uint32_t)dq);
+                    rnk[q] = lane;
+                }
+            } else if (dq <= k) {
+                if (lane < dq) {
+                    pos[q] = lane;
+                    rnk[q] = lane;
+                }
+            } else {
+                const int32_t ch = floyd_choice<G>(grp, seed, v[q], a.h, dq, k);
+                int r = 0;
+#pragma unroll
+                for (int l = 0; l < G; l++) {
+                    const int32_t cl = grp.shfl(ch, l);
+                    r += (l < k) && cl < ch;
+                }
+                if (lane < k) {
+                    pos[q] = ch;
+                    rnk[q] = r;
+                }
             }
-        } else {
-            if constexpr (G == 32) sample_node_wide(grp, a, seed, v, lo, d, out);
+        }
+#pragma unroll
+        for (int q = 0; q < Q; q++) u[q] = pos[q] >= 0 ? __ldg(a.indices + lo[q] + pos[q]) : 0;
+#pragma unroll
+        for (int q = 0; q < Q; q++) {
+            const int64_t idx = base + q;
+            if (idx >= F) break;
+            if (lane == 0) a.cnt[idx] = a.replace ? (d[q] > 0 ? k : 0) : min(d[q], k);
+            if (pos[q] >= 0) {
+                a.pad[idx * k + rnk[q]] = u[q];
+                mark_new(a.newbits, u[q]);
+            }
+        }
+        if (k > G) {
+            for (int q = 0; q < Q; q++) {
+                const int64_t idx = base + q;
+                if (idx >= F) break;
+                if (d[q] > 0) sample_node_slow<G>(grp, a, seed, v[q], lo[q], d[q], a.pad + idx * k);
+            }
         }
     }
 }
@@ -293,12 +344,12 @@ __global__ void __launch_bounds__(kSampleTile) compact_kernel(CompactArgs a) {
         const int64_t prefix = dev::lookback_block<kSampleTile>(a.tile_status, tile, agg, s_red, &s_nearest);
         if (threadIdx.x == 0) {
             if (lt == 0) {
-                dev::st_release(&a.ebase[h], kBaseReady | (uint64_t)prefix);
+                dev::st_flag(&a.ebase[h], kBaseReady | (uint64_t)prefix);
                 s_base = prefix;
             } else {
                 uint64_t b;
                 do {
-                    b = dev::ld_acquire(&a.ebase[h]);
+                    b = dev::ld_flag(&a.ebase[h]);
                 } while (!(b & kBaseReady));
                 s_base = (int64_t)(b & ~kBaseReady);
             }
@@ -312,8 +363,20 @@ __global__ void __launch_bounds__(kSampleTile) compact_kernel(CompactArgs a) {
                 a.offsets[ob + F] = rel + c;
                 a.counts[a.H + 1 + h] = rel + c;
             }
+        }
+        // copy + relabel this node's c edges: up to 16 padded ids and their 16 lidx loads in flight at once
+        if (idx < F) {
             const int32_t* p = a.pad[h] + idx * a.k[h];
-            for (int r = 0; r < c; r++) a.src[gpos + r] = __ldg(a.lidx + __ldg(p + r));
+            for (int r0 = 0; r0 < c; r0 += 16) {
+                int32_t id[16], li[16];
+#pragma unroll
+                for (int r = 0; r < 16; r++) id[r] = r0 + r < c ? __ldg(p + r0 + r) : 0;
+#pragma unroll
+                for (int r = 0; r < 16; r++) li[r] = r0 + r < c ? __ldg(a.lidx + id[r]) : 0;
+#pragma unroll
+                for (int r = 0; r < 16; r++)
+                    if (r0 + r < c) a.src[gpos + r0 + r] = li[r];
+            }
         }
         __syncthreads();
     }
@@ -346,13 +409,36 @@ __global__ void init_kernel(const uint64_t* call, int64_t n_seeds, int64_t n_ver
     if (tid == 0) counts[0] = n_seeds;
 }
 
+template <int G, int Q>
+void launch_sample_hop_q(const HopArgs& a, int64_t max_F, cudaStream_t stream) {
+    const int64_t groups = (max_F + Q - 1) / Q;
+    const int64_t blocks = std::max<int64_t>(1, (groups * G + 255) / 256);
+    hop_sample_kernel<G, Q><<<(int)std::min<int64_t>(blocks, 148 * 16), 256, 0, stream>>>(a);
+}
+
+// Small frontiers keep one node per group (latency: every node in flight at once); large frontiers batch
+// 4 nodes per group (throughput: 4 chains in flight per thread, a quarter of the threads).
 template <int G>
 void launch_sample_hop(const HopArgs& a, int64_t max_F, cudaStream_t stream) {
-    const int64_t blocks = std::max<int64_t>(1, (max_F * G + 255) / 256);
-    hop_sample_kernel<G><<<(int)std::min<int64_t>(blocks, 148 * 16), 256, 0, stream>>>(a);
+    if (max_F >= 65536) launch_sample_hop_q<G, 4>(a, max_F, stream);
+    else launch_sample_hop_q<G, 1>(a, max_F, stream);
 }
 
 }  // namespace
+
+// Same shared-memory carveout for every kernel of the library (see configure_gather_kernels).
+moment_status configure_sample_kernels(int carveout) {
+    if (carveout < 0) return MOMENT_OK;
+    const void* fns[] = {(const void*)init_kernel, (const void*)bitscan_kernel, (const void*)compact_kernel,
+                         (const void*)hop_sample_kernel<4, 1>, (const void*)hop_sample_kernel<8, 1>,
+                         (const void*)hop_sample_kernel<16, 1>, (const void*)hop_sample_kernel<32, 1>,
+                         (const void*)hop_sample_kernel<4, 4>, (const void*)hop_sample_kernel<8, 4>,
+                         (const void*)hop_sample_kernel<16, 4>, (const void*)hop_sample_kernel<32, 4>};
+    for (const void* f : fns)
+        MOMENT_TRY(cuda_check(cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, carveout),
+                              "carveout attribute"));
+    return MOMENT_OK;
+}
 
 // Validates the call on the host; enqueues nothing on error. The seeds pointer and rng_seed are read by
 // the kernels from the device call block `call` ([0] rng_seed, [1] seeds), written beforehand by the
