@@ -274,6 +274,39 @@ moment_status moment_gather_group(moment_ctx_t const* ctxs, int32_t world, const
                                   const int64_t* const* n_dev, int64_t max_n, void* const* out, void* stream);
 
 /* ================================================================================================
+ * H5 exchange for one process per GPU (the all-to-all transport; P:L391-393 relay through a peer).
+ * Per batch, after moment_bucket (route / qoff / qpos of this rank):
+ *   moment_gather_routed  : every row this rank reads itself (local HBM, peer HBM, host bins routed to
+ *                           itself); rows routed through another rank are left untouched.
+ *   moment_relay_pack     : words[2e] = placement word, words[2e+1] = output position of each request routed
+ *                           through another rank, ordered by destination rank then bin (device int64
+ *                           send_counts[world]); words: device uint64 [2 * max_n].
+ *   (caller) all-to-all of the counts, then of the words (2 per request)
+ *   moment_relay_serve    : rows[e] = row named by received placement word e, read by THIS rank from its own
+ *                           mapping of the host bin (its PCIe link); rows: device [n][R]
+ *   (caller) all-to-all of the rows back to the requesters (same splits as the words, in rows)
+ *   moment_relay_scatter  : out[words[2e+1]] = rows[e] on the requester.
+ * n_dev: device count or NULL (= max_n). Byte-exact with moment_gather of the same ids.
+ * ================================================================================================ */
+moment_status moment_gather_routed(moment_ctx_t ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n,
+                                   const int32_t* route, void* out, void* stream);
+moment_status moment_relay_pack(moment_ctx_t ctx, const int64_t* ids, int64_t max_n, const int64_t* qoff,
+                                const int64_t* qpos, uint64_t* words, int64_t* send_counts, void* stream);
+moment_status moment_relay_serve(moment_ctx_t ctx, const uint64_t* words, const int64_t* n_dev, int64_t max_n,
+                                 void* rows, void* stream);
+moment_status moment_relay_scatter(moment_ctx_t ctx, const uint64_t* words, const int64_t* n_dev, int64_t max_n,
+                                   const void* rows, void* out, void* stream);
+
+/* Cross-process device memory (another rank's HBM bin mapped into this process: the NVLink peer
+ * pointer of bin_ptr). export: 64-byte handle of the allocation containing dptr and dptr's byte offset in
+ * it; import: map the allocation (peer access enabled lazily) and return its base (add the offset);
+ * close: unmap (pass the base). */
+#define MOMENT_IPC_HANDLE_BYTES 64
+moment_status moment_ipc_export(const void* dptr, uint8_t* handle, int64_t* offset);
+moment_status moment_ipc_import(const uint8_t* handle, void** dptr);
+moment_status moment_ipc_close(void* dptr);
+
+/* ================================================================================================
  * One whole hot-path step on device buffers: moment_sample of `seeds` followed by moment_gather of F_H
  * into d_rows (NULL: sample only; rows relayed through other ranks are not supported here). The 2H + 3
  * kernels are replayed from a CUDA graph cached in the ctx (captured on the first call of a given shape:

@@ -414,3 +414,73 @@ extern "C" moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* cs
     return cuda_check(cudaMemcpyAsync(counts_host, out->counts, (2 * H + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s),
                       "moment_step_host: D2H");
 }
+
+// ---- H5 exchange for one process per GPU -------------------------------------------------------------
+extern "C" moment_status moment_gather_routed(moment_ctx_t ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n,
+                                              const int32_t* route, void* out, void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_gather_routed"));
+    if (!route || !ctx->placement) return fail(MOMENT_EINVAL, "moment_gather_routed: needs a route and a placement map");
+    return launch_gather(ctx, ids, n_dev, max_n, out, route, ctx->rank, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" moment_status moment_relay_pack(moment_ctx_t ctx, const int64_t* ids, int64_t max_n, const int64_t* qoff,
+                                           const int64_t* qpos, uint64_t* words, int64_t* send_counts, void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_relay_pack"));
+    if (max_n < 0 || (max_n > 0 && (!ids || !qoff || !qpos || !words)) || !send_counts)
+        return fail(MOMENT_EINVAL, "moment_relay_pack: null argument");
+    return launch_relay_pack(ctx, ids, qoff, qpos, max_n, words, send_counts, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" moment_status moment_relay_serve(moment_ctx_t ctx, const uint64_t* words, const int64_t* n_dev, int64_t max_n,
+                                            void* rows, void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_relay_serve"));
+    if (max_n < 0 || (max_n > 0 && (!words || !rows))) return fail(MOMENT_EINVAL, "moment_relay_serve: null argument");
+    if (ctx->n_bins <= 0) return fail(MOMENT_EINVAL, "moment_relay_serve: ctx has no bins");
+    return launch_relay_serve(ctx, words, n_dev, max_n, rows, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" moment_status moment_relay_scatter(moment_ctx_t ctx, const uint64_t* words, const int64_t* n_dev, int64_t max_n,
+                                              const void* rows, void* out, void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_relay_scatter"));
+    if (max_n < 0 || (max_n > 0 && (!words || !rows || !out))) return fail(MOMENT_EINVAL, "moment_relay_scatter: null argument");
+    return launch_relay_scatter(ctx, words, n_dev, max_n, rows, out, static_cast<cudaStream_t>(stream));
+}
+
+// ---- cross-process device memory (peer HBM bins of other ranks) -------------------------------------
+static_assert(sizeof(cudaIpcMemHandle_t) == MOMENT_IPC_HANDLE_BYTES, "IPC handle size");
+
+extern "C" moment_status moment_ipc_export(const void* dptr, uint8_t* handle, int64_t* offset) {
+    if (!dptr || !handle || !offset) return fail(MOMENT_EINVAL, "moment_ipc_export: null argument");
+    // the handle names the whole allocation: report dptr's offset from its base (cuMemGetAddressRange,
+    // resolved from the driver at run time so the library does not link libcuda)
+    using range_fn = int (*)(unsigned long long*, size_t*, unsigned long long);
+    static range_fn get_range = nullptr;
+    if (!get_range) {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        MOMENT_TRY(cuda_check(cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q),
+                              "moment_ipc_export: driver entry point"));
+        if (!fn || q != cudaDriverEntryPointSuccess) return fail(MOMENT_ECUDA, "moment_ipc_export: cuMemGetAddressRange missing");
+        get_range = reinterpret_cast<range_fn>(fn);
+    }
+    unsigned long long base = 0;
+    size_t size = 0;
+    if (get_range(&base, &size, reinterpret_cast<unsigned long long>(dptr)) != 0)
+        return fail(MOMENT_ECUDA, "moment_ipc_export: cuMemGetAddressRange failed");
+    cudaIpcMemHandle_t h;
+    MOMENT_TRY(cuda_check(cudaIpcGetMemHandle(&h, reinterpret_cast<void*>(base)), "moment_ipc_export"));
+    std::memcpy(handle, &h, sizeof(h));
+    *offset = (int64_t)(reinterpret_cast<unsigned long long>(dptr) - base);
+    return MOMENT_OK;
+}
+
+extern "C" moment_status moment_ipc_import(const uint8_t* handle, void** dptr) {
+    if (!dptr || !handle) return fail(MOMENT_EINVAL, "moment_ipc_import: null argument");
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, handle, sizeof(h));
+    return cuda_check(cudaIpcOpenMemHandle(dptr, h, cudaIpcMemLazyEnablePeerAccess), "moment_ipc_import");
+}
+
+extern "C" moment_status moment_ipc_close(void* dptr) {
+    return cuda_check(cudaIpcCloseMemHandle(dptr), "moment_ipc_close");
+}

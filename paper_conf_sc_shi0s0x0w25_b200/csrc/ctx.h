@@ -96,6 +96,12 @@ moment_status launch_relay(moment_ctx_s* server, moment_ctx_s* requester, const 
                            const int64_t* qoff, const int64_t* qpos, void* requester_out, cudaStream_t stream);
 moment_status launch_hotness(const int64_t* ids, const int64_t* n_dev, int64_t max_n, uint64_t* hot,
                              cudaStream_t stream);
+moment_status launch_relay_pack(moment_ctx_s* ctx, const int64_t* ids, const int64_t* qoff, const int64_t* qpos,
+                                int64_t max_n, uint64_t* words, int64_t* counts, cudaStream_t stream);
+moment_status launch_relay_serve(moment_ctx_s* ctx, const uint64_t* words, const int64_t* n_dev, int64_t max_n,
+                                 void* rows, cudaStream_t stream);
+moment_status launch_relay_scatter(moment_ctx_s* ctx, const uint64_t* words, const int64_t* n_dev, int64_t max_n,
+                                   const void* rows, void* out, cudaStream_t stream);
 moment_status configure_sample_kernels(int carveout);
 moment_status configure_gather_kernels(int carveout);
 

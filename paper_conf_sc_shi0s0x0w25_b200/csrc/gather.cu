@@ -458,6 +458,124 @@ moment_status launch_relay(moment_ctx_s* server, moment_ctx_s* requester, const 
     return cuda_check(cudaGetLastError(), "moment_gather: relay launch");
 }
 
+// ---- H5 exchange for one process per GPU (all-to-all transport) ---------------------------------------
+namespace {
+
+constexpr int kMaxSegs = 128;  // (destination rank, host bin) segments
+
+// Segments of this rank's relay queues in send order (destination h ascending, then host bin b):
+// q = b * world + h for h != self and host bins b. Computed redundantly by every block (<= 128 entries).
+__device__ int build_segments(const int64_t* qoff, const BinTable& bins, int n_bins, int world, int self,
+                              int64_t* seg_src, int64_t* seg_dst, int* seg_h) {
+    int n = 0;
+    int64_t dst = 0;
+    for (int h = 0; h < world; h++) {
+        if (h == self) continue;
+        for (int b = 0; b < n_bins; b++) {
+            if (bins.owner[b] >= 0) continue;
+            const int q = b * world + h;
+            seg_src[n] = qoff[q];
+            seg_dst[n] = dst;
+            seg_h[n] = h;
+            dst += qoff[q + 1] - qoff[q];
+            n++;
+        }
+    }
+    seg_dst[n] = dst;
+    return n;
+}
+
+// words[2e] = placement word of the row, words[2e+1] = its position in this rank's output; counts[h] =
+// entries for destination h (0 for self).
+__global__ void relay_pack_kernel(BinTable bins, const uint64_t* __restrict__ placement, const int64_t* __restrict__ ids,
+                                  const int64_t* __restrict__ qoff, const int64_t* __restrict__ qpos, int32_t n_bins,
+                                  int32_t world, int32_t self, uint64_t* __restrict__ words, int64_t* counts) {
+    __shared__ int64_t s_src[kMaxSegs + 1], s_dst[kMaxSegs + 1];
+    __shared__ int s_h[kMaxSegs + 1];
+    __shared__ int s_n;
+    if (threadIdx.x == 0) s_n = build_segments(qoff, bins, n_bins, world, self, s_src, s_dst, s_h);
+    __syncthreads();
+    const int ns = s_n;
+    if (blockIdx.x == 0 && threadIdx.x < world) {
+        int64_t c = 0;
+        for (int s = 0; s < ns; s++)
+            if (s_h[s] == (int)threadIdx.x) c += s_dst[s + 1] - s_dst[s];
+        counts[threadIdx.x] = c;
+    }
+    const int64_t total = s_dst[ns];
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+        int lo = 0, hi = ns - 1;
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (s_dst[mid] <= e) lo = mid;
+            else hi = mid - 1;
+        }
+        const int64_t i = __ldg(qpos + s_src[lo] + (e - s_dst[lo]));
+        words[2 * e] = __ldg(placement + __ldg(ids + i));
+        words[2 * e + 1] = (uint64_t)i;
+    }
+}
+
+// rows[e] = the row named by placement word words[2e], read by THIS rank (its host-bin mapping).
+__global__ void __launch_bounds__(kGatherThreads) relay_serve_kernel(BinTable bins, const uint64_t* __restrict__ words,
+                                                                     const int64_t* n_dev, int64_t max_n, FastDiv rv,
+                                                                     int64_t stride_vec, int4* __restrict__ rows) {
+    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+    const uint32_t total = (uint32_t)(n * rv.d);
+    for (uint32_t v = blockIdx.x * kGatherThreads + threadIdx.x; v < total; v += gridDim.x * kGatherThreads) {
+        const uint32_t e = fdiv(v, rv), col = v - e * rv.d;
+        const uint64_t p = __ldg(words + 2 * (int64_t)e);
+        rows[v] = ld_stream(bins.base[(int)(p >> 40)] + (int64_t)(p & kSlotMask) * stride_vec + col);
+    }
+}
+
+// out[words[2e+1]] = rows[e].
+__global__ void __launch_bounds__(kGatherThreads) relay_scatter_kernel(const uint64_t* __restrict__ words,
+                                                                       const int64_t* n_dev, int64_t max_n, FastDiv rv,
+                                                                       const int4* __restrict__ rows,
+                                                                       int4* __restrict__ out) {
+    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+    const uint32_t total = (uint32_t)(n * rv.d);
+    for (uint32_t v = blockIdx.x * kGatherThreads + threadIdx.x; v < total; v += gridDim.x * kGatherThreads) {
+        const uint32_t e = fdiv(v, rv), col = v - e * rv.d;
+        out[(int64_t)__ldg(words + 2 * (int64_t)e + 1) * rv.d + col] = ld_stream(rows + v);
+    }
+}
+
+}  // namespace
+
+moment_status launch_relay_pack(moment_ctx_s* ctx, const int64_t* ids, const int64_t* qoff, const int64_t* qpos,
+                                int64_t max_n, uint64_t* words, int64_t* counts, cudaStream_t stream) {
+    if (!ctx->placement) return fail(MOMENT_EINVAL, "moment_relay_pack: ctx has no placement map");
+    if (ctx->n_bins * (ctx->world - 1) > kMaxSegs) return fail(MOMENT_EUNSUPPORTED, "moment_relay_pack: too many segments");
+    const int grid = grid_for(std::max<int64_t>(max_n, 1), 256, 148 * 4);
+    relay_pack_kernel<<<grid, 256, 0, stream>>>(make_bins(ctx), ctx->placement, ids, qoff, qpos, ctx->n_bins, ctx->world,
+                                                ctx->rank, words, counts);
+    return cuda_check(cudaGetLastError(), "moment_relay_pack: launch");
+}
+
+moment_status launch_relay_serve(moment_ctx_s* ctx, const uint64_t* words, const int64_t* n_dev, int64_t max_n,
+                                 void* rows, cudaStream_t stream) {
+    const int64_t rv = ctx->row_bytes / 16;
+    if (max_n * rv >= (int64_t(1) << 32)) return fail(MOMENT_EUNSUPPORTED, "moment_relay_serve: too many rows");
+    if (max_n == 0) return MOMENT_OK;
+    relay_serve_kernel<<<grid_for(max_n * rv, kGatherThreads, 148 * 8), kGatherThreads, 0, stream>>>(
+        make_bins(ctx), words, n_dev, max_n, make_fastdiv((uint32_t)rv), ctx->row_stride / 16,
+        reinterpret_cast<int4*>(rows));
+    return cuda_check(cudaGetLastError(), "moment_relay_serve: launch");
+}
+
+moment_status launch_relay_scatter(moment_ctx_s* ctx, const uint64_t* words, const int64_t* n_dev, int64_t max_n,
+                                   const void* rows, void* out, cudaStream_t stream) {
+    const int64_t rv = ctx->row_bytes / 16;
+    if (max_n * rv >= (int64_t(1) << 32)) return fail(MOMENT_EUNSUPPORTED, "moment_relay_scatter: too many rows");
+    if (max_n == 0) return MOMENT_OK;
+    relay_scatter_kernel<<<grid_for(max_n * rv, kGatherThreads, 148 * 8), kGatherThreads, 0, stream>>>(
+        words, n_dev, max_n, make_fastdiv((uint32_t)rv), reinterpret_cast<const int4*>(rows),
+        reinterpret_cast<int4*>(out));
+    return cuda_check(cudaGetLastError(), "moment_relay_scatter: launch");
+}
+
 // Kernel attributes, set once per device: every kernel of the library asks for the same shared-memory
 // carveout (so consecutive kernels never force an L1/shared reconfiguration bubble on the SMs), and the
 // bulk gather may use up to kBulkStages x kBulkStageBudget bytes of dynamic shared memory.

@@ -1,0 +1,92 @@
+"""H5 exchange for one process per GPU: the per-batch relay of host rows through peer ranks.
+
+Orchestration only (torch.distributed is the transport, every byte is computed by libmoment.so kernels):
+
+  moment_bucket          routes (local / peer HBM / host direct / host via relay rank h), stable queues
+  moment_gather_routed   every row this rank reads itself (overlaps the exchange below)
+  moment_relay_pack      (placement word, output position) of each request routed through another rank
+  all-to-all             counts, then request words (2 x int64 per request)
+  moment_relay_serve     the relay rank reads the requested host rows over ITS PCIe link
+  all-to-all             rows back to the requesters (same splits, in rows)
+  moment_relay_scatter   rows into the requester's output positions
+
+With NCCL the collectives run on the GPU stream; with gloo (CPU tests, or several processes sharing one
+GPU) they are staged through host memory. `alltoallv` is the transport helper both use.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+
+import torch
+import torch.distributed as dist
+
+
+def _is_gloo(group) -> bool:
+    return dist.get_backend(group) == "gloo"
+
+
+def alltoallv(send: torch.Tensor, send_splits: list[int], recv_splits: list[int], group=None) -> torch.Tensor:
+    """Variable-size all-to-all of the leading dimension. Returns a tensor of sum(recv_splits) rows on
+    send's device (staged through host memory for gloo)."""
+    out_shape = (sum(recv_splits),) + tuple(send.shape[1:])
+    if _is_gloo(group) and send.is_cuda:
+        recv = torch.empty(out_shape, dtype=send.dtype)
+        dist.all_to_all_single(recv, send.cpu().contiguous(), recv_splits, send_splits, group=group)
+        return recv.to(send.device, non_blocking=False)
+    recv = torch.empty(out_shape, dtype=send.dtype, device=send.device)
+    dist.all_to_all_single(recv, send.contiguous(), recv_splits, send_splits, group=group)
+    return recv
+
+
+def exchange_counts(send_counts: torch.Tensor, group=None) -> list[int]:
+    """Each rank's number of requests for every other rank -> how many this rank will serve from each."""
+    world = dist.get_world_size(group)
+    send = send_counts.to(torch.int64).reshape(world)
+    recv = alltoallv(send.reshape(world, 1), [1] * world, [1] * world, group)
+    return [int(x) for x in recv.reshape(world).cpu()]
+
+
+@dataclass
+class ExchangeBuffers:
+    """Device buffers of one rank's exchange, sized once for max_n requests (receive buffers grow)."""
+
+    max_n: int
+    row_bytes: int
+    n_queues: int
+    device: torch.device
+    route: torch.Tensor = field(init=False)
+    qoff: torch.Tensor = field(init=False)
+    qpos: torch.Tensor = field(init=False)
+    words: torch.Tensor = field(init=False)
+    send_counts: torch.Tensor = field(init=False)
+
+    def __post_init__(self):
+        d = self.device
+        self.route = torch.empty(max(self.max_n, 1), dtype=torch.int32, device=d)
+        self.qoff = torch.empty(self.n_queues + 1, dtype=torch.int64, device=d)
+        self.qpos = torch.empty(max(self.max_n, 1), dtype=torch.int64, device=d)
+        self.words = torch.empty(2 * max(self.max_n, 1), dtype=torch.int64, device=d)
+        self.send_counts = torch.zeros(64, dtype=torch.int64, device=d)
+
+
+def gather_exchange(ctx, ids: torch.Tensor, out: torch.Tensor, bufs: ExchangeBuffers, *, n: int, group=None,
+                    stream=None) -> dict:
+    """Collective: out[:n] = rows of ids[:n] for every rank of `group` (ctx.rank == group rank).
+    Returns the per-batch traffic (requests sent to / served for each rank)."""
+    world = ctx.world
+    s = stream if stream is not None else torch.cuda.current_stream(ids.device)
+    with torch.cuda.stream(s):
+        ctx.bucket(ids, bufs.route, bufs.qoff, bufs.qpos, max_n=n, stream=s)
+        ctx.gather_routed(ids, bufs.route, out, max_n=n, stream=s)
+        ctx.relay_pack(ids, bufs.qoff, bufs.qpos, bufs.words, bufs.send_counts, max_n=n, stream=s)
+        send = [int(x) for x in bufs.send_counts[:world].cpu()]  # synchronises the stream
+        recv = exchange_counts(torch.tensor(send, dtype=torch.int64), group)
+        n_send, n_recv = sum(send), sum(recv)
+        words_in = alltoallv(bufs.words[: 2 * n_send].view(n_send, 2), send, recv, group).reshape(-1)
+        rows_srv = torch.empty((max(n_recv, 1), ctx.row_bytes), dtype=torch.uint8, device=ids.device)
+        if n_recv:
+            ctx.relay_serve(words_in, rows_srv, n=n_recv, stream=s)
+        rows_back = alltoallv(rows_srv[:n_recv], recv, send, group)
+        if n_send:
+            ctx.relay_scatter(bufs.words, rows_back, out, n=n_send, stream=s)
+    return {"sent": send, "served": recv}

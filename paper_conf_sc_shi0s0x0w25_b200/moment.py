@@ -28,7 +28,8 @@ EXPORTED = [
     "moment_topology_free", "moment_maxflow", "moment_place", "moment_place_pack", "moment_plan", "moment_plan_info",
     "moment_plan_free", "moment_ctx_create", "moment_ctx_free", "moment_ctx_workspace_bytes", "moment_sample_bounds",
     "moment_sample", "moment_sample_check", "moment_hotness", "moment_bucket", "moment_gather", "moment_gather_group",
-    "moment_step", "moment_step_host",
+    "moment_step", "moment_step_host", "moment_gather_routed", "moment_relay_pack", "moment_relay_serve",
+    "moment_relay_scatter", "moment_ipc_export", "moment_ipc_import", "moment_ipc_close",
 ]
 
 
@@ -119,6 +120,13 @@ def lib():
             "moment_gather_group": ([P, I32, P, P, I64, P, P], I32),
             "moment_step": ([P, P, P, I64, P, P, P, P], I32),
             "moment_step_host": ([P, P, P, I64, P, P, P, P, P], I32),
+            "moment_gather_routed": ([P, P, P, I64, P, P, P], I32),
+            "moment_relay_pack": ([P, P, I64, P, P, P, P, P], I32),
+            "moment_relay_serve": ([P, P, P, I64, P, P], I32),
+            "moment_relay_scatter": ([P, P, P, I64, P, P, P], I32),
+            "moment_ipc_export": ([P, P, P], I32),
+            "moment_ipc_import": ([P, P], I32),
+            "moment_ipc_close": ([P], I32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -408,6 +416,48 @@ class Ctx:
         a[1].rng_seed = rng_seed & 0xFFFFFFFFFFFFFFFF
         _check(lib().moment_step_host(self.handle, a[4], seeds_host.data_ptr(), seeds_host.numel(), a[5], a[6],
                                       _ptr(rows), counts_host.data_ptr(), _stream(stream)))
+
+
+    # ---- H5 exchange for one process per GPU (see exchange.py for the orchestration) ----
+    def gather_routed(self, ids, route, out, *, n_dev=None, max_n: int | None = None, stream=None):
+        mn = ids.numel() if max_n is None else max_n
+        _check(lib().moment_gather_routed(self.handle, ids.data_ptr(), _ptr(n_dev), mn, route.data_ptr(),
+                                          out.data_ptr(), _stream(stream)))
+
+    def relay_pack(self, ids, qoff, qpos, words, send_counts, *, max_n: int | None = None, stream=None):
+        mn = ids.numel() if max_n is None else max_n
+        _check(lib().moment_relay_pack(self.handle, ids.data_ptr(), mn, qoff.data_ptr(), qpos.data_ptr(),
+                                       words.data_ptr(), send_counts.data_ptr(), _stream(stream)))
+
+    def relay_serve(self, words, rows, *, n: int, stream=None):
+        _check(lib().moment_relay_serve(self.handle, words.data_ptr(), None, n, rows.data_ptr(), _stream(stream)))
+
+    def relay_scatter(self, words, rows, out, *, n: int, stream=None):
+        _check(lib().moment_relay_scatter(self.handle, words.data_ptr(), None, n, rows.data_ptr(), out.data_ptr(),
+                                          _stream(stream)))
+
+
+IPC_HANDLE_BYTES = 64
+
+
+def ipc_export(tensor) -> tuple[bytes, int]:
+    """(64-byte CUDA IPC handle of the allocation holding `tensor`, byte offset of the tensor in it)."""
+    h = (C.c_uint8 * IPC_HANDLE_BYTES)()
+    off = C.c_int64()
+    _check(lib().moment_ipc_export(tensor.data_ptr(), C.cast(h, P), C.byref(off)))
+    return bytes(h), off.value
+
+
+def ipc_import(handle: bytes) -> int:
+    """Map another process's device allocation into this one; returns its base address (add the offset)."""
+    h = (C.c_uint8 * IPC_HANDLE_BYTES).from_buffer_copy(handle)
+    ptr = C.c_void_p()
+    _check(lib().moment_ipc_import(C.cast(h, P), C.byref(ptr)))
+    return ptr.value
+
+
+def ipc_close(ptr: int):
+    _check(lib().moment_ipc_close(ptr))
 
 
 def gather_group(ctxs, ids, out, *, n_dev=None, max_n: int, stream=None):

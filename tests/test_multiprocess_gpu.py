@@ -1,0 +1,93 @@
+"""One process per rank on the GPU path (H4-H7 with the all-to-all transport), 2 processes sharing cuda:0.
+
+Each rank owns one HBM bin (its feature rows by the DDAK placement); the other rank's bin is mapped
+through CUDA IPC (moment_ipc_export / import — the peer-load pointer of the NVLink path); both host bins
+are pinned host memory; the quota relays part of every rank's host rows through the other rank. Each rank
+samples its own seeds and runs exchange.gather_exchange (bucket -> routed gather -> relay pack ->
+all-to-all -> relay serve -> all-to-all -> scatter) over a gloo group; the rows must equal the oracle's
+table[ids] byte for byte.
+"""
+import numpy as np
+import pytest
+import torch
+
+from mp_util import run_world
+
+pytestmark = pytest.mark.gpu
+
+
+def _rank_main(rank, world):
+    import torch.distributed as dist
+
+    import oracle
+    import paper_conf_sc_shi0s0x0w25_b200 as M
+    import workloads as W
+    from paper_conf_sc_shi0s0x0w25_b200.exchange import ExchangeBuffers, gather_exchange
+
+    oracle.build()
+    torch.cuda.set_device(0)
+    dev = "cuda:0"
+    cfg = W.CONFIGS["C1"]
+    g = W.rmat_csr(cfg["n"], cfg["m"], device=dev)
+    n = g.n
+    table = W.feature_table(n, 32, torch.float32, device="cpu")  # 128-byte rows
+    R = table.shape[1]
+    rng = np.random.default_rng(7)  # identical on every rank: one global placement
+    hot = rng.pareto(1.0, n).astype(np.uint64)
+    owners = list(range(world)) + [-1, -1]
+    tiers = [M.TIER_GPU_HBM] * world + [M.TIER_HOST_DRAM] * 2
+    caps = [n // (4 * world)] * world + [n // 2, n]
+    bin_of, slot_of, *_ = M.place(None, hot, caps, bin_tier=tiers, bin_traffic=[100] * world + [10, 10])
+    bins = []
+    for b in range(world + 2):
+        sel = np.nonzero(bin_of == b)[0]
+        buf = torch.zeros((max(1, int(slot_of[sel].max()) + 1 if len(sel) else 1), R), dtype=torch.uint8)
+        buf[torch.as_tensor(slot_of[sel])] = table[torch.as_tensor(sel)]
+        bins.append(buf)
+    mine = bins[rank].to(dev)  # this rank's HBM bin
+    handle, off = M.ipc_export(mine)
+    shared = [None] * world
+    dist.all_gather_object(shared, (handle, off))
+    imported = {}
+    ptrs = []
+    for b in range(world):
+        if b == rank:
+            ptrs.append(mine.data_ptr())
+        else:
+            base = M.ipc_import(shared[b][0])
+            imported[b] = base
+            ptrs.append(base + shared[b][1])
+    host = [bins[world].pin_memory(), bins[world + 1].pin_memory()]
+    ptrs += [h.data_ptr() for h in host]
+    placement = torch.as_tensor(M.place_pack(bin_of, slot_of).view(np.int64), device=dev)
+    quota = np.zeros((world + 2, world), np.int64)
+    quota[world] = [3, 2] if world == 2 else np.arange(1, world + 1)
+    quota[world + 1] = [1, 4] if world == 2 else np.arange(world, 0, -1)
+    ctx = M.Ctx(n_vertices=n, max_seeds=512, max_fanout=[10, 5], rank=rank, world=world, device=0, row_bytes=R,
+                bin_owner=owners, bin_ptr=ptrs, placement=placement, quota=quota)
+    train = W.training_set(g, min_count=512 * world)
+    seeds = W.epoch_batches(train, 512, 0, rank=rank, world=world)[0]
+    bufs = M.SampleBuffers.allocate(512, [10, 5], n, dev)
+    ctx.sample(g.indptr, g.indices, seeds, [10, 5], 900 + rank, bufs)
+    torch.cuda.synchronize()
+    nF = int(bufs.counts[2])
+    ids = bufs.nodes[:nF].contiguous()
+    out = torch.zeros((nF, R), dtype=torch.uint8, device=dev)
+    xb = ExchangeBuffers(max_n=nF, row_bytes=R, n_queues=(world + 2) * world, device=torch.device(dev))
+    info = gather_exchange(ctx, ids, out, xb, n=nF)
+    torch.cuda.synchronize()
+    ok = bool(np.array_equal(out.cpu().numpy(), oracle.gather(table.numpy(), ids.cpu().numpy())))
+    dist.barrier()  # every rank done with the others' bins before any mapping goes away
+    for base in imported.values():
+        M.ipc_close(base)
+    dist.barrier()
+    return {"ok": ok, "sent": info["sent"], "served": info["served"], "nF": nF}
+
+
+def test_gather_exchange_two_processes_one_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    res = run_world(_rank_main, 2)
+    assert all(r["ok"] for r in res), res
+    assert res[0]["sent"][1] == res[1]["served"][0] and res[1]["sent"][0] == res[0]["served"][1]
+    assert res[0]["sent"][1] > 0 and res[1]["sent"][0] > 0
