@@ -2,6 +2,7 @@
 // points of include/moment.h: moment_sample, moment_gather, moment_gather_group, moment_bucket,
 // moment_hotness, moment_step_host.
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <string>
 #include <cstring>
@@ -96,6 +97,16 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     if (const char* gp = std::getenv("MOMENT_GATHER_PATH")) {
         const std::string v(gp);
         c->gather_path = v == "ldg" ? 1 : (v == "bulk" ? 2 : 0);
+    }
+    if (const char* v = std::getenv("MOMENT_BULK"))
+        std::sscanf(v, "%d,%d,%d", &c->bulk_stages, &c->bulk_blocks_per_sm, &c->bulk_stage_kb);
+    if (const char* v = std::getenv("MOMENT_HOP_GRID")) c->hop_grid_per_sm = std::max(1, std::atoi(v));
+    if (const char* v = std::getenv("MOMENT_COMPACT_GRID")) c->compact_grid_per_sm = std::max(1, std::atoi(v));
+    if (const char* l2 = std::getenv("MOMENT_GATHER_L2")) {  // "<load><store>" digits, e.g. "01"
+        if (std::strlen(l2) == 2) {
+            c->l2_load_policy = l2[0] - '0';
+            c->l2_store_policy = l2[1] - '0';
+        }
     }
     if (a->quota) c->quota.assign(a->quota, a->quota + (size_t)a->n_bins * a->world);
     // bounds per hop

@@ -20,6 +20,9 @@ struct moment_ctx_s {
     int64_t row_bytes = 0, row_stride = 0;
     int32_t n_bins = 0;
     int32_t gather_path = 0;  // 0 auto (TMA bulk copies for local rows), 1 LDG.128 only, 2 bulk (MOMENT_GATHER_PATH)
+    int32_t l2_load_policy = 0, l2_store_policy = 1;  // bulk gather L2 hints: 0 normal, 1 evict_first, 2 evict_last
+    int32_t hop_grid_per_sm = 4, compact_grid_per_sm = 1;  // launch caps (MOMENT_HOP_GRID / MOMENT_COMPACT_GRID)
+    int32_t bulk_stages = 4, bulk_blocks_per_sm = 4, bulk_stage_kb = 14;  // bulk gather shape (MOMENT_BULK="S,B,KB")
     std::vector<int32_t> bin_owner;
     std::vector<void*> bin_ptr;
     const uint64_t* placement = nullptr;

@@ -89,9 +89,7 @@ __global__ void __launch_bounds__(kGatherThreads) gather_kernel(BinTable bins, c
 // tiles are in flight per block, so an SM keeps kStages x blocks x 32 rows of reads outstanding with a
 // handful of instructions per row.
 constexpr int kBulkMaxRows = 32;
-constexpr int kBulkStageBudget = 14 * 1024;  // bytes per stage: 4 stages x 4 blocks per SM fit in smem
-constexpr int kBulkStages = 4;
-constexpr int kBulkBlocksPerSM = 4;
+constexpr int kBulkSmemMax = 200 * 1024;  // dynamic shared memory a bulk-gather block may request
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -113,15 +111,25 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "r"(parity)
         : "memory");
 }
-__device__ __forceinline__ void bulk_load(void* dst_smem, const void* src, uint32_t bytes, uint64_t* bar) {
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                     smem_u32(dst_smem)),
-                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
-                 : "memory");
+// L2 policies for the bulk copies: the gathered batch streams through L2 (evict_first) so it does not
+// push the sampler's working set (CSR of hot vertices, bitmaps, lidx) out between batches.
+__device__ __forceinline__ uint64_t l2_policy(int kind) {
+    uint64_t p;
+    if (kind == 1) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    else if (kind == 2) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    else asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+    return p;
 }
-__device__ __forceinline__ void bulk_store(void* dst, const void* src_smem, uint32_t bytes) {
-    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src_smem)),
-                 "r"(bytes)
+__device__ __forceinline__ void bulk_load(void* dst_smem, const void* src, uint32_t bytes, uint64_t* bar, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+            smem_u32(dst_smem)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+        : "memory");
+}
+__device__ __forceinline__ void bulk_store(void* dst, const void* src_smem, uint32_t bytes, uint64_t pol) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;" ::"l"(dst),
+                 "r"(smem_u32(src_smem)), "r"(bytes), "l"(pol)
                  : "memory");
     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
@@ -141,13 +149,16 @@ __device__ __forceinline__ const char* row_src(const BinTable& bins, const uint6
     return reinterpret_cast<const char*>(bins.base[0]) + id * stride;
 }
 
+template <int kBulkStages>
 __global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const uint64_t* __restrict__ placement,
                                                          const int64_t* __restrict__ ids, const int64_t* n_dev,
                                                          int64_t max_n, uint32_t R, int64_t stride,
-                                                         int rows_per_tile, char* __restrict__ out) {
+                                                         int rows_per_tile, int l2_load, int l2_store,
+                                                         char* __restrict__ out) {
     extern __shared__ __align__(128) char stage[];  // kBulkStages * rows_per_tile * R
     __shared__ __align__(8) uint64_t full[kBulkStages];
     const int lane = threadIdx.x;
+    const uint64_t pol_ld = l2_policy(l2_load), pol_st = l2_policy(l2_store);
     const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
     const int64_t n_tiles = (n + rows_per_tile - 1) / rows_per_tile;
     if (lane == 0)
@@ -155,19 +166,29 @@ __global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const ui
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     __syncwarp();
     const int64_t t0 = blockIdx.x, dt = gridDim.x;
-    auto issue = [&](int64_t tile, int s) {
+    // the row id of this lane in `tile` (loaded ahead of time: an id load never sits on the issue path)
+    auto load_id = [&](int64_t tile) -> int64_t {
+        const int64_t r = tile * rows_per_tile + lane;
+        return (tile < n_tiles && lane < rows_per_tile && r < n) ? __ldg(ids + r) : -1;
+    };
+    auto issue = [&](int64_t tile, int s, int64_t id) {
         const int64_t row0 = tile * rows_per_tile;
         const int rows = (int)min((int64_t)rows_per_tile, n - row0);
         if (lane == 0) mbar_expect_tx(&full[s], (uint32_t)rows * R);
         __syncwarp();
-        if (lane < rows) {
-            const char* src = row_src(bins, placement, __ldg(ids + row0 + lane), stride);
-            bulk_load(stage + ((size_t)s * rows_per_tile + lane) * R, src, R, &full[s]);
-        }
+        if (lane < rows)
+            bulk_load(stage + ((size_t)s * rows_per_tile + lane) * R, row_src(bins, placement, id, stride), R, &full[s],
+                      pol_ld);
     };
-    // prologue: fill the pipeline
+    // prologue: all ids of the first kBulkStages tiles in flight together, then fill the pipeline
+    int64_t pre[kBulkStages];
+#pragma unroll
+    for (int s = 0; s < kBulkStages; s++) pre[s] = load_id(t0 + s * dt);
     int64_t next = t0;
-    for (int s = 0; s < kBulkStages && next < n_tiles; s++, next += dt) issue(next, s);
+#pragma unroll
+    for (int s = 0; s < kBulkStages; s++, next += dt)
+        if (next < n_tiles) issue(next, s, pre[s]);
+    int64_t next_id = load_id(next);
     // steady state: store the tile that landed, then refill the stage of the PREVIOUS tile, whose store
     // was issued one iteration ago (wait_group.read 1: every store but the newest has read its stage).
     int it = 0;
@@ -177,13 +198,14 @@ __global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const ui
         const int64_t row0 = tile * rows_per_tile;
         const int rows = (int)min((int64_t)rows_per_tile, n - row0);
         if (lane == 0) {
-            bulk_store(out + row0 * (int64_t)R, stage + (size_t)s * rows_per_tile * R, (uint32_t)rows * R);
+            bulk_store(out + row0 * (int64_t)R, stage + (size_t)s * rows_per_tile * R, (uint32_t)rows * R, pol_st);
             if (it > 0) bulk_wait_read<1>();
         }
         __syncwarp();
         if (it > 0 && next < n_tiles) {
-            issue(next, (it - 1) % kBulkStages);
+            issue(next, (it - 1) % kBulkStages, next_id);
             next += dt;
+            next_id = load_id(next);
         }
     }
     if (lane == 0) bulk_wait_all();
@@ -408,13 +430,23 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
     for (int b = 0; b < ctx->n_bins; b++) all_local &= ctx->bin_owner[b] == ctx->rank;
     const bool bulk = ctx->gather_path == 2 || (ctx->gather_path == 0 && route == nullptr && all_local);
     if (bulk && route == nullptr) {
-        const int rows = (int)std::max<int64_t>(1, std::min<int64_t>(kBulkMaxRows, kBulkStageBudget / ctx->row_bytes));
-        const size_t smem = (size_t)kBulkStages * rows * ctx->row_bytes;
+        // tiles of <= 32 rows, `stages` tiles in flight per 1-warp block, `bps` blocks per SM, each stage at
+        // most `stage_kb` KB (defaults 4 / 4 / 14: 4 x 4 x 14 KB fits the SM's shared memory)
+        const int stages = ctx->bulk_stages, bps = ctx->bulk_blocks_per_sm;
+        const int rows = (int)std::max<int64_t>(1, std::min<int64_t>(kBulkMaxRows, ctx->bulk_stage_kb * 1024 / ctx->row_bytes));
+        const size_t smem = (size_t)stages * rows * ctx->row_bytes;
+        if (smem > (size_t)kBulkSmemMax) return fail(MOMENT_EINVAL, "moment_gather: bulk stage config needs %zu B smem", smem);
         const int64_t tiles = (max_n + rows - 1) / rows;
-        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, 148 * kBulkBlocksPerSM));
-        gather_bulk_kernel<<<grid, 32, smem, stream>>>(make_bins(ctx), ctx->placement, ids, n_dev, max_n,
-                                                       (uint32_t)ctx->row_bytes, ctx->row_stride, rows,
-                                                       reinterpret_cast<char*>(out));
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)148 * bps));
+        auto launch = [&](auto kern) {
+            kern<<<grid, 32, smem, stream>>>(make_bins(ctx), ctx->placement, ids, n_dev, max_n, (uint32_t)ctx->row_bytes,
+                                             ctx->row_stride, rows, ctx->l2_load_policy, ctx->l2_store_policy,
+                                             reinterpret_cast<char*>(out));
+        };
+        if (stages <= 2) launch(gather_bulk_kernel<2>);
+        else if (stages <= 4) launch(gather_bulk_kernel<4>);
+        else if (stages <= 6) launch(gather_bulk_kernel<6>);
+        else launch(gather_bulk_kernel<8>);
     } else {
         const int grid = grid_for(max_n * rv, kGatherThreads * kGatherUnroll, 148 * 8);
         gather_kernel<<<grid, kGatherThreads, 0, stream>>>(make_bins(ctx), ctx->placement, ids, n_dev, max_n,
@@ -578,9 +610,10 @@ moment_status launch_relay_scatter(moment_ctx_s* ctx, const uint64_t* words, con
 
 // Kernel attributes, set once per device: every kernel of the library asks for the same shared-memory
 // carveout (so consecutive kernels never force an L1/shared reconfiguration bubble on the SMs), and the
-// bulk gather may use up to kBulkStages x kBulkStageBudget bytes of dynamic shared memory.
+// bulk gather may use up to kBulkSmemMax bytes of dynamic shared memory.
 moment_status configure_gather_kernels(int carveout) {
-    const void* fns[] = {(const void*)gather_kernel, (const void*)gather_bulk_kernel, (const void*)relay_kernel,
+    const void* fns[] = {(const void*)gather_kernel, (const void*)gather_bulk_kernel<2>, (const void*)gather_bulk_kernel<4>,
+                         (const void*)gather_bulk_kernel<6>, (const void*)gather_bulk_kernel<8>, (const void*)relay_kernel,
                          (const void*)bucket_count_kernel, (const void*)bucket_scan_kernel,
                          (const void*)bucket_route_kernel, (const void*)queue_count_kernel,
                          (const void*)queue_scan_kernel, (const void*)queue_scatter_kernel, (const void*)hotness_kernel};
@@ -588,9 +621,11 @@ moment_status configure_gather_kernels(int carveout) {
         if (carveout >= 0)
             MOMENT_TRY(cuda_check(cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, carveout),
                                   "carveout attribute"));
-    return cuda_check(cudaFuncSetAttribute((const void*)gather_bulk_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                           kBulkStages * kBulkStageBudget),
-                      "bulk gather smem attribute");
+    for (const void* f : {(const void*)gather_bulk_kernel<2>, (const void*)gather_bulk_kernel<4>,
+                          (const void*)gather_bulk_kernel<6>, (const void*)gather_bulk_kernel<8>})
+        MOMENT_TRY(cuda_check(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmemMax),
+                              "bulk gather smem attribute"));
+    return MOMENT_OK;
 }
 
 moment_status launch_hotness(const int64_t* ids, const int64_t* n_dev, int64_t max_n, uint64_t* hot, cudaStream_t stream) {

@@ -41,6 +41,7 @@ struct HopArgs {
     const uint64_t* call;  // device call block: [0] = rng_seed, [1] = seeds pointer (written per call)
     int32_t h, k;
     int32_t replace;
+    int32_t grid_per_sm;   // launch cap: blocks per SM (grid-stride beyond it)
 };
 
 // Fire-and-forget: the result is unused, so this is a RED.OR the issuing warp never waits on.
@@ -413,7 +414,7 @@ template <int G, int Q>
 void launch_sample_hop_q(const HopArgs& a, int64_t max_F, cudaStream_t stream) {
     const int64_t groups = (max_F + Q - 1) / Q;
     const int64_t blocks = std::max<int64_t>(1, (groups * G + 255) / 256);
-    hop_sample_kernel<G, Q><<<(int)std::min<int64_t>(blocks, 148 * 16), 256, 0, stream>>>(a);
+    hop_sample_kernel<G, Q><<<(int)std::min<int64_t>(blocks, (int64_t)148 * a.grid_per_sm), 256, 0, stream>>>(a);
 }
 
 // Small frontiers keep one node per group (latency: every node in flight at once); large frontiers batch
@@ -489,7 +490,7 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
     for (int h = 0; h < H; h++) {
         const int k = p->fanout[h];
         HopArgs a{csr->indptr, csr->indices, out->nodes, out->counts, ctx->pad + pad_off, ctx->cnt + cnt_off,
-                  ctx->newbits, call, h, k, replace};
+                  ctx->newbits, call, h, k, replace, ctx->hop_grid_per_sm};
         if (k <= 4) launch_sample_hop<4>(a, F_bound, stream);
         else if (k <= 8) launch_sample_hop<8>(a, F_bound, stream);
         else if (k <= 16) launch_sample_hop<16>(a, F_bound, stream);
@@ -515,7 +516,8 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
     ca.ebase = ctx->ebase;
     ca.ticket = ctx->tickets;
     ca.H = H;
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(std::max(comp_tiles, (F_bound + 1023) / 1024), 148 * 4));
+    const int grid = (int)std::max<int64_t>(
+        1, std::min<int64_t>(std::max(comp_tiles, (F_bound + 1023) / 1024), (int64_t)148 * ctx->compact_grid_per_sm));
     compact_kernel<<<grid, kSampleTile, 0, stream>>>(ca);
     return cuda_check(cudaGetLastError(), "moment_sample: launch");
 }

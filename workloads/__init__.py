@@ -28,6 +28,9 @@ CONFIGS = {
     # BASELINE.json configs[0..4]; n, m = CSR entries, R = row bytes (dim * dtype size), fanout, batch.
     "C1": dict(n=1 << 16, m=1 << 20, dim=128, dtype=torch.float32, fanout=(10, 5), batch=1024,
                desc="R-MAT 2^16, avg degree 16, 128-d fp32, fanout [10,5], batch 1024, 1 GPU"),
+    # experiment only (not a BASELINE config): C2's per-vertex shape on a graph whose CSR fits in L2
+    "X_L2": dict(n=1 << 18, m=1 << 22, dim=100, dtype=torch.float32, fanout=(15, 10, 5), batch=1024,
+                 desc="experiment: R-MAT 2^18 / 2^22 edges (CSR 18 MB, L2-resident), C2 fanout and rows"),
     "C2": dict(n=2_449_029, m=61_859_140, dim=100, dtype=torch.float32, fanout=(15, 10, 5), batch=1024,
                desc="ogbn-products-shaped: 2.45M vertices, 61.9M edges, 100-d fp32, fanout [15,10,5], batch 1024, "
                     "all features in HBM"),
