@@ -92,9 +92,11 @@ __device__ __forceinline__ int64_t lookback_warp(uint64_t* status, int64_t tile,
         const int64_t j = end - lane;
         uint64_t s = kFlagPrefix;  // "before tile 0" acts as a zero prefix (never reached: tile 0 is a prefix)
         if (j >= 0) {
-            do {
+            s = ld_flag(&status[j]);
+            while ((s & ~kValMask) == 0) {
+                __nanosleep(64);
                 s = ld_flag(&status[j]);
-            } while ((s & ~kValMask) == 0);
+            }
         }
         const unsigned pre = __ballot_sync(0xffffffffu, (s & ~kValMask) == kFlagPrefix);
         const int stop = pre ? __ffs(pre) - 1 : 32;
@@ -125,9 +127,11 @@ __device__ __forceinline__ int64_t lookback_block(uint64_t* status, int64_t tile
         const int64_t j = end - threadIdx.x;
         uint64_t s = 0;
         if (j >= 0) {
-            do {
+            s = ld_flag(&status[j]);
+            while ((s & ~kValMask) == 0) {  // back off: polling warps must not crowd out working ones
+                __nanosleep(64);
                 s = ld_flag(&status[j]);
-            } while ((s & ~kValMask) == 0);
+            }
         }
         if (threadIdx.x == 0) *nearest = NT;
         __syncthreads();

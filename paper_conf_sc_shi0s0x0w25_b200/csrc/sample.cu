@@ -349,9 +349,11 @@ __global__ void __launch_bounds__(kSampleTile) compact_kernel(CompactArgs a) {
                 s_base = prefix;
             } else {
                 uint64_t b;
-                do {
+                b = dev::ld_flag(&a.ebase[h]);
+                while (!(b & kBaseReady)) {
+                    __nanosleep(64);
                     b = dev::ld_flag(&a.ebase[h]);
-                } while (!(b & kBaseReady));
+                }
                 s_base = (int64_t)(b & ~kBaseReady);
             }
         }

@@ -353,3 +353,96 @@ def test_moment_step_many_in_flight(orc, c1):
     for b in [0, 1, 40, 63, 64, 65, 79]:
         want = orc.sample(ip, ix, batches[b].cpu().numpy(), [6, 3], 1000 + b)
         assert_same_sample(bufs[b].result(), want)
+
+
+@pytest.mark.parametrize("name", ["C3"])
+def test_full_size_config_sample_and_gather(orc, name):
+    """BASELINE config at full size (C3: 111 M vertices, 1.6 B edges, 57 GB of 128-d fp32 features in
+    HBM): one batch of the bench's shape, whole-sample parity with the oracle and 4096 sampled rows of the
+    gather checked against the feature generator."""
+    _need_gpu()
+    cfg = W.CONFIGS[name]
+    g = W.rmat_csr(cfg["n"], cfg["m"], device=DEV)
+    torch.cuda.empty_cache()
+    fan = list(cfg["fanout"])
+    train = W.training_set(g, min_count=cfg["batch"])
+    seeds = W.epoch_batches(train, cfg["batch"], 0)[0]
+    table = W.feature_table(cfg["n"], cfg["dim"], cfg["dtype"], device=DEV)
+    R = table.shape[1]
+    ctx = M.Ctx(n_vertices=g.n, max_seeds=cfg["batch"], max_fanout=fan, device=0, row_bytes=R, bin_owner=[0],
+                bin_ptr=[table.data_ptr()])
+    bufs = M.SampleBuffers.allocate(cfg["batch"], fan, g.n, DEV)
+    rows = torch.empty((bufs.nodes.numel(), R), dtype=torch.uint8, device=DEV)
+    rng = W.batch_rng_seed(11, 0, 0, 0)
+    ctx.step(g.indptr, g.indices, seeds, fan, rng, bufs, rows)
+    torch.cuda.synchronize()
+    got = bufs.result()
+    want = orc.sample(g.indptr.cpu().numpy(), g.indices.cpu().numpy(), seeds.cpu().numpy(), fan, rng)
+    assert_same_sample(got, want)
+    nF = int(want["counts"][len(fan)])
+    pick = np.random.default_rng(0).integers(0, nF, 4096)
+    ids = torch.as_tensor(want["nodes"][pick])
+    assert np.array_equal(rows[torch.as_tensor(pick, device=DEV)].cpu().numpy(),
+                          W.feature_rows(ids, cfg["dim"], cfg["dtype"]).numpy())
+    del table, g, rows
+    torch.cuda.empty_cache()
+
+
+def test_c4_full_size_tiered_gather(orc):
+    """C4 at full graph size (244 M vertices, 1.73 B edges, 768-d fp16 = 1536-byte rows): whole-sample
+    parity, then the tiered gather: the hottest vertices (pre-sampling hotness, moment_place DDAK) in a
+    32 GiB HBM cache, every other row read zero-copy from pinned host DRAM. 375 GB of features exceed the
+    host, so the host tier is a ring of R_phys physical rows and row(v) := feature(v mod R_phys) for every
+    tier (SURVEY §8(d) fallback); the checked bytes still cross PCIe."""
+    _need_gpu()
+    cfg = W.CONFIGS["C4"]
+    g = W.rmat_csr(cfg["n"], cfg["m"], device=DEV)
+    torch.cuda.empty_cache()
+    n, fan, B = g.n, list(cfg["fanout"]), cfg["batch"]
+    R = cfg["dim"] * 2
+    R_phys = 1 << 23
+    train = W.training_set(g, min_count=B * 8)
+    batches = W.epoch_batches(train, B, 0)
+    ctx0 = M.Ctx(n_vertices=n, max_seeds=B, max_fanout=fan, device=0)
+    bufs = M.SampleBuffers.allocate(B, fan, n, DEV)
+    hot = torch.zeros(n, dtype=torch.int64, device=DEV)
+    for b in range(4):  # P2: pre-sampling hotness
+        ctx0.step(g.indptr, g.indices, batches[b], fan, W.batch_rng_seed(3, 99, 0, b), bufs, None)
+        ctx0.hotness(bufs.nodes, hot, n_dev=bufs.counts[3:4], max_n=bufs.nodes.numel())
+    cap_hbm = (32 << 30) // R
+    bin_of, slot_of, *_ = M.place(None, hot.cpu().numpy().astype(np.uint64), [cap_hbm, n], bin_tier=[1, 2],
+                                  bin_traffic=[6_469_000, 55_000])
+    del hot
+    v_all = np.arange(n, dtype=np.int64)
+    host = bin_of == 1
+    slot_of[host] = v_all[host] % R_phys  # ring host tier
+    placement = torch.as_tensor(M.place_pack(bin_of, slot_of).view(np.int64), device=DEV)
+    hbm_v = torch.as_tensor(v_all[bin_of == 0][np.argsort(slot_of[bin_of == 0])], device=DEV)
+    hbm = torch.empty((max(1, len(hbm_v)), R), dtype=torch.uint8, device=DEV)
+    for c0 in range(0, len(hbm_v), 1 << 22):
+        hbm[c0:c0 + (1 << 22)] = W.feature_rows(hbm_v[c0:c0 + (1 << 22)] % R_phys, cfg["dim"], cfg["dtype"])
+    ring = torch.empty((R_phys, R), dtype=torch.uint8).pin_memory()
+    for c0 in range(0, R_phys, 1 << 22):
+        ids = torch.arange(c0, min(R_phys, c0 + (1 << 22)), device=DEV)
+        ring[c0:c0 + len(ids)] = W.feature_rows(ids, cfg["dim"], cfg["dtype"]).cpu()
+    ctx = M.Ctx(n_vertices=n, max_seeds=B, max_fanout=fan, device=0, row_bytes=R, bin_owner=[0, -1],
+                bin_ptr=[hbm.data_ptr(), ring.data_ptr()], placement=placement)
+    rows = torch.empty((bufs.nodes.numel(), R), dtype=torch.uint8, device=DEV)
+    ip, ix = g.indptr.cpu().numpy(), g.indices.cpu().numpy()
+    for b in (5, 6):
+        rng = W.batch_rng_seed(3, 0, 0, b)
+        ctx.sample(g.indptr, g.indices, batches[b], fan, rng, bufs)
+        ctx.gather(bufs.nodes, rows, n_dev=bufs.counts[3:4], max_n=bufs.nodes.numel())
+        torch.cuda.synchronize()
+        got = bufs.result()
+        want = orc.sample(ip, ix, batches[b].cpu().numpy(), fan, rng)
+        assert_same_sample(got, want)
+        nF = int(want["counts"][len(fan)])
+        pick = np.random.default_rng(b).integers(0, nF, 8192)
+        ids = torch.as_tensor(want["nodes"][pick] % R_phys)
+        assert np.array_equal(rows[torch.as_tensor(pick, device=DEV)].cpu().numpy(),
+                              W.feature_rows(ids, cfg["dim"], cfg["dtype"]).numpy())
+        in_hbm = (bin_of[want["nodes"]] == 0).mean()
+        assert 0.0 < in_hbm < 1.0  # both tiers exercised
+    del hbm, ring, g, rows
+    torch.cuda.empty_cache()
