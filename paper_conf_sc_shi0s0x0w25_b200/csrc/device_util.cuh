@@ -62,7 +62,7 @@ __device__ __forceinline__ int64_t block_exclusive_scan(int64_t x, int64_t* tota
 }
 
 // Decoupled look-back (single-pass chained scan). Descriptor: bits 62..63 = state (0 empty,
-// 1 aggregate, 2 inclusive prefix), bits 0..61 = value. Called by ONE thread per tile; tiles are taken
+// 1 aggregate, 2 inclusive prefix), bits 0..61 = value. Called by one warp / block per tile; tiles are taken
 // in increasing order through an atomic ticket, so every predecessor tile is owned by a running block.
 constexpr uint64_t kFlagAgg = 1ull << 62, kFlagPrefix = 2ull << 62, kValMask = (1ull << 62) - 1;
 
@@ -151,26 +151,6 @@ __device__ __forceinline__ int64_t lookback_block(uint64_t* status, int64_t tile
         if (stop < NT || end - NT < 0) break;
     }
     if (threadIdx.x == 0) st_flag(&status[tile], kFlagPrefix | (uint64_t)(exclusive + aggregate));
-    return exclusive;
-}
-
-__device__ __forceinline__ int64_t lookback(uint64_t* status, int64_t tile, int64_t aggregate) {
-    using ref = cuda::atomic_ref<unsigned long long, cuda::thread_scope_device>;
-    if (tile == 0) {
-        ref(*reinterpret_cast<unsigned long long*>(&status[0])).store(kFlagPrefix | (uint64_t)aggregate, cuda::memory_order_release);
-        return 0;
-    }
-    ref(*reinterpret_cast<unsigned long long*>(&status[tile])).store(kFlagAgg | (uint64_t)aggregate, cuda::memory_order_release);
-    int64_t exclusive = 0;
-    for (int64_t j = tile - 1; j >= 0;) {
-        const uint64_t s = ref(*reinterpret_cast<unsigned long long*>(&status[j])).load(cuda::memory_order_acquire);
-        const uint64_t flag = s & ~kValMask;
-        if (flag == 0) continue;  // predecessor not published yet: spin
-        exclusive += (int64_t)(s & kValMask);
-        if (flag == kFlagPrefix) break;
-        j--;
-    }
-    ref(*reinterpret_cast<unsigned long long*>(&status[tile])).store(kFlagPrefix | (uint64_t)(exclusive + aggregate), cuda::memory_order_release);
     return exclusive;
 }
 

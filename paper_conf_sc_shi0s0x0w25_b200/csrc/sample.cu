@@ -28,6 +28,10 @@ constexpr int kScanWords = kBitscanWordsPerThread;  // bitmap words per bitscan 
 constexpr int kScanTileWords = kBitscanTileWords;   // 1024 words = 32768 ids per tile
 static_assert(kScanWords == 4, "bitscan loads one uint4 per thread");
 constexpr int kMaxHops = 16;
+#ifndef MOMENT_SAMPLE_MIN_BLOCKS
+#define MOMENT_SAMPLE_MIN_BLOCKS 6  // __launch_bounds__ min blocks per SM of the sampler kernels (<= 40 registers:
+                                    // measured +5-8 % vs uncapped at 1 and 8 batches in flight)
+#endif
 constexpr uint64_t kBaseReady = 1ull << 63;
 
 struct HopArgs {
@@ -150,7 +154,7 @@ __device__ __forceinline__ void sample_node_slow(const cg::thread_block_tile<G>&
 // choices (lane i owns choice i: Floyd / all / with replacement) and neighbour loads are issued as Q
 // independent batches, so each thread keeps Q dependent chains in flight instead of one.
 template <int G, int Q>
-__global__ void __launch_bounds__(256) hop_sample_kernel(HopArgs a) {
+__global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_kernel(HopArgs a) {
     const int64_t F = a.counts[a.h];
     const uint64_t seed = a.call[0];
     auto grp = cg::tiled_partition<G>(cg::this_thread_block());
@@ -307,7 +311,7 @@ struct CompactArgs {
     const int32_t* cnt[kMaxHops];
 };
 
-__global__ void __launch_bounds__(kSampleTile) compact_kernel(CompactArgs a) {
+__global__ void __launch_bounds__(kSampleTile, MOMENT_SAMPLE_MIN_BLOCKS) compact_kernel(CompactArgs a) {
     __shared__ int64_t s_red[kSampleTile / 32];
     __shared__ uint32_t s_tile;
     __shared__ int s_nearest;

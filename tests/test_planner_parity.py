@@ -29,12 +29,6 @@ def test_library_exports_every_declared_symbol():
     assert L.moment_version() >= 1
 
 
-def _graph_topology(n, links, s, t):
-    """Wrap a plain s-t graph as a topology: s = SOURCE, t = SINK, first hop STORAGE, others interconnect,
-    predecessors of t COMPUTE. Only used for max-flow parity on arbitrary graphs."""
-    return None
-
-
 def flow_certificate(n, links, s, t, value, flow):
     bal = [0] * n
     for (u, v, c), f in zip(links, flow):
