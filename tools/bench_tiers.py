@@ -108,12 +108,26 @@ def run_mode(mode, g, table_dev, hot, args, batches, R, dev, fanout):
     gather_ms = sum(a.elapsed_time(b) for a, b in zip(g0, g1))
     nb = len(batches)
     host_bytes = host_rows * R
+    # P5 prediction: the time-bisection plan of this batch's demand on the 1-GPU topology
+    # (HBM bin -> GPU at the measured copy bandwidth, host bin -> CPU -> GPU port at the measured H2D),
+    # against the measured gather time
+    topo1 = M.topology([(M.NODE_STORAGE, M.TIER_GPU_HBM, 0), (M.NODE_STORAGE, M.TIER_HOST_DRAM, 0),
+                        (M.NODE_INTERCONNECT, 0, -1), (M.NODE_COMPUTE, 0, 0)],
+                       [(0, 3, 6_469_000), (1, 2, 400_000), (2, 3, int(args.h2d * 1000))])
+    N1 = topo1.info()[0]
+    demand = np.zeros(N1, np.int64)
+    demand[0] = int(hbm_rows * R / nb)
+    demand[1] = int(host_bytes / nb)
+    # HBM: each row is read once from the HBM bin and written once to the batch buffer (r + w bytes)
+    plan = M.plan(topo1, [3], demand, 0, 6_469_000 // 2).info()
     out = {"placement": mode, "seeds_per_s": nb * args.batch / (ms / 1e3), "ms_per_batch": ms / nb,
            "gather_ms_per_batch": gather_ms / nb, "rows_per_batch": (hbm_rows + host_rows) / nb,
            "hbm_hit_rate": hbm_rows / max(1, hbm_rows + host_rows),
            "host_bytes_per_batch": host_bytes / nb, "hbm_bytes_per_batch": hbm_rows * R / nb,
            "host_link_GBs_in_gather": host_bytes / (gather_ms / 1e3) / 1e9,
            "host_link_frac_of_h2d": host_bytes / (gather_ms / 1e3) / 1e9 / args.h2d,
+           "plan_t_star_us": plan["t_star"], "plan_t_ingest_us": plan["t_ingest"], "plan_t_hbm_us": plan["t_hbm"],
+           "prediction_error": abs(plan["t_star"] - gather_ms / nb * 1e3) / (gather_ms / nb * 1e3),
            "bin_rows": [int(x) for x in used], "bin_traffic": [int(x) for x in traffic]}
     del bins, ctx
     torch.cuda.empty_cache()
