@@ -25,9 +25,9 @@ namespace cg = cooperative_groups;
 namespace moment {
 namespace {
 
-constexpr int kScanWords = kBitscanWordsPerThread;  // bitmap words per bitscan thread (4: one uint4)
-constexpr int kScanTileWords = kBitscanTileWords;   // 1024 words = 32768 ids per tile
-static_assert(kScanWords == 4, "bitscan loads one uint4 per thread");
+constexpr int kScanWords = kBitscanWordsPerThread;  // bitmap words per bitscan thread (uint4 loads)
+constexpr int kScanTileWords = kBitscanTileWords;   // words per tile
+static_assert(kScanWords % 4 == 0, "bitscan loads whole uint4s");
 constexpr int kMaxHops = 16;
 #ifndef MOMENT_SAMPLE_MIN_BLOCKS
 #define MOMENT_SAMPLE_MIN_BLOCKS 6  // __launch_bounds__ min blocks per SM of the sampler kernels (<= 40 registers:
@@ -256,10 +256,14 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
         uint32_t nb[kScanWords], nw[kScanWords];
         int cnt = 0;
         if (w0 + kScanWords <= a.n_words) {
-            const uint4 n4 = __ldcg(reinterpret_cast<const uint4*>(a.newbits + w0));
-            const uint4 v4 = __ldcg(reinterpret_cast<const uint4*>(a.visited + w0));
-            nb[0] = n4.x; nb[1] = n4.y; nb[2] = n4.z; nb[3] = n4.w;
-            nw[0] = n4.x & ~v4.x; nw[1] = n4.y & ~v4.y; nw[2] = n4.z & ~v4.z; nw[3] = n4.w & ~v4.w;
+#pragma unroll
+            for (int q4 = 0; q4 < kScanWords / 4; q4++) {
+                const uint4 n4 = __ldcg(reinterpret_cast<const uint4*>(a.newbits + w0) + q4);
+                const uint4 v4 = __ldcg(reinterpret_cast<const uint4*>(a.visited + w0) + q4);
+                nb[4 * q4] = n4.x; nb[4 * q4 + 1] = n4.y; nb[4 * q4 + 2] = n4.z; nb[4 * q4 + 3] = n4.w;
+                nw[4 * q4] = n4.x & ~v4.x; nw[4 * q4 + 1] = n4.y & ~v4.y;
+                nw[4 * q4 + 2] = n4.z & ~v4.z; nw[4 * q4 + 3] = n4.w & ~v4.w;
+            }
         } else {
 #pragma unroll
             for (int q = 0; q < kScanWords; q++) {
@@ -425,11 +429,13 @@ void launch_sample_hop_q(const HopArgs& a, int64_t max_F, cudaStream_t stream) {
 }
 
 // Small frontiers keep one node per group (latency: every node in flight at once); large frontiers batch
-// 4 nodes per group (throughput: 4 chains in flight per thread, a quarter of the threads).
+// `big_q` nodes per group (throughput: that many chains in flight per thread, 1/big_q of the warps).
 template <int G>
-void launch_sample_hop(const HopArgs& a, int64_t max_F, cudaStream_t stream) {
-    if (max_F >= 65536) launch_sample_hop_q<G, 4>(a, max_F, stream);
-    else launch_sample_hop_q<G, 1>(a, max_F, stream);
+void launch_sample_hop(const HopArgs& a, int64_t max_F, int big_q, cudaStream_t stream) {
+    if (max_F < 65536 || big_q <= 1) launch_sample_hop_q<G, 1>(a, max_F, stream);
+    else if (big_q <= 2) launch_sample_hop_q<G, 2>(a, max_F, stream);
+    else if (big_q <= 4) launch_sample_hop_q<G, 4>(a, max_F, stream);
+    else launch_sample_hop_q<G, 8>(a, max_F, stream);
 }
 
 }  // namespace
@@ -440,8 +446,12 @@ moment_status configure_sample_kernels(int carveout) {
     const void* fns[] = {(const void*)init_kernel, (const void*)bitscan_kernel, (const void*)compact_kernel,
                          (const void*)hop_sample_kernel<4, 1>, (const void*)hop_sample_kernel<8, 1>,
                          (const void*)hop_sample_kernel<16, 1>, (const void*)hop_sample_kernel<32, 1>,
+                         (const void*)hop_sample_kernel<4, 2>, (const void*)hop_sample_kernel<8, 2>,
+                         (const void*)hop_sample_kernel<16, 2>, (const void*)hop_sample_kernel<32, 2>,
                          (const void*)hop_sample_kernel<4, 4>, (const void*)hop_sample_kernel<8, 4>,
-                         (const void*)hop_sample_kernel<16, 4>, (const void*)hop_sample_kernel<32, 4>};
+                         (const void*)hop_sample_kernel<16, 4>, (const void*)hop_sample_kernel<32, 4>,
+                         (const void*)hop_sample_kernel<4, 8>, (const void*)hop_sample_kernel<8, 8>,
+                         (const void*)hop_sample_kernel<16, 8>, (const void*)hop_sample_kernel<32, 8>};
     for (const void* f : fns)
         MOMENT_TRY(cuda_check(cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, carveout),
                               "carveout attribute"));
@@ -498,10 +508,11 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         const int k = p->fanout[h];
         HopArgs a{csr->indptr, csr->indices, out->nodes, out->counts, ctx->pad + pad_off, ctx->cnt + cnt_off,
                   ctx->newbits, call, h, k, replace, ctx->hop_grid_per_sm};
-        if (k <= 4) launch_sample_hop<4>(a, F_bound, stream);
-        else if (k <= 8) launch_sample_hop<8>(a, F_bound, stream);
-        else if (k <= 16) launch_sample_hop<16>(a, F_bound, stream);
-        else launch_sample_hop<32>(a, F_bound, stream);
+        const int q = ctx->hop_nodes_per_group;
+        if (k <= 4) launch_sample_hop<4>(a, F_bound, q, stream);
+        else if (k <= 8) launch_sample_hop<8>(a, F_bound, q, stream);
+        else if (k <= 16) launch_sample_hop<16>(a, F_bound, q, stream);
+        else launch_sample_hop<32>(a, F_bound, q, stream);
         ScanArgs s{out->nodes, out->counts, ctx->lidx, ctx->newbits, ctx->visited,
                    ctx->tile_status + ctx->bitscan_tiles_off[h], ctx->tickets + 1 + h, ctx->n_words, h};
         bitscan_kernel<<<(int)std::min<int64_t>(n_scan_tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
