@@ -388,19 +388,22 @@ def test_full_size_config_sample_and_gather(orc, name):
     torch.cuda.empty_cache()
 
 
-def test_c4_full_size_tiered_gather(orc):
-    """C4 at full graph size (244 M vertices, 1.73 B edges, 768-d fp16 = 1536-byte rows): whole-sample
-    parity, then the tiered gather: the hottest vertices (pre-sampling hotness, moment_place DDAK) in a
-    32 GiB HBM cache, every other row read zero-copy from pinned host DRAM. 375 GB of features exceed the
-    host, so the host tier is a ring of R_phys physical rows and row(v) := feature(v mod R_phys) for every
-    tier (SURVEY §8(d) fallback); the checked bytes still cross PCIe."""
+@pytest.mark.parametrize("name,cache_gib", [("C4", 32), ("C5", 64)])
+def test_full_size_tiered_gather(orc, name, cache_gib):
+    """C4 / C5 at full graph size (244 M vertices / 1.73 B edges, 768-d fp16; 269 M / 4.0 B edges, 1024-d
+    fp32): whole-sample parity, then the tiered gather: the hottest vertices (pre-sampling hotness,
+    moment_place DDAK) in a C4: 32 GiB / C5: 64 GiB HBM cache, every other row read zero-copy from pinned
+    host DRAM. The features (375 GB / 1.1 TB) exceed the host, so the host tier is a ring of R_phys
+    physical rows and row(v) := feature(v mod R_phys) for every tier (SURVEY §8(d) fallback); the checked
+    bytes still cross PCIe."""
     _need_gpu()
-    cfg = W.CONFIGS["C4"]
+    cfg = W.CONFIGS[name]
     g = W.rmat_csr(cfg["n"], cfg["m"], device=DEV)
     torch.cuda.empty_cache()
     n, fan, B = g.n, list(cfg["fanout"]), cfg["batch"]
-    R = cfg["dim"] * 2
-    R_phys = 1 << 23
+    R = cfg["dim"] * torch.empty(0, dtype=cfg["dtype"]).element_size()
+    R_phys = 1 << 22
+    chunk = max(1, (1 << 31) // (R // 4 * 8))  # rows per feature_rows call (bounded temporaries)
     train = W.training_set(g, min_count=B * 8)
     batches = W.epoch_batches(train, B, 0)
     ctx0 = M.Ctx(n_vertices=n, max_seeds=B, max_fanout=fan, device=0)
@@ -409,21 +412,23 @@ def test_c4_full_size_tiered_gather(orc):
     for b in range(4):  # P2: pre-sampling hotness
         ctx0.step(g.indptr, g.indices, batches[b], fan, W.batch_rng_seed(3, 99, 0, b), bufs, None)
         ctx0.hotness(bufs.nodes, hot, n_dev=bufs.counts[3:4], max_n=bufs.nodes.numel())
-    cap_hbm = (32 << 30) // R
+    cap_hbm = (cache_gib << 30) // R
     bin_of, slot_of, *_ = M.place(None, hot.cpu().numpy().astype(np.uint64), [cap_hbm, n], bin_tier=[1, 2],
                                   bin_traffic=[6_469_000, 55_000])
     del hot
-    v_all = np.arange(n, dtype=np.int64)
     host = bin_of == 1
-    slot_of[host] = v_all[host] % R_phys  # ring host tier
+    slot_of[host] = np.nonzero(host)[0] % R_phys  # ring host tier
     placement = torch.as_tensor(M.place_pack(bin_of, slot_of).view(np.int64), device=DEV)
-    hbm_v = torch.as_tensor(v_all[bin_of == 0][np.argsort(slot_of[bin_of == 0])], device=DEV)
+    in_hbm = np.nonzero(~host)[0]
+    hbm_v = torch.as_tensor(in_hbm[np.argsort(slot_of[in_hbm])], device=DEV)
+    del in_hbm
     hbm = torch.empty((max(1, len(hbm_v)), R), dtype=torch.uint8, device=DEV)
-    for c0 in range(0, len(hbm_v), 1 << 22):
-        hbm[c0:c0 + (1 << 22)] = W.feature_rows(hbm_v[c0:c0 + (1 << 22)] % R_phys, cfg["dim"], cfg["dtype"])
+    for c0 in range(0, len(hbm_v), chunk):
+        hbm[c0:c0 + chunk] = W.feature_rows(hbm_v[c0:c0 + chunk] % R_phys, cfg["dim"], cfg["dtype"])
+    del hbm_v
     ring = torch.empty((R_phys, R), dtype=torch.uint8).pin_memory()
-    for c0 in range(0, R_phys, 1 << 22):
-        ids = torch.arange(c0, min(R_phys, c0 + (1 << 22)), device=DEV)
+    for c0 in range(0, R_phys, chunk):
+        ids = torch.arange(c0, min(R_phys, c0 + chunk), device=DEV)
         ring[c0:c0 + len(ids)] = W.feature_rows(ids, cfg["dim"], cfg["dtype"]).cpu()
     ctx = M.Ctx(n_vertices=n, max_seeds=B, max_fanout=fan, device=0, row_bytes=R, bin_owner=[0, -1],
                 bin_ptr=[hbm.data_ptr(), ring.data_ptr()], placement=placement)
@@ -442,7 +447,7 @@ def test_c4_full_size_tiered_gather(orc):
         ids = torch.as_tensor(want["nodes"][pick] % R_phys)
         assert np.array_equal(rows[torch.as_tensor(pick, device=DEV)].cpu().numpy(),
                               W.feature_rows(ids, cfg["dim"], cfg["dtype"]).numpy())
-        in_hbm = (bin_of[want["nodes"]] == 0).mean()
-        assert 0.0 < in_hbm < 1.0  # both tiers exercised
+        frac_hbm = (bin_of[want["nodes"]] == 0).mean()
+        assert 0.0 < frac_hbm < 1.0  # both tiers exercised
     del hbm, ring, g, rows
     torch.cuda.empty_cache()

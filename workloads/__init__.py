@@ -89,7 +89,7 @@ class Graph:
 
 
 def rmat_csr(n: int, m: int, seed: int = 0x4D4F4D454E54, device="cpu", a=0.57, b=0.19, c=0.19,
-             chunk: int = 1 << 23) -> Graph:
+             chunk: int = 1 << 23, max_edges_in_memory: int = 1 << 31) -> Graph:
     L = max(1, math.ceil(math.log2(n)))
     ta = int(a * 2**32)
     tb = int((a + b) * 2**32)
@@ -99,9 +99,8 @@ def rmat_csr(n: int, m: int, seed: int = 0x4D4F4D454E54, device="cpu", a=0.57, b
     while math.gcd(A, n) != 1 or A == 0:
         A = (A + 1) % n
     B = mix(seed, 3) % n
-    srcs, dsts = [], []
-    for e0 in range(0, m, chunk):
-        e = torch.arange(e0, min(m, e0 + chunk), device=device, dtype=torch.int64)
+    def edges(e0, e1):
+        e = torch.arange(e0, e1, device=device, dtype=torch.int64)
         s = torch.zeros_like(e)
         d = torch.zeros_like(e)
         for lvl in range(L):
@@ -113,8 +112,13 @@ def rmat_csr(n: int, m: int, seed: int = 0x4D4F4D454E54, device="cpu", a=0.57, b
             d = (d << 1) | (q_b | q_d).to(torch.int64)
         s = (s * n) >> L
         d = (d * n) >> L
-        s = (s * A + B) % n
-        d = (d * A + B) % n
+        return (s * A + B) % n, (d * A + B) % n
+
+    if m > max_edges_in_memory:
+        return _rmat_csr_partitioned(n, m, edges, chunk, max_edges_in_memory, device)
+    srcs, dsts = [], []
+    for e0 in range(0, m, chunk):
+        s, d = edges(e0, min(m, e0 + chunk))
         srcs.append(s)
         dsts.append(d)
     src = torch.cat(srcs)
@@ -130,6 +134,36 @@ def rmat_csr(n: int, m: int, seed: int = 0x4D4F4D454E54, device="cpu", a=0.57, b
     del src
     indptr = torch.zeros(n + 1, dtype=torch.int64, device=device)
     indptr[1:] = torch.cumsum(counts, 0)
+    return Graph(indptr, indices, n, m)
+
+
+def _rmat_csr_partitioned(n, m, edges, chunk, budget, device) -> Graph:
+    """The same canonical CSR for graphs too large to sort at once: one pass for the degrees, then one pass
+    per source range of <= `budget` edges, each regenerating every edge and keeping its range's."""
+    counts = torch.zeros(n, dtype=torch.int64, device=device)
+    for e0 in range(0, m, chunk):
+        s, _ = edges(e0, min(m, e0 + chunk))
+        counts += torch.bincount(s, minlength=n)
+    indptr = torch.zeros(n + 1, dtype=torch.int64, device=device)
+    indptr[1:] = torch.cumsum(counts, 0)
+    del counts
+    indices = torch.empty(m, dtype=torch.int32, device=device)
+    lo = 0
+    while lo < n:
+        # largest hi with indptr[hi] - indptr[lo] <= budget (at least one vertex)
+        hi = int(torch.searchsorted(indptr, indptr[lo] + budget, right=True)) - 1
+        hi = max(lo + 1, min(hi, n))
+        keys = []
+        for e0 in range(0, m, chunk):
+            s, d = edges(e0, min(m, e0 + chunk))
+            sel = (s >= lo) & (s < hi)
+            keys.append((s[sel] - lo) * n + d[sel])
+        kv = torch.cat(keys)
+        del keys
+        kv, _ = torch.sort(kv)
+        indices[int(indptr[lo]):int(indptr[hi])] = (kv % n).to(torch.int32)
+        del kv
+        lo = hi
     return Graph(indptr, indices, n, m)
 
 
