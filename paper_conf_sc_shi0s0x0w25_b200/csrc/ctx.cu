@@ -102,6 +102,8 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
         std::sscanf(v, "%d,%d,%d", &c->bulk_stages, &c->bulk_blocks_per_sm, &c->bulk_stage_kb);
     if (const char* v = std::getenv("MOMENT_HOP_GRID")) c->hop_grid_per_sm = std::max(1, std::atoi(v));
     if (const char* v = std::getenv("MOMENT_HOP_Q")) c->hop_nodes_per_group = std::max(1, std::atoi(v));
+    if (const char* v = std::getenv("MOMENT_HOP_WARP")) c->hop_warp_segmented = std::atoi(v) != 0;
+    if (const char* v = std::getenv("MOMENT_STEP_FORK")) c->step_fork = std::atoi(v) != 0;
     if (const char* v = std::getenv("MOMENT_COMPACT_GRID")) c->compact_grid_per_sm = std::max(1, std::atoi(v));
     if (const char* l2 = std::getenv("MOMENT_GATHER_L2")) {  // "<load><store>" digits, e.g. "01"
         if (std::strlen(l2) == 2) {
@@ -206,6 +208,9 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
             }
         }
         if ((st = cuda_check(cudaStreamCreateWithFlags(&c->cap_stream, cudaStreamNonBlocking), "moment_ctx_create: stream")) != MOMENT_OK) break;
+        if ((st = cuda_check(cudaStreamCreateWithFlags(&c->cap_side, cudaStreamNonBlocking), "moment_ctx_create: stream")) != MOMENT_OK) break;
+        if ((st = cuda_check(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming), "moment_ctx_create: event")) != MOMENT_OK) break;
+        if ((st = cuda_check(cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming), "moment_ctx_create: event")) != MOMENT_OK) break;
         if ((st = cuda_check(cudaMemset(c->ws, 0, c->ws_bytes), "moment_ctx_create: memset")) != MOMENT_OK) break;
         if ((st = cuda_check(cudaMemset(c->lidx, 0xFF, a->n_vertices * sizeof(int32_t)), "moment_ctx_create: memset")) != MOMENT_OK) break;
         if (a->n_bins > 0) {
@@ -232,6 +237,9 @@ extern "C" moment_status moment_ctx_free(moment_ctx_t ctx) {
     cudaSetDevice(ctx->device);
     if (ctx->step_exec) cudaGraphExecDestroy(ctx->step_exec);
     if (ctx->cap_stream) cudaStreamDestroy(ctx->cap_stream);
+    if (ctx->cap_side) cudaStreamDestroy(ctx->cap_side);
+    if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
+    if (ctx->ev_join) cudaEventDestroy(ctx->ev_join);
     cudaError_t e = ctx->ws ? cudaFree(ctx->ws) : cudaSuccess;
     cudaSetDevice(cur);
     delete ctx;
@@ -288,9 +296,17 @@ moment_status run_step(moment_ctx_s* c, const moment_csr* csr, int64_t n_seeds, 
             c->step_exec = nullptr;
         }
         MOMENT_TRY(cuda_check(cudaStreamBeginCapture(c->cap_stream, cudaStreamCaptureModeThreadLocal), "capture"));
-        moment_status st = launch_sample(c, csr, c->d_call, n_seeds, p, out, c->cap_stream);
-        if (st == MOMENT_OK && rows)
+        const bool fork = rows && c->step_fork;
+        moment_status st = launch_sample(c, csr, c->d_call, n_seeds, p, out, c->cap_stream, fork ? c->ev_fork : nullptr);
+        if (st == MOMENT_OK && rows && !fork)
             st = launch_gather(c, out->nodes, out->counts + H, out->cap_nodes, rows, nullptr, c->rank, c->cap_stream);
+        if (st == MOMENT_OK && fork) {  // gather on a branch that joins after the compaction
+            st = cuda_check(cudaStreamWaitEvent(c->cap_side, c->ev_fork, 0), "moment_step: fork");
+            if (st == MOMENT_OK)
+                st = launch_gather(c, out->nodes, out->counts + H, out->cap_nodes, rows, nullptr, c->rank, c->cap_side);
+            if (st == MOMENT_OK) st = cuda_check(cudaEventRecord(c->ev_join, c->cap_side), "moment_step: join");
+            if (st == MOMENT_OK) st = cuda_check(cudaStreamWaitEvent(c->cap_stream, c->ev_join, 0), "moment_step: join");
+        }
         cudaGraph_t g = nullptr;
         cudaError_t e = cudaStreamEndCapture(c->cap_stream, &g);
         if (st != MOMENT_OK) {

@@ -23,6 +23,7 @@ struct moment_ctx_s {
     int32_t l2_load_policy = 0, l2_store_policy = 1;  // bulk gather L2 hints: 0 normal, 1 evict_first, 2 evict_last
     int32_t hop_grid_per_sm = 4, compact_grid_per_sm = 1;  // launch caps (MOMENT_HOP_GRID / MOMENT_COMPACT_GRID)
     int32_t hop_nodes_per_group = 4;  // nodes per lane group on large frontiers (MOMENT_HOP_Q: 1, 2, 4, 8)
+    int32_t hop_warp_segmented = 1;   // k <= 32: k-lane groups packed in a warp (MOMENT_HOP_WARP=0: 2^n tiles)
     int32_t bulk_stages = 4, bulk_blocks_per_sm = 4, bulk_stage_kb = 14;  // bulk gather shape (MOMENT_BULK="S,B,KB")
     std::vector<int32_t> bin_owner;
     std::vector<void*> bin_ptr;
@@ -57,7 +58,10 @@ struct moment_ctx_s {
     // per-call arguments the kernels read from device memory (so one captured graph serves every batch)
     uint64_t* d_call = nullptr;         // [2]: rng_seed, seeds pointer (written by set_call_kernel per call)
     // cached CUDA graph of one moment_step (sample + gather), re-captured when its shape changes
-    cudaStream_t cap_stream = nullptr;
+    // (the gather needs only F_H, known after the last bitscan: it runs on a branch beside the compaction)
+    cudaStream_t cap_stream = nullptr, cap_side = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    int32_t step_fork = 1;  // MOMENT_STEP_FORK=0: gather after compact on one chain
     cudaGraphExec_t step_exec = nullptr;
     struct StepKey {
         const void* indptr = nullptr;
@@ -90,8 +94,10 @@ constexpr int kMaxFanout = 1024;
 // Launchers (defined in sample.cu / gather.cu).
 moment_status check_sample(const moment_ctx_s* ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
                            const moment_sample_params* p, const moment_sample_out* out);
+// `after_hops`, if given, is recorded on `stream` once F_H is final (after the last bitscan, before compact).
 moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint64_t* call, int64_t n_seeds,
-                            const moment_sample_params* p, const moment_sample_out* out, cudaStream_t stream);
+                            const moment_sample_params* p, const moment_sample_out* out, cudaStream_t stream,
+                            cudaEvent_t after_hops = nullptr);
 moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n, void* out,
                             const int32_t* route, int32_t serve_rank, cudaStream_t stream);
 moment_status launch_bucket(moment_ctx_s* ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n,

@@ -432,7 +432,8 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
     if (bulk && route == nullptr) {
         // tiles of <= 32 rows, `stages` tiles in flight per 1-warp block, `bps` blocks per SM, each stage at
         // most `stage_kb` KB (defaults 4 / 4 / 14: 4 x 4 x 14 KB fits the SM's shared memory)
-        const int stages = ctx->bulk_stages, bps = ctx->bulk_blocks_per_sm;
+        const int bps = ctx->bulk_blocks_per_sm;  // stages rounded up to an instantiated pipeline depth
+        const int stages = ctx->bulk_stages <= 2 ? 2 : ctx->bulk_stages <= 4 ? 4 : ctx->bulk_stages <= 6 ? 6 : 8;
         const int rows = (int)std::max<int64_t>(1, std::min<int64_t>(kBulkMaxRows, ctx->bulk_stage_kb * 1024 / ctx->row_bytes));
         const size_t smem = (size_t)stages * rows * ctx->row_bytes;
         if (smem > (size_t)kBulkSmemMax) return fail(MOMENT_EINVAL, "moment_gather: bulk stage config needs %zu B smem", smem);

@@ -228,6 +228,93 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_kern
     }
 }
 
+// Warp-segmented sampler for k <= 32: a warp holds NG = floor(32 / k) groups of exactly k lanes (lane i of
+// group g owns choice i), so 32 mod k lanes idle instead of G - k per power-of-two tile (k = 5: 30 of 32
+// lanes busy, not 20). Control flow is warp-uniform: every group runs the same steps under per-group
+// predicates and the collectives span the whole warp (match_any keyed by (group, t), ballots read at the
+// group's bit offset), so groups never diverge and no convergence barriers are needed. Step q of a warp
+// handles the NG consecutive frontier nodes base + q * NG + g: its pad stores are one run of NG * k ints.
+// Same choices as floyd_choice (same draws, same resolution rule), only the lane layout differs.
+template <int Q>
+__global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp_kernel(HopArgs a) {
+    constexpr unsigned kFull = 0xffffffffu;
+    const int64_t F = a.counts[a.h];
+    const uint64_t seed = a.call[0];
+    const int k = a.k;
+    const int lane = threadIdx.x & 31;
+    const int NG = 32 / k;
+    const int g = lane / k;  // NG for the idle lanes
+    const int i = lane - g * k;
+    const bool live = g < NG;
+    const int gbase = g * k;
+    const unsigned below = (1u << lane) - 1u;
+    const int64_t per_warp = (int64_t)NG * Q;
+    const int64_t warps = (int64_t)gridDim.x * 8;
+    for (int64_t base = ((int64_t)blockIdx.x * 8 + threadIdx.x / 32) * per_warp; base < F; base += warps * per_warp) {
+        int64_t idx[Q], v[Q], lo[Q];
+        int32_t d[Q], pos[Q], rnk[Q], u[Q];
+#pragma unroll
+        for (int q = 0; q < Q; q++) {
+            idx[q] = base + (int64_t)q * NG + g;
+            v[q] = (live && idx[q] < F) ? a.nodes[idx[q]] : -1;
+        }
+#pragma unroll
+        for (int q = 0; q < Q; q++) {
+            lo[q] = 0;
+            d[q] = 0;
+            if (v[q] >= 0) {
+                lo[q] = __ldg(a.indptr + v[q]);
+                d[q] = (int32_t)(__ldg(a.indptr + v[q] + 1) - lo[q]);
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < Q; q++) {
+            const int32_t dq = d[q];
+            pos[q] = -1;
+            rnk[q] = i;
+            if (a.replace) {  // uniform over the launch
+                if (dq > 0) pos[q] = (int32_t)dev::uniform(dev::draw(seed, v[q], a.h, i), (uint32_t)dq);
+                continue;
+            }
+            const bool floyd = dq > k;
+            if (!floyd && i < dq) pos[q] = i;  // d <= k: every neighbour, in CSR order
+            if (!__any_sync(kFull, floyd)) continue;
+            const int32_t jj = dq - k + i;
+            const int32_t t = floyd ? (int32_t)dev::uniform(dev::draw(seed, v[q], a.h, i), (uint32_t)(jj + 1))
+                                    : -1 - lane;  // unique sentinel: never matches
+            const unsigned same = __match_any_sync(kFull, ((uint64_t)(uint32_t)g << 32) | (uint32_t)t);
+            const bool dup_a = floyd && (same & below) != 0;
+            const int lstar = gbase + (t - (dq - k));  // the earlier lane of this group whose j equals t
+            const bool ref = floyd && !dup_a && t >= dq - k && lstar < lane;
+            unsigned dup = __ballot_sync(kFull, dup_a);
+            for (;;) {
+                const bool now = dup_a || (ref && ((dup >> lstar) & 1u));
+                const unsigned nd = __ballot_sync(kFull, now);
+                if (nd == dup) break;
+                dup = nd;
+            }
+            const int32_t c = ((dup >> lane) & 1u) ? jj : t;
+            int r = 0;
+            for (int l = 0; l < k; l++) r += __shfl_sync(kFull, c, gbase + l) < c;
+            if (floyd) {
+                pos[q] = c;
+                rnk[q] = r;
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < Q; q++) u[q] = pos[q] >= 0 ? __ldg(a.indices + lo[q] + pos[q]) : 0;
+#pragma unroll
+        for (int q = 0; q < Q; q++) {
+            if (!live || idx[q] >= F) continue;
+            if (i == 0) a.cnt[idx[q]] = a.replace ? (d[q] > 0 ? k : 0) : min(d[q], k);
+            if (pos[q] >= 0) {
+                a.pad[idx[q] * k + rnk[q]] = u[q];
+                mark_new(a.newbits, u[q]);
+            }
+        }
+    }
+}
+
 struct ScanArgs {
     int64_t* nodes;
     int64_t* counts;
@@ -438,6 +525,20 @@ void launch_sample_hop(const HopArgs& a, int64_t max_F, int big_q, cudaStream_t 
     else launch_sample_hop_q<G, 8>(a, max_F, stream);
 }
 
+template <int Q>
+void launch_sample_warp_q(const HopArgs& a, int64_t max_F, cudaStream_t stream) {
+    const int64_t per_warp = (int64_t)(32 / a.k) * Q;
+    const int64_t warps = (max_F + per_warp - 1) / per_warp;
+    const int64_t blocks = std::max<int64_t>(1, (warps + 7) / 8);
+    hop_sample_warp_kernel<Q><<<(int)std::min<int64_t>(blocks, (int64_t)148 * a.grid_per_sm), 256, 0, stream>>>(a);
+}
+
+void launch_sample_warp(const HopArgs& a, int64_t max_F, int big_q, cudaStream_t stream) {
+    if (max_F < 65536 || big_q <= 1) launch_sample_warp_q<1>(a, max_F, stream);
+    else if (big_q <= 2) launch_sample_warp_q<2>(a, max_F, stream);
+    else launch_sample_warp_q<4>(a, max_F, stream);
+}
+
 }  // namespace
 
 // Same shared-memory carveout for every kernel of the library (see configure_gather_kernels).
@@ -451,7 +552,9 @@ moment_status configure_sample_kernels(int carveout) {
                          (const void*)hop_sample_kernel<4, 4>, (const void*)hop_sample_kernel<8, 4>,
                          (const void*)hop_sample_kernel<16, 4>, (const void*)hop_sample_kernel<32, 4>,
                          (const void*)hop_sample_kernel<4, 8>, (const void*)hop_sample_kernel<8, 8>,
-                         (const void*)hop_sample_kernel<16, 8>, (const void*)hop_sample_kernel<32, 8>};
+                         (const void*)hop_sample_kernel<16, 8>, (const void*)hop_sample_kernel<32, 8>,
+                         (const void*)hop_sample_warp_kernel<1>, (const void*)hop_sample_warp_kernel<2>,
+                         (const void*)hop_sample_warp_kernel<4>};
     for (const void* f : fns)
         MOMENT_TRY(cuda_check(cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, carveout),
                               "carveout attribute"));
@@ -489,7 +592,8 @@ moment_status check_sample(const moment_ctx_s* ctx, const moment_csr* csr, const
 
 // Enqueues the 2H + 2 kernels of one sample call (arguments already validated by check_sample).
 moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint64_t* call, int64_t n_seeds,
-                            const moment_sample_params* p, const moment_sample_out* out, cudaStream_t stream) {
+                            const moment_sample_params* p, const moment_sample_out* out, cudaStream_t stream,
+                            cudaEvent_t after_hops) {
     const int H = p->n_hops;
     const int check = (p->flags & MOMENT_SAMPLE_CHECK) ? 1 : 0;
     const int replace = (p->flags & MOMENT_SAMPLE_REPLACE) ? 1 : 0;
@@ -509,7 +613,8 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         HopArgs a{csr->indptr, csr->indices, out->nodes, out->counts, ctx->pad + pad_off, ctx->cnt + cnt_off,
                   ctx->newbits, call, h, k, replace, ctx->hop_grid_per_sm};
         const int q = ctx->hop_nodes_per_group;
-        if (k <= 4) launch_sample_hop<4>(a, F_bound, q, stream);
+        if (ctx->hop_warp_segmented && k <= 32) launch_sample_warp(a, F_bound, q, stream);
+        else if (k <= 4) launch_sample_hop<4>(a, F_bound, q, stream);
         else if (k <= 8) launch_sample_hop<8>(a, F_bound, q, stream);
         else if (k <= 16) launch_sample_hop<16>(a, F_bound, q, stream);
         else launch_sample_hop<32>(a, F_bound, q, stream);
@@ -524,6 +629,7 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         comp_tiles += (F_bound + kSampleTile - 1) / kSampleTile;
         F_bound = std::min(F_bound + F_bound * (int64_t)k, ctx->n_vertices);
     }
+    if (after_hops) MOMENT_TRY(cuda_check(cudaEventRecord(after_hops, stream), "moment_sample: fork event"));
     ca.offsets = out->offsets;
     ca.src = out->src;
     ca.counts = out->counts;

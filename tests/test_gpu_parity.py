@@ -57,7 +57,8 @@ def test_sample_c1_full_size(orc, c1):
         assert_same_sample(got, want)
 
 
-@pytest.mark.parametrize("fanout", [[15, 10, 5], [3], [1, 1, 1, 1], [25, 10], [33, 2], [64], [200]])
+@pytest.mark.parametrize("fanout", [[15, 10, 5], [3], [1, 1, 1, 1], [25, 10], [33, 2], [64], [200], [7, 11, 13],
+                                    [32, 2], [16, 31]])
 @pytest.mark.parametrize("n_seeds", [1, 257, 1000])
 def test_sample_fanouts_and_ragged(orc, c1, fanout, n_seeds):
     _, g = c1
@@ -67,7 +68,20 @@ def test_sample_fanouts_and_ragged(orc, c1, fanout, n_seeds):
     assert_same_sample(got, want)
 
 
-@pytest.mark.parametrize("fanout", [[10, 5], [40]])
+@pytest.mark.parametrize("fanout", [[15, 10, 5], [7, 3], [20]])
+def test_sample_power_of_two_tiles(orc, c1, fanout, monkeypatch):
+    """The power-of-two lane-tile sampler (MOMENT_HOP_WARP=0; always used for k > 32) gives the same result as
+    the warp-segmented one (the default for k <= 32)."""
+    _, g = c1
+    monkeypatch.setenv("MOMENT_HOP_WARP", "0")
+    seeds = np.random.default_rng(5).choice(g.n, 1000, replace=False)
+    got, want = sample_both(orc, g, seeds, fanout, 4242)
+    assert_same_sample(got, want)
+    got, want = sample_both(orc, g, seeds, fanout, 4243, flags=M.SAMPLE_REPLACE)
+    assert_same_sample(got, want)
+
+
+@pytest.mark.parametrize("fanout", [[10, 5], [40], [7, 13]])
 def test_sample_replace(orc, c1, fanout):
     _, g = c1
     seeds = np.random.default_rng(3).choice(g.n, 700, replace=False)
