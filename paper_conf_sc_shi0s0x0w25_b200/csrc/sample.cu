@@ -340,27 +340,26 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
         const int64_t tile = s_tile;
         if (tile >= n_tiles) break;
         const int64_t w0 = tile * kScanTileWords + (int64_t)threadIdx.x * kScanWords;
-        uint32_t nb[kScanWords], nw[kScanWords];
-        int cnt = 0;
+        uint32_t nb[kScanWords], vs[kScanWords];
         if (w0 + kScanWords <= a.n_words) {
 #pragma unroll
             for (int q4 = 0; q4 < kScanWords / 4; q4++) {
                 const uint4 n4 = __ldcg(reinterpret_cast<const uint4*>(a.newbits + w0) + q4);
                 const uint4 v4 = __ldcg(reinterpret_cast<const uint4*>(a.visited + w0) + q4);
                 nb[4 * q4] = n4.x; nb[4 * q4 + 1] = n4.y; nb[4 * q4 + 2] = n4.z; nb[4 * q4 + 3] = n4.w;
-                nw[4 * q4] = n4.x & ~v4.x; nw[4 * q4 + 1] = n4.y & ~v4.y;
-                nw[4 * q4 + 2] = n4.z & ~v4.z; nw[4 * q4 + 3] = n4.w & ~v4.w;
+                vs[4 * q4] = v4.x; vs[4 * q4 + 1] = v4.y; vs[4 * q4 + 2] = v4.z; vs[4 * q4 + 3] = v4.w;
             }
         } else {
 #pragma unroll
             for (int q = 0; q < kScanWords; q++) {
                 const int64_t w = w0 + q;
                 nb[q] = w < a.n_words ? __ldcg(a.newbits + w) : 0u;
-                nw[q] = w < a.n_words ? nb[q] & ~__ldcg(a.visited + w) : 0u;
+                vs[q] = w < a.n_words ? __ldcg(a.visited + w) : 0u;
             }
         }
+        int cnt = 0;
 #pragma unroll
-        for (int q = 0; q < kScanWords; q++) cnt += __popc(nw[q]);
+        for (int q = 0; q < kScanWords; q++) cnt += __popc(nb[q] & ~vs[q]);
         int64_t agg;
         const int64_t excl = dev::block_exclusive_scan<kBitscanThreads>(cnt, &agg, s_red);
         const int64_t prefix = dev::lookback_block<kBitscanThreads>(a.tile_status, tile, agg, s_red, &s_nearest);
@@ -369,7 +368,8 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
 #pragma unroll
         for (int q = 0; q < kScanWords; q++) {
             const int64_t w = w0 + q;
-            uint32_t bits = nw[q];
+            const uint32_t nw = nb[q] & ~vs[q];
+            uint32_t bits = nw;
             while (bits) {
                 const int b = __ffs(bits) - 1;
                 bits &= bits - 1;
@@ -378,10 +378,8 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
                 a.lidx[id] = (int32_t)pos;
                 pos++;
             }
-            if (nb[q]) {
-                a.newbits[w] = 0u;
-                a.visited[w] |= nw[q];
-            }
+            if (nb[q]) a.newbits[w] = 0u;
+            if (nw) a.visited[w] = vs[q] | nw;  // no re-read: the tile owns its words
         }
         __syncthreads();
     }

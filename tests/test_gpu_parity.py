@@ -68,12 +68,13 @@ def test_sample_fanouts_and_ragged(orc, c1, fanout, n_seeds):
     assert_same_sample(got, want)
 
 
+@pytest.mark.parametrize("knob", ["MOMENT_HOP_WARP"])
 @pytest.mark.parametrize("fanout", [[15, 10, 5], [7, 3], [20]])
-def test_sample_power_of_two_tiles(orc, c1, fanout, monkeypatch):
-    """The power-of-two lane-tile sampler (MOMENT_HOP_WARP=0; always used for k > 32) gives the same result as
-    the warp-segmented one (the default for k <= 32)."""
+def test_sample_kernel_variants(orc, c1, fanout, knob, monkeypatch):
+    """The other sampler kernel gives the same result as the default: MOMENT_HOP_WARP=0 selects the
+    power-of-two lane tiles (always used for k > 32)."""
     _, g = c1
-    monkeypatch.setenv("MOMENT_HOP_WARP", "0")
+    monkeypatch.setenv(knob, "0")
     seeds = np.random.default_rng(5).choice(g.n, 1000, replace=False)
     got, want = sample_both(orc, g, seeds, fanout, 4242)
     assert_same_sample(got, want)
