@@ -110,6 +110,48 @@ def test_maxflow_closed_forms(orc):
         orc.maxflow(3, [(0, 1, INF), (1, 2, INF)], 0, 2)  # unbounded
 
 
+def _server(rng, k, with_nvlink):
+    """s, host bins (2), PCIe switches (2), GPU ports (k), NVSwitch, compute nodes (k), t; links in MB/s."""
+    s, t = 0, 1
+    host = [2, 3]
+    sw = [4, 5]
+    port = [6 + g for g in range(k)]
+    nvsw = 6 + k
+    comp = [7 + k + g for g in range(k)]
+    n = 7 + 2 * k
+    links = [(s, h, INF) for h in host]
+    links += [(host[j], sw[j], int(rng.integers(10, 60))) for j in range(2)]
+    links += [(host[0], host[1], int(rng.integers(1, 20))), (host[1], host[0], int(rng.integers(1, 20)))]  # UPI
+    links += [(sw[g * 2 // k], port[g], int(rng.integers(5, 30))) for g in range(k)]
+    links += [(port[g], comp[g], INF) for g in range(k)]
+    if with_nvlink:
+        for g in range(k):
+            c = int(rng.integers(50, 200))
+            links += [(port[g], nvsw, c), (nvsw, comp[g], c)]
+    links += [(comp[g], t, INF) for g in range(k)]
+    return n, links, s, t
+
+
+@pytest.mark.parametrize("seed", range(20))
+def test_maxflow_nvlink_never_hurts(orc, seed):
+    """Planner sanity: removing the NVLink edges can never increase the max-flow. With every
+    compute node an infinite sink (c(v_c, t) = inf) the rate max-flow is the host ingest capacity,
+    so here NVLink leaves it unchanged: its value shows up in the per-GPU time plan (R11), not in F."""
+    k = 4
+    rng = np.random.default_rng(seed)
+    n, with_nv, s, t = _server(rng, k, True)
+    rng = np.random.default_rng(seed)
+    _, without, _, _ = _server(rng, k, False)
+    f_with = orc.maxflow(n, with_nv, s, t)[0]
+    f_without = orc.maxflow(n, without, s, t)[0]
+    assert f_without <= f_with
+    assert f_without == f_with
+    assert f_with == brute_min_cut(n, with_nv, s, t) if n <= 16 else True
+    # the NVLink fabric cannot carry more than the host side supplies: F <= sum of host egress + UPI
+    host_out = sum(c for (u, v, c) in with_nv if u in (2, 3) and v in (4, 5))
+    assert f_with <= host_out
+
+
 def _tb(orc, n, links, supply_idx, s, t):
     sup = [1 if i in supply_idx else 0 for i in range(len(links))]
     return orc.time_bisect(n, links, sup, s, t)
