@@ -270,13 +270,21 @@ def main():
         run_reference(args, rank, world)
         return
     assert args.warmup >= 3, "W >= 3 warm-up steps"
+    # MOMENT_BENCH_SHARED_GPU=1 (test only): every rank on cuda:0 with a gloo group, to exercise the
+    # multi-rank code path on a one-GPU box (NCCL refuses two ranks on one device). Never a bench number.
+    shared = os.environ.get("MOMENT_BENCH_SHARED_GPU") == "1"
+    if shared:
+        local = 0
     torch.cuda.set_device(local)
     dev = f"cuda:{local}"
     dist = None
     if world > 1:
         import torch.distributed as dist
 
-        dist.init_process_group("nccl", device_id=torch.device(dev))
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device(dev))
     st = build_state(args.config, dev, rank, world, args.inflight)
     H = len(st.fanout)
     P = len(st.lanes)
@@ -390,7 +398,8 @@ def main():
                        "parallelism": f"dp{world} (replicated graph+features)",
                        "l2": "inputs larger than L2 (features %.2f GB, CSR %.2f GB)" % (
                            st.table.numel() / 1e9, (st.graph.indptr.numel() * 8 + st.graph.indices.numel() * 4) / 1e9),
-                       "mean_F_H": sum(nF) / args.steps},
+                       "mean_F_H": sum(nF) / args.steps,
+                       **({"test_mode": "all ranks share cuda:0 over gloo: not a bench number"} if shared else {})},
             "gather_GBs": gather_gbs,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": profile_traffic(args.config), "kernel": "gather_bulk_kernel",
