@@ -297,10 +297,37 @@ moment_status moment_relay_serve(moment_ctx_t ctx, const uint64_t* words, const 
 moment_status moment_relay_scatter(moment_ctx_t ctx, const uint64_t* words, const int64_t* n_dev, int64_t max_n,
                                    const void* rows, void* out, void* stream);
 
+/* ================================================================================================
+ * H5 exchange over peer memory (one process per GPU, no all-to-all). Every rank owns an
+ * inbox (device uint64 [world][cap][2]) and inbox counts (device int64 [world]); peers map them, and each
+ * other's batch outputs, with moment_ipc_import (NVLink peer pointers on one node). Per batch:
+ *   moment_bucket, moment_gather_routed (as above), then
+ *   moment_relay_push       : the requests this rank routes through rank h are written straight into h's
+ *                             inbox slot for this rank (peer stores): peer_inbox[h] = &inbox_h[self][0][0],
+ *                             and their number into peer_count[h] = &count_h[self] (0 when none); entries
+ *                             for h == self are ignored (may be NULL). Requests beyond cap: MOMENT_EOVERFLOW
+ *                             is not detectable on the device, so the caller sizes cap >= max_n.
+ *   (caller) barrier: every rank's pushes are complete and visible (stream synchronize + process barrier)
+ *   moment_relay_serve_push : for every source g != self, the min(count[g], cap) requests of inbox[g] are
+ *                             read from THIS rank's mapping of the host bins (its PCIe link) and stored
+ *                             straight into g's output (peer stores): peer_out[g] = g's out base,
+ *                             out_g[position] = row. peer_out[self] is ignored.
+ *   (caller) barrier: every served row is complete before the requesters read their outputs.
+ * Host arrays peer_inbox / peer_count / peer_out have `world` entries; world <= MOMENT_MAX_WORLD.
+ * Byte-exact with moment_gather of the same ids.
+ * ================================================================================================ */
+#define MOMENT_MAX_WORLD 64
+moment_status moment_relay_push(moment_ctx_t ctx, const int64_t* ids, int64_t max_n, const int64_t* qoff,
+                                const int64_t* qpos, uint64_t* const* peer_inbox, int64_t* const* peer_count,
+                                void* stream);
+moment_status moment_relay_serve_push(moment_ctx_t ctx, const uint64_t* inbox, const int64_t* inbox_count,
+                                      int64_t cap, void* const* peer_out, void* stream);
+
 /* Cross-process device memory (another rank's HBM bin mapped into this process: the NVLink peer
  * pointer of bin_ptr). export: 64-byte handle of the allocation containing dptr and dptr's byte offset in
  * it; import: map the allocation (peer access enabled lazily) and return its base (add the offset);
- * close: unmap (pass the base). */
+ * close: unmap (pass the base). Imports are reference-counted per handle (several exported buffers may share
+ * one allocation): every import needs its own close, the mapping goes away with the last. */
 #define MOMENT_IPC_HANDLE_BYTES 64
 moment_status moment_ipc_export(const void* dptr, uint8_t* handle, int64_t* offset);
 moment_status moment_ipc_import(const uint8_t* handle, void** dptr);

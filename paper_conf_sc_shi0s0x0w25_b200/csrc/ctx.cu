@@ -474,6 +474,25 @@ extern "C" moment_status moment_relay_scatter(moment_ctx_t ctx, const uint64_t* 
     return launch_relay_scatter(ctx, words, n_dev, max_n, rows, out, static_cast<cudaStream_t>(stream));
 }
 
+extern "C" moment_status moment_relay_push(moment_ctx_t ctx, const int64_t* ids, int64_t max_n, const int64_t* qoff,
+                                           const int64_t* qpos, uint64_t* const* peer_inbox, int64_t* const* peer_count,
+                                           void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_relay_push"));
+    if (max_n < 0 || (max_n > 0 && (!ids || !qoff || !qpos)) || !peer_inbox || !peer_count)
+        return fail(MOMENT_EINVAL, "moment_relay_push: null argument");
+    return launch_relay_push(ctx, ids, qoff, qpos, max_n, peer_inbox, peer_count, static_cast<cudaStream_t>(stream));
+}
+
+extern "C" moment_status moment_relay_serve_push(moment_ctx_t ctx, const uint64_t* inbox, const int64_t* inbox_count,
+                                                 int64_t cap, void* const* peer_out, void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_relay_serve_push"));
+    if (cap < 0 || !inbox || !inbox_count || !peer_out) return fail(MOMENT_EINVAL, "moment_relay_serve_push: null argument");
+    if (ctx->n_bins <= 0) return fail(MOMENT_EINVAL, "moment_relay_serve_push: ctx has no bins");
+    if (cap * (ctx->row_bytes / 16) >= (int64_t(1) << 40))
+        return fail(MOMENT_EUNSUPPORTED, "moment_relay_serve_push: cap %lld too large", (long long)cap);
+    return launch_relay_serve_push(ctx, inbox, inbox_count, cap, peer_out, static_cast<cudaStream_t>(stream));
+}
+
 // ---- cross-process device memory (peer HBM bins of other ranks) -------------------------------------
 static_assert(sizeof(cudaIpcMemHandle_t) == MOMENT_IPC_HANDLE_BYTES, "IPC handle size");
 
@@ -502,13 +521,42 @@ extern "C" moment_status moment_ipc_export(const void* dptr, uint8_t* handle, in
     return MOMENT_OK;
 }
 
+// An allocation can be opened only once per process, but several exported buffers may live in one
+// allocation (a caching allocator's segment): imports are reference-counted per handle.
+namespace {
+std::mutex g_ipc_mu;
+struct IpcMapping {
+    std::string handle;
+    void* base;
+    int refs;
+};
+std::vector<IpcMapping> g_ipc;
+}  // namespace
+
 extern "C" moment_status moment_ipc_import(const uint8_t* handle, void** dptr) {
     if (!dptr || !handle) return fail(MOMENT_EINVAL, "moment_ipc_import: null argument");
+    std::lock_guard<std::mutex> lock(g_ipc_mu);
+    const std::string key(reinterpret_cast<const char*>(handle), MOMENT_IPC_HANDLE_BYTES);
+    for (auto& m : g_ipc)
+        if (m.handle == key) {
+            m.refs++;
+            *dptr = m.base;
+            return MOMENT_OK;
+        }
     cudaIpcMemHandle_t h;
     std::memcpy(&h, handle, sizeof(h));
-    return cuda_check(cudaIpcOpenMemHandle(dptr, h, cudaIpcMemLazyEnablePeerAccess), "moment_ipc_import");
+    MOMENT_TRY(cuda_check(cudaIpcOpenMemHandle(dptr, h, cudaIpcMemLazyEnablePeerAccess), "moment_ipc_import"));
+    g_ipc.push_back({key, *dptr, 1});
+    return MOMENT_OK;
 }
 
 extern "C" moment_status moment_ipc_close(void* dptr) {
+    std::lock_guard<std::mutex> lock(g_ipc_mu);
+    for (size_t i = 0; i < g_ipc.size(); i++)
+        if (g_ipc[i].base == dptr) {
+            if (--g_ipc[i].refs > 0) return MOMENT_OK;
+            g_ipc.erase(g_ipc.begin() + (long)i);
+            break;
+        }
     return cuda_check(cudaIpcCloseMemHandle(dptr), "moment_ipc_close");
 }

@@ -112,6 +112,11 @@ moment_status launch_relay_serve(moment_ctx_s* ctx, const uint64_t* words, const
                                  void* rows, cudaStream_t stream);
 moment_status launch_relay_scatter(moment_ctx_s* ctx, const uint64_t* words, const int64_t* n_dev, int64_t max_n,
                                    const void* rows, void* out, cudaStream_t stream);
+moment_status launch_relay_push(moment_ctx_s* ctx, const int64_t* ids, const int64_t* qoff, const int64_t* qpos,
+                                int64_t max_n, uint64_t* const* peer_inbox, int64_t* const* peer_count,
+                                cudaStream_t stream);
+moment_status launch_relay_serve_push(moment_ctx_s* ctx, const uint64_t* inbox, const int64_t* inbox_count, int64_t cap,
+                                      void* const* peer_out, cudaStream_t stream);
 moment_status configure_sample_kernels(int carveout);
 moment_status configure_gather_kernels(int carveout);
 

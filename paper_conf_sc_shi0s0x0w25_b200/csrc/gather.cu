@@ -465,6 +465,8 @@ moment_status launch_bucket(moment_ctx_s* ctx, const int64_t* ids, const int64_t
     const int32_t Q = ctx->n_bins * ctx->world;
     if (Q > kMaxQueues) return fail(MOMENT_EUNSUPPORTED, "moment_bucket: n_bins * world = %d > %d", Q, kMaxQueues);
     MOMENT_TRY(cuda_pending("moment_bucket: pending CUDA error"));
+    if (max_n == 0)  // no requests: empty queues (the tile kernels below would read stale tile counts)
+        return cuda_check(cudaMemsetAsync(qoff, 0, (size_t)(Q + 1) * sizeof(int64_t), stream), "moment_bucket: empty");
     const int64_t n_tiles = std::max<int64_t>(1, (max_n + kBucketTile - 1) / kBucketTile);
     const int grid = (int)std::min<int64_t>(n_tiles, 148 * 2);
     bucket_count_kernel<<<grid, 256, 0, stream>>>(ctx->placement, ids, n_dev, max_n, ctx->n_bins, ctx->bk_tile_counts);
@@ -575,6 +577,81 @@ __global__ void __launch_bounds__(kGatherThreads) relay_scatter_kernel(const uin
     }
 }
 
+// ---- the same exchange over peer memory (no all-to-all) ------------------------------------------------
+struct PeerInboxes {
+    uint64_t* inbox[MOMENT_MAX_WORLD];  // rank h's inbox slot for this rank (peer pointer)
+    int64_t* count[MOMENT_MAX_WORLD];   // rank h's count slot for this rank (peer pointer)
+};
+struct PeerOuts {
+    int4* out[MOMENT_MAX_WORLD];  // rank g's batch output (peer pointer)
+};
+
+// relay_pack with the words stored straight into the destination rank's inbox: one 16-byte peer store per
+// request (placement word, output position), and the per-destination count into the peer's count slot.
+__global__ void relay_push_kernel(BinTable bins, const uint64_t* __restrict__ placement, const int64_t* __restrict__ ids,
+                                  const int64_t* __restrict__ qoff, const int64_t* __restrict__ qpos, int32_t n_bins,
+                                  int32_t world, int32_t self, PeerInboxes peers) {
+    __shared__ int64_t s_src[kMaxSegs + 1], s_dst[kMaxSegs + 1], s_hbase[MOMENT_MAX_WORLD];
+    __shared__ int s_h[kMaxSegs + 1];
+    __shared__ int s_n;
+    if (threadIdx.x == 0) {
+        s_n = build_segments(qoff, bins, n_bins, world, self, s_src, s_dst, s_h);
+        for (int h = 0; h < world; h++) s_hbase[h] = -1;
+        for (int s = s_n - 1; s >= 0; s--) s_hbase[s_h[s]] = s_dst[s];  // first word of destination h
+    }
+    __syncthreads();
+    const int ns = s_n;
+    if (blockIdx.x == 0 && threadIdx.x < world && (int)threadIdx.x != self) {
+        int64_t c = 0;
+        for (int s = 0; s < ns; s++)
+            if (s_h[s] == (int)threadIdx.x) c += s_dst[s + 1] - s_dst[s];
+        *peers.count[threadIdx.x] = c;
+    }
+    const int64_t total = s_dst[ns];
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+        int lo = 0, hi = ns - 1;
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (s_dst[mid] <= e) lo = mid;
+            else hi = mid - 1;
+        }
+        const int h = s_h[lo];
+        const int64_t i = __ldg(qpos + s_src[lo] + (e - s_dst[lo]));
+        const ulonglong2 w = make_ulonglong2(__ldg(placement + __ldg(ids + i)), (unsigned long long)i);
+        reinterpret_cast<ulonglong2*>(peers.inbox[h])[e - s_hbase[h]] = w;
+    }
+}
+
+// Serve every source rank's inbox: read the host row named by each request from THIS rank's mapping of
+// the host bins and store it straight into the source's output row (peer stores).
+__global__ void __launch_bounds__(kGatherThreads) relay_serve_push_kernel(BinTable bins, const uint64_t* __restrict__ inbox,
+                                                                          const int64_t* __restrict__ inbox_count,
+                                                                          int64_t cap, int32_t world, int32_t self,
+                                                                          FastDiv rv, int64_t stride_vec, PeerOuts outs) {
+    __shared__ int64_t s_off[MOMENT_MAX_WORLD + 1];
+    if (threadIdx.x == 0) {
+        int64_t o = 0;
+        for (int g = 0; g < world; g++) {
+            s_off[g] = o;
+            o += g == self ? 0 : min(max(inbox_count[g], (int64_t)0), cap);
+        }
+        s_off[world] = o;
+    }
+    __syncthreads();
+    const int64_t total = s_off[world] * rv.d;
+    for (int64_t v = (int64_t)blockIdx.x * kGatherThreads + threadIdx.x; v < total; v += (int64_t)gridDim.x * kGatherThreads) {
+        const int64_t e = v / rv.d;
+        const int col = (int)(v - e * rv.d);
+        int g = 0;
+        while (s_off[g + 1] <= e) g++;
+        const int64_t r = e - s_off[g];
+        const uint64_t* w = inbox + 2 * ((int64_t)g * cap + r);
+        const uint64_t p = __ldg(w), pos = __ldg(w + 1);
+        outs.out[g][(int64_t)pos * rv.d + col] =
+            ld_stream(bins.base[(int)(p >> 40)] + (int64_t)(p & kSlotMask) * stride_vec + col);
+    }
+}
+
 }  // namespace
 
 moment_status launch_relay_pack(moment_ctx_s* ctx, const int64_t* ids, const int64_t* qoff, const int64_t* qpos,
@@ -607,6 +684,45 @@ moment_status launch_relay_scatter(moment_ctx_s* ctx, const uint64_t* words, con
         words, n_dev, max_n, make_fastdiv((uint32_t)rv), reinterpret_cast<const int4*>(rows),
         reinterpret_cast<int4*>(out));
     return cuda_check(cudaGetLastError(), "moment_relay_scatter: launch");
+}
+
+moment_status launch_relay_push(moment_ctx_s* ctx, const int64_t* ids, const int64_t* qoff, const int64_t* qpos,
+                                int64_t max_n, uint64_t* const* peer_inbox, int64_t* const* peer_count,
+                                cudaStream_t stream) {
+    if (!ctx->placement) return fail(MOMENT_EINVAL, "moment_relay_push: ctx has no placement map");
+    if (ctx->world > MOMENT_MAX_WORLD) return fail(MOMENT_EUNSUPPORTED, "moment_relay_push: world > %d", MOMENT_MAX_WORLD);
+    if (ctx->n_bins * (ctx->world - 1) > kMaxSegs) return fail(MOMENT_EUNSUPPORTED, "moment_relay_push: too many segments");
+    PeerInboxes p{};
+    for (int h = 0; h < ctx->world; h++) {
+        if (h == ctx->rank) continue;
+        if (!peer_inbox[h] || !peer_count[h] || (reinterpret_cast<uintptr_t>(peer_inbox[h]) & 15))
+            return fail(MOMENT_EINVAL, "moment_relay_push: peer %d inbox / count null or inbox not 16-byte aligned", h);
+        p.inbox[h] = peer_inbox[h];
+        p.count[h] = peer_count[h];
+    }
+    const int grid = grid_for(std::max<int64_t>(max_n, 1), 256, 148 * 4);
+    relay_push_kernel<<<grid, 256, 0, stream>>>(make_bins(ctx), ctx->placement, ids, qoff, qpos, ctx->n_bins, ctx->world,
+                                                ctx->rank, p);
+    return cuda_check(cudaGetLastError(), "moment_relay_push: launch");
+}
+
+moment_status launch_relay_serve_push(moment_ctx_s* ctx, const uint64_t* inbox, const int64_t* inbox_count, int64_t cap,
+                                      void* const* peer_out, cudaStream_t stream) {
+    if (ctx->world > MOMENT_MAX_WORLD) return fail(MOMENT_EUNSUPPORTED, "moment_relay_serve_push: world > %d", MOMENT_MAX_WORLD);
+    PeerOuts o{};
+    for (int g = 0; g < ctx->world; g++) {
+        if (g == ctx->rank) continue;
+        if (!peer_out[g] || (reinterpret_cast<uintptr_t>(peer_out[g]) & 15))
+            return fail(MOMENT_EINVAL, "moment_relay_serve_push: peer %d output null or not 16-byte aligned", g);
+        o.out[g] = reinterpret_cast<int4*>(peer_out[g]);
+    }
+    const int64_t rv = ctx->row_bytes / 16;
+    // grid sized for the worst case (every source's full inbox); blocks without work exit at once
+    const int grid = grid_for(std::max<int64_t>(cap * (ctx->world - 1) * rv, 1), kGatherThreads, 148 * 8);
+    relay_serve_push_kernel<<<grid, kGatherThreads, 0, stream>>>(make_bins(ctx), inbox, inbox_count, cap, ctx->world,
+                                                                 ctx->rank, make_fastdiv((uint32_t)rv),
+                                                                 ctx->row_stride / 16, o);
+    return cuda_check(cudaGetLastError(), "moment_relay_serve_push: launch");
 }
 
 // Kernel attributes, set once per device: every kernel of the library asks for the same shared-memory

@@ -90,3 +90,74 @@ def gather_exchange(ctx, ids: torch.Tensor, out: torch.Tensor, bufs: ExchangeBuf
         if n_send:
             ctx.relay_scatter(bufs.words, rows_back, out, n=n_send, stream=s)
     return {"sent": send, "served": recv}
+
+
+class PeerExchange:
+    """H5 over peer memory (one process per GPU, no all-to-all): requests are stored straight into the
+    relay rank's inbox and served rows straight into the requester's output, both by libmoment.so kernels
+    through CUDA-IPC-mapped peer pointers (NVLink loads/stores between the GPUs of one node).
+
+    Setup is collective over `group`: this rank allocates its inbox (int64 [world][cap][2]), inbox counts
+    (int64 [world]) and batch output (uint8 [cap][R]), exports them, and maps every peer's. Per batch
+    (`gather`): bucket -> routed gather (own rows) -> relay_push (peer stores) -> barrier -> relay_serve_push
+    (peer stores into the requesters' outputs) -> barrier. The two barriers are the only host
+    synchronisation; with NCCL they are device collectives, with gloo host ones.
+    """
+
+    def __init__(self, ctx, max_n: int, row_bytes: int, device, group=None):
+        import paper_conf_sc_shi0s0x0w25_b200 as M
+
+        self.M, self.ctx, self.group = M, ctx, group
+        self.world, self.rank = ctx.world, ctx.rank
+        self.cap = max(1, int(max_n))
+        dev = torch.device(device)
+        self.inbox = torch.zeros((self.world, self.cap, 2), dtype=torch.int64, device=dev)
+        self.count = torch.zeros(self.world, dtype=torch.int64, device=dev)
+        self.out = torch.zeros((self.cap, row_bytes), dtype=torch.uint8, device=dev)
+        self.route = torch.empty(self.cap, dtype=torch.int32, device=dev)
+        self.qoff = torch.empty(64 * self.world + 1, dtype=torch.int64, device=dev)
+        self.qpos = torch.empty(self.cap, dtype=torch.int64, device=dev)
+        mine = [M.ipc_export(t) for t in (self.inbox, self.count, self.out)]
+        everyone = [None] * self.world
+        dist.all_gather_object(everyone, mine, group=group)
+        self._bases = []
+        self.peer_inbox = [0] * self.world
+        self.peer_count = [0] * self.world
+        self.peer_out = [0] * self.world
+        slot_bytes = self.cap * 2 * 8
+        for h in range(self.world):
+            if h == self.rank:
+                continue
+            addr = []
+            for handle, off in everyone[h]:
+                base = M.ipc_import(handle)
+                self._bases.append(base)
+                addr.append(base + off)
+            self.peer_inbox[h] = addr[0] + self.rank * slot_bytes  # rank h's inbox slot for this rank
+            self.peer_count[h] = addr[1] + self.rank * 8
+            self.peer_out[h] = addr[2]
+        dist.barrier(group=group)
+
+    def gather(self, ids: torch.Tensor, n: int, stream=None) -> torch.Tensor:
+        """Collective: returns this rank's output view [n, R] = rows of ids[:n]."""
+        assert n <= self.cap
+        s = stream if stream is not None else torch.cuda.current_stream(ids.device)
+        ctx = self.ctx
+        with torch.cuda.stream(s):
+            ctx.bucket(ids, self.route, self.qoff, self.qpos, max_n=n, stream=s)
+            ctx.gather_routed(ids, self.route, self.out, max_n=n, stream=s)
+            ctx.relay_push(ids, self.qoff, self.qpos, self.peer_inbox, self.peer_count, max_n=n, stream=s)
+        s.synchronize()
+        dist.barrier(group=self.group)  # every rank's requests are in its relays' inboxes
+        with torch.cuda.stream(s):
+            ctx.relay_serve_push(self.inbox, self.count, self.cap, self.peer_out, stream=s)
+        s.synchronize()
+        dist.barrier(group=self.group)  # every relayed row is in its requester's output
+        return self.out[:n]
+
+    def close(self):
+        """Collective: unmap the peers' buffers once every rank is done with them."""
+        dist.barrier(group=self.group)
+        for b in self._bases:
+            self.M.ipc_close(b)
+        self._bases = []

@@ -29,8 +29,10 @@ EXPORTED = [
     "moment_plan_free", "moment_ctx_create", "moment_ctx_free", "moment_ctx_workspace_bytes", "moment_sample_bounds",
     "moment_sample", "moment_sample_check", "moment_hotness", "moment_bucket", "moment_gather", "moment_gather_group",
     "moment_step", "moment_step_host", "moment_gather_routed", "moment_relay_pack", "moment_relay_serve",
-    "moment_relay_scatter", "moment_ipc_export", "moment_ipc_import", "moment_ipc_close",
+    "moment_relay_scatter", "moment_relay_push", "moment_relay_serve_push", "moment_ipc_export", "moment_ipc_import",
+    "moment_ipc_close",
 ]
+MAX_WORLD = 64
 
 
 class MomentError(RuntimeError):
@@ -124,6 +126,8 @@ def lib():
             "moment_relay_pack": ([P, P, I64, P, P, P, P, P], I32),
             "moment_relay_serve": ([P, P, P, I64, P, P], I32),
             "moment_relay_scatter": ([P, P, P, I64, P, P, P], I32),
+            "moment_relay_push": ([P, P, I64, P, P, P, P, P], I32),
+            "moment_relay_serve_push": ([P, P, P, I64, P, P], I32),
             "moment_ipc_export": ([P, P, P], I32),
             "moment_ipc_import": ([P, P], I32),
             "moment_ipc_close": ([P], I32),
@@ -435,6 +439,22 @@ class Ctx:
     def relay_scatter(self, words, rows, out, *, n: int, stream=None):
         _check(lib().moment_relay_scatter(self.handle, words.data_ptr(), None, n, rows.data_ptr(), out.data_ptr(),
                                           _stream(stream)))
+
+    # ---- the same exchange over peer memory (see exchange.PeerExchange) ----
+    def relay_push(self, ids, qoff, qpos, peer_inbox: list[int], peer_count: list[int], *, max_n: int | None = None,
+                   stream=None):
+        """peer_inbox[h] / peer_count[h]: device addresses of rank h's inbox / count slot for this rank."""
+        mn = ids.numel() if max_n is None else max_n
+        inb = (C.c_void_p * len(peer_inbox))(*[p or None for p in peer_inbox])
+        cnt = (C.c_void_p * len(peer_count))(*[p or None for p in peer_count])
+        _check(lib().moment_relay_push(self.handle, ids.data_ptr(), mn, qoff.data_ptr(), qpos.data_ptr(),
+                                       C.cast(inb, P), C.cast(cnt, P), _stream(stream)))
+
+    def relay_serve_push(self, inbox, inbox_count, cap: int, peer_out: list[int], *, stream=None):
+        """Serve every source's inbox into its output (peer_out[g]: device address of rank g's output)."""
+        outs = (C.c_void_p * len(peer_out))(*[p or None for p in peer_out])
+        _check(lib().moment_relay_serve_push(self.handle, inbox.data_ptr(), inbox_count.data_ptr(), cap,
+                                             C.cast(outs, P), _stream(stream)))
 
 
 IPC_HANDLE_BYTES = 64

@@ -235,6 +235,10 @@ def test_gather_tiered_and_bucket_vs_oracle(orc, c1):
     assert np.array_equal(route.cpu().numpy(), o_route)
     assert np.array_equal(qoff.cpu().numpy(), o_qoff)
     assert np.array_equal(qpos.cpu().numpy(), o_qpos)
+    # an empty request list right after a full one: empty queues, not the previous call's tile counts
+    ctx.bucket(ids, route, qoff, qpos, max_n=0)
+    assert not qoff.cpu().numpy().any()
+    assert np.array_equal(orc.bucket(0, world, owners, quota, bin_of[ids.cpu().numpy()[:0]])[1], qoff.cpu().numpy())
     # single-rank gather refuses quotas that relay through another rank
     out = torch.empty((nF, R), dtype=torch.uint8, device=DEV)
     with pytest.raises(M.MomentError) as e:

@@ -16,13 +16,13 @@ from mp_util import run_world
 pytestmark = pytest.mark.gpu
 
 
-def _rank_main(rank, world):
+def _rank_main(rank, world, transport="alltoall"):
     import torch.distributed as dist
 
     import oracle
     import paper_conf_sc_shi0s0x0w25_b200 as M
     import workloads as W
-    from paper_conf_sc_shi0s0x0w25_b200.exchange import ExchangeBuffers, gather_exchange
+    from paper_conf_sc_shi0s0x0w25_b200.exchange import ExchangeBuffers, PeerExchange, gather_exchange
 
     oracle.build()
     torch.cuda.set_device(0)
@@ -72,11 +72,30 @@ def _rank_main(rank, world):
     torch.cuda.synchronize()
     nF = int(bufs.counts[2])
     ids = bufs.nodes[:nF].contiguous()
-    out = torch.zeros((nF, R), dtype=torch.uint8, device=dev)
-    xb = ExchangeBuffers(max_n=nF, row_bytes=R, n_queues=(world + 2) * world, device=torch.device(dev))
-    info = gather_exchange(ctx, ids, out, xb, n=nF)
-    torch.cuda.synchronize()
-    ok = bool(np.array_equal(out.cpu().numpy(), oracle.gather(table.numpy(), ids.cpu().numpy())))
+    want = oracle.gather(table.numpy(), ids.cpu().numpy())
+    if transport == "peer":
+        # the exchange buffers are sized for the largest batch of any rank; two batches check reuse
+        nmax = [None] * world
+        dist.all_gather_object(nmax, int(bufs.nodes.numel()))
+        px = PeerExchange(ctx, max(nmax), R, dev)
+        ok = True
+        for rep in range(2):
+            out = px.gather(ids, nF)
+            torch.cuda.synchronize()
+            ok &= bool(np.array_equal(out.cpu().numpy(), want))
+        # an empty batch on this rank still serves the other's requests
+        out = px.gather(ids, 0 if rank == 0 else nF)
+        torch.cuda.synchronize()
+        if rank == 1:
+            ok &= bool(np.array_equal(out.cpu().numpy(), want))
+        px.close()
+        info = {"sent": [0] * world, "served": [0] * world}
+    else:
+        out = torch.zeros((nF, R), dtype=torch.uint8, device=dev)
+        xb = ExchangeBuffers(max_n=nF, row_bytes=R, n_queues=(world + 2) * world, device=torch.device(dev))
+        info = gather_exchange(ctx, ids, out, xb, n=nF)
+        torch.cuda.synchronize()
+        ok = bool(np.array_equal(out.cpu().numpy(), want))
     dist.barrier()  # every rank done with the others' bins before any mapping goes away
     for base in imported.values():
         M.ipc_close(base)
@@ -91,3 +110,12 @@ def test_gather_exchange_two_processes_one_gpu():
     assert all(r["ok"] for r in res), res
     assert res[0]["sent"][1] == res[1]["served"][0] and res[1]["sent"][0] == res[0]["served"][1]
     assert res[0]["sent"][1] > 0 and res[1]["sent"][0] > 0
+
+
+def test_peer_exchange_two_processes_one_gpu():
+    """The same exchange with no all-to-all: requests and relayed rows move by peer stores into CUDA-IPC
+    mapped inboxes / outputs (moment_relay_push, moment_relay_serve_push), byte-exact with the oracle."""
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    res = run_world(_rank_main, 2, "peer")
+    assert all(r["ok"] for r in res), res
