@@ -419,7 +419,7 @@ def main():
                        **({"test_mode": "all ranks share cuda:0 over gloo: not a bench number"} if shared else {})},
             "gather_GBs": gather_gbs,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                         "traffic": profile_traffic(args.config), "kernel": "gather_bulk_kernel",
+                         "traffic": profile_traffic(args.config), "kernel": "gather_tma4_kernel",
                          "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})",
                          "alg_bytes_per_launch": alg_bytes, "launch_ms": gather_ms,
                          "gather_share_of_step": gather_ms / (ms / args.steps),

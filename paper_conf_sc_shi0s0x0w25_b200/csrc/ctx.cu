@@ -96,8 +96,10 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     c->placement = a->placement;
     if (const char* gp = std::getenv("MOMENT_GATHER_PATH")) {
         const std::string v(gp);
-        c->gather_path = v == "ldg" ? 1 : (v == "bulk" ? 2 : 0);
+        c->gather_path = v == "ldg" ? 1 : (v == "bulk" ? 2 : (v == "tma4" ? 3 : 0));
     }
+    if (const char* v = std::getenv("MOMENT_TMA_PROMO")) c->tma_promo = std::max(0, std::min(3, std::atoi(v)));
+    if (const char* v = std::getenv("MOMENT_TMA4_BLOCKS")) c->tma4_blocks_per_sm = std::max(1, std::atoi(v));
     if (const char* v = std::getenv("MOMENT_BULK"))
         std::sscanf(v, "%d,%d,%d", &c->bulk_stages, &c->bulk_blocks_per_sm, &c->bulk_stage_kb);
     if (const char* v = std::getenv("MOMENT_HOP_GRID")) c->hop_grid_per_sm = std::max(1, std::atoi(v));

@@ -1,5 +1,6 @@
 // ctx.h — device context of one rank and the small device helpers shared by the kernels.
 #pragma once
+#include <cuda.h>  // CUtensorMap (type only: the encoder is resolved through cudaGetDriverEntryPoint)
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -19,7 +20,14 @@ struct moment_ctx_s {
     int64_t max_nodes = 0, max_edges = 0, max_offsets = 0;
     int64_t row_bytes = 0, row_stride = 0;
     int32_t n_bins = 0;
-    int32_t gather_path = 0;  // 0 auto (TMA bulk copies for local rows), 1 LDG.128 only, 2 bulk (MOMENT_GATHER_PATH)
+    int32_t gather_path = 0;  // 0 auto (TMA bulk copies for local rows), 1 LDG.128 only, 2 bulk, 3 tma4 (MOMENT_GATHER_PATH)
+    // tile::gather4 tensor map of the replicated table (built on first use) and its L2 promotion
+    CUtensorMap tma_map{};
+    const void* tma_base = nullptr;
+    // L2 promotion of the gathered rows: 64 B (measured: a 400-byte row then costs 448 B of DRAM reads instead
+    // of the 512 B whole 128-byte lines the default fetches; MOMENT_TMA_PROMO: 0 none, 1 64B, 2 128B, 3 256B)
+    int32_t tma_promo = 1;
+    int32_t tma4_blocks_per_sm = 3;  // 1-warp gather4 blocks per SM, 4 stages of 8 x 4 rows (MOMENT_TMA4_BLOCKS)
     int32_t l2_load_policy = 0, l2_store_policy = 1;  // bulk gather L2 hints: 0 normal, 1 evict_first, 2 evict_last
     int32_t hop_grid_per_sm = 4, compact_grid_per_sm = 1;  // launch caps (MOMENT_HOP_GRID / MOMENT_COMPACT_GRID)
     int32_t hop_nodes_per_group = 4;  // nodes per lane group on large frontiers (MOMENT_HOP_Q: 1, 2, 4, 8)

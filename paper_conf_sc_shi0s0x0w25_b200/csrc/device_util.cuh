@@ -34,6 +34,24 @@ __device__ __forceinline__ uint32_t uniform(uint32_t r, uint32_t m) {
     return (uint32_t)(((uint64_t)r * (uint64_t)m) >> 32);
 }
 
+// Read-only random loads with a 64-byte L2 fetch size hint (the default fetches the whole 128-byte line a
+// lone 4- or 8-byte read touches).
+__device__ __forceinline__ int32_t ld_rand(const int32_t* p) {
+    int32_t v;
+    asm("ld.global.nc.L2::64B.b32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ int64_t ld_rand(const int64_t* p) {
+    int64_t v;
+    asm("ld.global.nc.L2::64B.b64 %0, [%1];" : "=l"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ uint64_t ld_rand(const uint64_t* p) {
+    uint64_t v;
+    asm("ld.global.nc.L2::64B.b64 %0, [%1];" : "=l"(v) : "l"(p));
+    return v;
+}
+
 // Block-wide exclusive scan of one int64 per thread (blockDim.x == NT, multiple of 32).
 template <int NT>
 __device__ __forceinline__ int64_t block_exclusive_scan(int64_t x, int64_t* total, int64_t* warp_sums) {

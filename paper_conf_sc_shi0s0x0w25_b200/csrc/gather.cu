@@ -19,9 +19,11 @@ struct BinTable {
     int8_t owner[MOMENT_MAX_BINS];      // owning rank of an HBM bin, -1 for a host-DRAM bin
 };
 
+// Row vectors: no L1 allocation, 64-byte L2 fetch size (a row fetches its 64-byte chunks, not whole 128-byte
+// lines: profiles/r01_dram_granularity.txt).
 __device__ __forceinline__ int4 ld_stream(const int4* p) {
     int4 r;
-    asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0, %1, %2, %3}, [%4];"
+    asm volatile("ld.global.nc.L1::no_allocate.L2::64B.v4.s32 {%0, %1, %2, %3}, [%4];"
                  : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
                  : "l"(p));
     return r;
@@ -63,7 +65,7 @@ __global__ void __launch_bounds__(kGatherThreads) gather_kernel(BinTable bins, c
                 const int64_t id = __ldg(ids + row);
                 const int4* src;
                 if (placement) {
-                    const uint64_t p = __ldg(placement + id);
+                    const uint64_t p = dev::ld_rand(placement + id);
                     const int b = (int)(p >> 40);
                     if (route && bins.owner[b] < 0 && (__ldg(route + row) % world) != self) {
                         live[u] = false;
@@ -143,7 +145,7 @@ __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wa
 __device__ __forceinline__ const char* row_src(const BinTable& bins, const uint64_t* placement, int64_t id,
                                                int64_t stride) {
     if (placement) {
-        const uint64_t p = __ldg(placement + id);
+        const uint64_t p = dev::ld_rand(placement + id);
         return reinterpret_cast<const char*>(bins.base[(int)(p >> 40)]) + (int64_t)(p & kSlotMask) * stride;
     }
     return reinterpret_cast<const char*>(bins.base[0]) + id * stride;
@@ -209,6 +211,80 @@ __global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const ui
         }
     }
     if (lane == 0) bulk_wait_all();
+}
+
+// TMA tile::gather4 variant of the bulk gather (sm_100a): one tensor copy fetches FOUR rows of the
+// replicated table (a 2-D tensor map over [n rows][R / 4 words] with the table's row stride), so a
+// 32-row tile is 8 copies instead of 32. The tensor map also carries the L2 promotion (fetch) size of the
+// reads. Each group of 4 rows lands at a 128-byte aligned smem slot (G bytes) and is stored back with its
+// own bulk copy (per-lane bulk groups). Rows past the end of a tile repeat the tile's first row and are
+// not stored.
+constexpr int kTma4Rows = 32;  // rows per tile = 8 groups of 4
+template <int kStages>
+__global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                         const int64_t* __restrict__ ids, const int64_t* n_dev,
+                                                         int64_t max_n, uint32_t R, int l2_store, char* __restrict__ out) {
+    extern __shared__ __align__(128) char stage[];  // kStages * 8 * G
+    __shared__ __align__(8) uint64_t full[kStages];
+    const int lane = threadIdx.x;
+    const uint32_t G = (4 * R + 127) & ~127u;
+    const uint64_t pol_st = l2_policy(l2_store);
+    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+    const int64_t n_tiles = (n + kTma4Rows - 1) / kTma4Rows;
+    if (lane == 0)
+        for (int s = 0; s < kStages; s++) mbar_init(&full[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    __syncwarp();
+    const int64_t t0 = blockIdx.x, dt = gridDim.x;
+    auto load_id = [&](int64_t tile) -> int32_t {
+        const int64_t r = tile * kTma4Rows + lane;
+        return (tile < n_tiles && r < n) ? (int32_t)__ldg(ids + r) : -1;
+    };
+    auto issue = [&](int64_t tile, int s, int32_t id) {
+        const int rows = (int)min((int64_t)kTma4Rows, n - tile * kTma4Rows);
+        const int groups = (rows + 3) >> 2;
+        const int32_t first = __shfl_sync(0xffffffffu, id, 0);
+        const int32_t rid = lane < rows ? id : first;
+        const int g = lane & 7;
+        const int32_t r0 = __shfl_sync(0xffffffffu, rid, 4 * g), r1 = __shfl_sync(0xffffffffu, rid, 4 * g + 1);
+        const int32_t r2 = __shfl_sync(0xffffffffu, rid, 4 * g + 2), r3 = __shfl_sync(0xffffffffu, rid, 4 * g + 3);
+        if (lane == 0) mbar_expect_tx(&full[s], (uint32_t)groups * 4u * R);
+        __syncwarp();
+        if (lane < groups)
+            asm volatile(
+                "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes [%0], [%1, {%2, "
+                "%3, %4, %5, %6}], [%7];" ::"r"(smem_u32(stage + ((size_t)s * 8 + lane) * G)),
+                "l"(&tmap), "r"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(&full[s]))
+                : "memory");
+    };
+    int32_t pre[kStages];
+#pragma unroll
+    for (int s = 0; s < kStages; s++) pre[s] = load_id(t0 + s * dt);
+    int64_t next = t0;
+#pragma unroll
+    for (int s = 0; s < kStages; s++, next += dt)
+        if (next < n_tiles) issue(next, s, pre[s]);
+    int32_t next_id = load_id(next);
+    int it = 0;
+    for (int64_t tile = t0; tile < n_tiles; tile += dt, it++) {
+        const int s = it % kStages;
+        mbar_wait(&full[s], (uint32_t)((it / kStages) & 1));
+        const int64_t row0 = tile * kTma4Rows;
+        const int rows = (int)min((int64_t)kTma4Rows, n - row0);
+        const int groups = (rows + 3) >> 2;
+        if (lane < groups) {
+            bulk_store(out + (row0 + 4 * lane) * (int64_t)R, stage + ((size_t)s * 8 + lane) * G,
+                       (uint32_t)min(4, rows - 4 * lane) * R, pol_st);
+        }
+        if (it > 0) bulk_wait_read<1>();  // this lane's store of the previous tile has read its slot
+        __syncwarp();
+        if (it > 0 && next < n_tiles) {
+            issue(next, (it - 1) % kStages, next_id);
+            next += dt;
+            next_id = load_id(next);
+        }
+    }
+    bulk_wait_all();
 }
 
 // Relay service (H7): this rank (server) reads the host rows that `requester` routed through it and
@@ -414,6 +490,34 @@ int grid_for(int64_t work_items, int per_block, int max_blocks) {
     return (int)std::max<int64_t>(1, std::min<int64_t>((work_items + per_block - 1) / per_block, max_blocks));
 }
 
+// Tensor map of the replicated table for tile::gather4: 2-D, 32-bit elements, [n_vertices][R / 4] with the
+// table's row stride, box = one row; built once per table pointer (cuTensorMapEncodeTiled is resolved
+// from the driver at run time, so the library does not link libcuda).
+moment_status encode_table_map(moment_ctx_s* ctx) {
+    using encode_fn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+    static encode_fn encode = nullptr;
+    if (!encode) {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        MOMENT_TRY(cuda_check(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q),
+                              "moment_gather: driver entry point"));
+        if (!fn || q != cudaDriverEntryPointSuccess) return fail(MOMENT_ECUDA, "moment_gather: cuTensorMapEncodeTiled missing");
+        encode = reinterpret_cast<encode_fn>(fn);
+    }
+    const cuuint64_t dims[2] = {(cuuint64_t)(ctx->row_bytes / 4), (cuuint64_t)ctx->n_vertices};
+    const cuuint64_t strides[1] = {(cuuint64_t)ctx->row_stride};
+    const cuuint32_t box[2] = {(cuuint32_t)(ctx->row_bytes / 4), 1};
+    const cuuint32_t estr[2] = {1, 1};
+    const CUresult r = encode(&ctx->tma_map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, ctx->bin_ptr[0], dims, strides, box, estr,
+                              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                              (CUtensorMapL2promotion)ctx->tma_promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return fail(MOMENT_ECUDA, "moment_gather: cuTensorMapEncodeTiled failed (%d)", (int)r);
+    ctx->tma_base = ctx->bin_ptr[0];
+    return MOMENT_OK;
+}
+
 }  // namespace
 
 moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n, void* out,
@@ -428,7 +532,22 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
     if (max_n == 0) return MOMENT_OK;
     bool all_local = true;
     for (int b = 0; b < ctx->n_bins; b++) all_local &= ctx->bin_owner[b] == ctx->rank;
+    // auto: tile::gather4 for a replicated table whose row fits one box (<= 256 words), TMA bulk copies for
+    // other local rows, LDG.128 for routed / remote rows
+    const bool tma4_ok = route == nullptr && ctx->n_bins == 1 && !ctx->placement && all_local && ctx->row_bytes / 4 <= 256;
+    const bool tma4 = tma4_ok && (ctx->gather_path == 3 || ctx->gather_path == 0);
     const bool bulk = ctx->gather_path == 2 || (ctx->gather_path == 0 && route == nullptr && all_local);
+    if (tma4) {
+        if (ctx->tma_base != ctx->bin_ptr[0]) MOMENT_TRY(encode_table_map(ctx));
+        const uint32_t G = (uint32_t)((4 * ctx->row_bytes + 127) & ~int64_t(127));
+        const int stages = 4, bps = ctx->tma4_blocks_per_sm;
+        const size_t smem = (size_t)stages * 8 * G;
+        const int64_t tiles = (max_n + kTma4Rows - 1) / kTma4Rows;
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)148 * bps));
+        gather_tma4_kernel<4><<<grid, 32, smem, stream>>>(ctx->tma_map, ids, n_dev, max_n, (uint32_t)ctx->row_bytes,
+                                                          ctx->l2_store_policy, reinterpret_cast<char*>(out));
+        return cuda_check(cudaGetLastError(), "moment_gather: tma4 launch");
+    }
     if (bulk && route == nullptr) {
         // tiles of <= 32 rows, `stages` tiles in flight per 1-warp block, `bps` blocks per SM, each stage at
         // most `stage_kb` KB (defaults 4 / 4 / 14: 4 x 4 x 14 KB fits the SM's shared memory)
@@ -739,7 +858,8 @@ moment_status configure_gather_kernels(int carveout) {
             MOMENT_TRY(cuda_check(cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, carveout),
                                   "carveout attribute"));
     for (const void* f : {(const void*)gather_bulk_kernel<2>, (const void*)gather_bulk_kernel<4>,
-                          (const void*)gather_bulk_kernel<6>, (const void*)gather_bulk_kernel<8>})
+                          (const void*)gather_bulk_kernel<6>, (const void*)gather_bulk_kernel<8>,
+                          (const void*)gather_tma4_kernel<4>})
         MOMENT_TRY(cuda_check(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmemMax),
                               "bulk gather smem attribute"));
     return MOMENT_OK;

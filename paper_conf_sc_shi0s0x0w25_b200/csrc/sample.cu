@@ -172,8 +172,8 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_kern
             lo[q] = 0;
             d[q] = 0;
             if (v[q] >= 0) {
-                lo[q] = __ldg(a.indptr + v[q]);
-                d[q] = (int32_t)(__ldg(a.indptr + v[q] + 1) - lo[q]);
+                lo[q] = dev::ld_rand(a.indptr + v[q]);
+                d[q] = (int32_t)(dev::ld_rand(a.indptr + v[q] + 1) - lo[q]);
             }
         }
 #pragma unroll
@@ -207,7 +207,7 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_kern
             }
         }
 #pragma unroll
-        for (int q = 0; q < Q; q++) u[q] = pos[q] >= 0 ? __ldg(a.indices + lo[q] + pos[q]) : 0;
+        for (int q = 0; q < Q; q++) u[q] = pos[q] >= 0 ? dev::ld_rand(a.indices + lo[q] + pos[q]) : 0;
 #pragma unroll
         for (int q = 0; q < Q; q++) {
             const int64_t idx = base + q;
@@ -263,8 +263,8 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp
             lo[q] = 0;
             d[q] = 0;
             if (v[q] >= 0) {
-                lo[q] = __ldg(a.indptr + v[q]);
-                d[q] = (int32_t)(__ldg(a.indptr + v[q] + 1) - lo[q]);
+                lo[q] = dev::ld_rand(a.indptr + v[q]);
+                d[q] = (int32_t)(dev::ld_rand(a.indptr + v[q] + 1) - lo[q]);
             }
         }
 #pragma unroll
@@ -302,7 +302,7 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp
             }
         }
 #pragma unroll
-        for (int q = 0; q < Q; q++) u[q] = pos[q] >= 0 ? __ldg(a.indices + lo[q] + pos[q]) : 0;
+        for (int q = 0; q < Q; q++) u[q] = pos[q] >= 0 ? dev::ld_rand(a.indices + lo[q] + pos[q]) : 0;
 #pragma unroll
         for (int q = 0; q < Q; q++) {
             if (!live || idx[q] >= F) continue;
@@ -469,7 +469,7 @@ __global__ void __launch_bounds__(kSampleTile, MOMENT_SAMPLE_MIN_BLOCKS) compact
 #pragma unroll
                 for (int r = 0; r < 16; r++) id[r] = r0 + r < c ? __ldg(p + r0 + r) : 0;
 #pragma unroll
-                for (int r = 0; r < 16; r++) li[r] = r0 + r < c ? __ldg(a.lidx + id[r]) : 0;
+                for (int r = 0; r < 16; r++) li[r] = r0 + r < c ? dev::ld_rand(a.lidx + id[r]) : 0;
 #pragma unroll
                 for (int r = 0; r < 16; r++)
                     if (r0 + r < c) a.src[gpos + r0 + r] = li[r];

@@ -145,7 +145,7 @@ def test_sample_reused_ctx_many_batches(orc, c1):
         assert_same_sample(got, want)
 
 
-@pytest.mark.parametrize("path", ["auto", "ldg", "bulk"])
+@pytest.mark.parametrize("path", ["auto", "ldg", "bulk", "tma4"])
 @pytest.mark.parametrize("dim,dtype", [(4, torch.float32), (12, torch.float32), (100, torch.float32),
                                        (128, torch.float32), (768, torch.float16), (1024, torch.float32)])
 def test_gather_replicated(orc, dim, dtype, path, monkeypatch):
