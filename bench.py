@@ -112,7 +112,8 @@ class State:
                         counts_host, stream=L.stream)
 
     def launches_per_step(self):
-        return 1 + 1 + 2 * len(self.fanout) + 1 + 1  # set_call, init, (sample, bitscan) per hop, compact, gather
+        # set_call, (sample, bitscan) per hop (the first hop's sampler also initialises the call), compact, gather
+        return 1 + 2 * len(self.fanout) + 1 + 1
 
 
 def build_state(name, device="cuda:0", rank=0, world=1, inflight=1):

@@ -106,6 +106,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     if (const char* v = std::getenv("MOMENT_HOP_Q")) c->hop_nodes_per_group = std::max(1, std::atoi(v));
     if (const char* v = std::getenv("MOMENT_HOP_WARP")) c->hop_warp_segmented = std::atoi(v) != 0;
     if (const char* v = std::getenv("MOMENT_STEP_FORK")) c->step_fork = std::atoi(v) != 0;
+    if (const char* v = std::getenv("MOMENT_INIT_KERNEL")) c->init_in_hop0 = std::atoi(v) == 0;
     if (const char* v = std::getenv("MOMENT_COMPACT_GRID")) c->compact_grid_per_sm = std::max(1, std::atoi(v));
     if (const char* l2 = std::getenv("MOMENT_GATHER_L2")) {  // "<load><store>" digits, e.g. "01"
         if (std::strlen(l2) == 2) {

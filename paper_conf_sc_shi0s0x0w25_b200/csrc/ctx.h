@@ -32,6 +32,7 @@ struct moment_ctx_s {
     int32_t hop_grid_per_sm = 4, compact_grid_per_sm = 1;  // launch caps (MOMENT_HOP_GRID / MOMENT_COMPACT_GRID)
     int32_t hop_nodes_per_group = 4;  // nodes per lane group on large frontiers (MOMENT_HOP_Q: 1, 2, 4, 8)
     int32_t hop_warp_segmented = 1;   // k <= 32: k-lane groups packed in a warp (MOMENT_HOP_WARP=0: 2^n tiles)
+    int32_t init_in_hop0 = 1;         // the first hop's sampler also initialises the call (MOMENT_INIT_KERNEL=1: separate)
     int32_t bulk_stages = 4, bulk_blocks_per_sm = 4, bulk_stage_kb = 14;  // bulk gather shape (MOMENT_BULK="S,B,KB")
     std::vector<int32_t> bin_owner;
     std::vector<void*> bin_ptr;

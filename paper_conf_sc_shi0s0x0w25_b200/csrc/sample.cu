@@ -49,6 +49,25 @@ struct HopArgs {
     int32_t grid_per_sm;   // launch cap: blocks per SM (grid-stride beyond it)
 };
 
+// The per-call initialisation that the first hop's sampler does itself (hop_sample_warp_kernel<Q, true>):
+// F_0 = seeds (read from the call block), their lidx / visited entries, the seed checks, and zeroed tile
+// descriptors, tickets and hop bases for the scans that follow.
+struct InitArgs {
+    int64_t n_seeds, n_vertices;
+    int64_t* nodes;
+    int64_t* counts;
+    int32_t* lidx;
+    uint32_t* visited;
+    uint32_t* error_flag;
+    int32_t check;
+    uint64_t* tile_status;
+    int64_t n_tile_status;
+    uint32_t* tickets;
+    int32_t n_tickets;
+    uint64_t* ebase;
+    int32_t n_ebase;
+};
+
 // Fire-and-forget: the result is unused, so this is a RED.OR the issuing warp never waits on.
 __device__ __forceinline__ void mark_new(uint32_t* newbits, int32_t u) {
     atomicOr(newbits + (u >> 5), 1u << (u & 31));
@@ -235,11 +254,19 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_kern
 // group's bit offset), so groups never diverge and no convergence barriers are needed. Step q of a warp
 // handles the NG consecutive frontier nodes base + q * NG + g: its pad stores are one run of NG * k ints.
 // Same choices as floyd_choice (same draws, same resolution rule), only the lane layout differs.
-template <int Q>
-__global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp_kernel(HopArgs a) {
+template <int Q, bool kInit>
+__global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp_kernel(HopArgs a, InitArgs in) {
     constexpr unsigned kFull = 0xffffffffu;
-    const int64_t F = a.counts[a.h];
+    const int64_t F = kInit ? in.n_seeds : a.counts[a.h];
     const uint64_t seed = a.call[0];
+    const int64_t* seeds = kInit ? reinterpret_cast<const int64_t*>(a.call[1]) : nullptr;
+    if (kInit) {
+        const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (int64_t)gridDim.x * blockDim.x;
+        for (int64_t j = tid; j < in.n_tile_status; j += nth) in.tile_status[j] = 0;
+        for (int64_t j = tid; j < in.n_tickets; j += nth) in.tickets[j] = 0;
+        for (int64_t j = tid; j < in.n_ebase; j += nth) in.ebase[j] = 0;
+        if (tid == 0) in.counts[0] = in.n_seeds;
+    }
     const int k = a.k;
     const int lane = threadIdx.x & 31;
     const int NG = 32 / k;
@@ -256,7 +283,27 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp
 #pragma unroll
         for (int q = 0; q < Q; q++) {
             idx[q] = base + (int64_t)q * NG + g;
-            v[q] = (live && idx[q] < F) ? a.nodes[idx[q]] : -1;
+            if (kInit) {  // F_0 = seeds; an out-of-range seed is flagged and replaced by vertex 0 (never written)
+                v[q] = -1;
+                if (live && idx[q] < F) {
+                    const int64_t sv = seeds[idx[q]];
+                    const bool bad = sv < 0 || sv >= in.n_vertices;
+                    v[q] = bad ? 0 : sv;
+                    if (i == 0) {
+                        in.nodes[idx[q]] = v[q];
+                        if (bad) {
+                            atomicOr(in.error_flag, 1u);
+                        } else {
+                            in.lidx[sv] = (int32_t)idx[q];
+                            const uint32_t bit = 1u << (sv & 31);
+                            const uint32_t old = atomicOr(in.visited + (sv >> 5), bit);
+                            if (in.check && (old & bit)) atomicOr(in.error_flag, 2u);
+                        }
+                    }
+                }
+            } else {
+                v[q] = (live && idx[q] < F) ? a.nodes[idx[q]] : -1;
+            }
         }
 #pragma unroll
         for (int q = 0; q < Q; q++) {
@@ -523,12 +570,13 @@ void launch_sample_hop(const HopArgs& a, int64_t max_F, int big_q, cudaStream_t 
     else launch_sample_hop_q<G, 8>(a, max_F, stream);
 }
 
-template <int Q>
-void launch_sample_warp_q(const HopArgs& a, int64_t max_F, cudaStream_t stream) {
+template <int Q, bool kInit = false>
+void launch_sample_warp_q(const HopArgs& a, int64_t max_F, cudaStream_t stream, const InitArgs& in = InitArgs{}) {
     const int64_t per_warp = (int64_t)(32 / a.k) * Q;
     const int64_t warps = (max_F + per_warp - 1) / per_warp;
     const int64_t blocks = std::max<int64_t>(1, (warps + 7) / 8);
-    hop_sample_warp_kernel<Q><<<(int)std::min<int64_t>(blocks, (int64_t)148 * a.grid_per_sm), 256, 0, stream>>>(a);
+    hop_sample_warp_kernel<Q, kInit>
+        <<<(int)std::min<int64_t>(blocks, (int64_t)148 * a.grid_per_sm), 256, 0, stream>>>(a, in);
 }
 
 void launch_sample_warp(const HopArgs& a, int64_t max_F, int big_q, cudaStream_t stream) {
@@ -551,8 +599,8 @@ moment_status configure_sample_kernels(int carveout) {
                          (const void*)hop_sample_kernel<16, 4>, (const void*)hop_sample_kernel<32, 4>,
                          (const void*)hop_sample_kernel<4, 8>, (const void*)hop_sample_kernel<8, 8>,
                          (const void*)hop_sample_kernel<16, 8>, (const void*)hop_sample_kernel<32, 8>,
-                         (const void*)hop_sample_warp_kernel<1>, (const void*)hop_sample_warp_kernel<2>,
-                         (const void*)hop_sample_warp_kernel<4>};
+                         (const void*)hop_sample_warp_kernel<1, false>, (const void*)hop_sample_warp_kernel<2, false>,
+                         (const void*)hop_sample_warp_kernel<4, false>, (const void*)hop_sample_warp_kernel<1, true>};
     for (const void* f : fns)
         MOMENT_TRY(cuda_check(cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, carveout),
                               "carveout attribute"));
@@ -595,7 +643,12 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
     const int H = p->n_hops;
     const int check = (p->flags & MOMENT_SAMPLE_CHECK) ? 1 : 0;
     const int replace = (p->flags & MOMENT_SAMPLE_REPLACE) ? 1 : 0;
-    {
+    // the first hop initialises the call itself when it runs the warp-segmented sampler (one launch fewer)
+    const bool init_in_hop0 = H > 0 && ctx->hop_warp_segmented && p->fanout[0] <= 32 && ctx->init_in_hop0;
+    const InitArgs init{n_seeds, ctx->n_vertices, out->nodes, out->counts, ctx->lidx, ctx->visited, ctx->error_flag,
+                        check, ctx->tile_status, ctx->n_tile_status, ctx->tickets, 1 + std::max(1, ctx->max_hops),
+                        ctx->ebase, std::max(1, ctx->max_hops)};
+    if (!init_in_hop0) {
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n_seeds + 255) / 256, 148 * 4));
         init_kernel<<<grid, 256, 0, stream>>>(call, n_seeds, ctx->n_vertices, out->nodes, ctx->lidx, ctx->visited,
                                               out->counts, ctx->error_flag, check, ctx->tile_status, ctx->n_tile_status,
@@ -611,7 +664,8 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         HopArgs a{csr->indptr, csr->indices, out->nodes, out->counts, ctx->pad + pad_off, ctx->cnt + cnt_off,
                   ctx->newbits, call, h, k, replace, ctx->hop_grid_per_sm};
         const int q = ctx->hop_nodes_per_group;
-        if (ctx->hop_warp_segmented && k <= 32) launch_sample_warp(a, F_bound, q, stream);
+        if (h == 0 && init_in_hop0) launch_sample_warp_q<1, true>(a, F_bound, stream, init);
+        else if (ctx->hop_warp_segmented && k <= 32) launch_sample_warp(a, F_bound, q, stream);
         else if (k <= 4) launch_sample_hop<4>(a, F_bound, q, stream);
         else if (k <= 8) launch_sample_hop<8>(a, F_bound, q, stream);
         else if (k <= 16) launch_sample_hop<16>(a, F_bound, q, stream);

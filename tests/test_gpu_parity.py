@@ -68,13 +68,14 @@ def test_sample_fanouts_and_ragged(orc, c1, fanout, n_seeds):
     assert_same_sample(got, want)
 
 
-@pytest.mark.parametrize("knob", ["MOMENT_HOP_WARP"])
+@pytest.mark.parametrize("knob", [("MOMENT_HOP_WARP", "0"), ("MOMENT_INIT_KERNEL", "1")])
 @pytest.mark.parametrize("fanout", [[15, 10, 5], [7, 3], [20]])
 def test_sample_kernel_variants(orc, c1, fanout, knob, monkeypatch):
-    """The other sampler kernel gives the same result as the default: MOMENT_HOP_WARP=0 selects the
-    power-of-two lane tiles (always used for k > 32)."""
+    """The other sampler kernels give the same result as the default: MOMENT_HOP_WARP=0 selects the
+    power-of-two lane tiles (always used for k > 32), MOMENT_INIT_KERNEL=1 a separate init kernel instead of
+    the first hop's sampler initialising the call."""
     _, g = c1
-    monkeypatch.setenv(knob, "0")
+    monkeypatch.setenv(*knob)
     seeds = np.random.default_rng(5).choice(g.n, 1000, replace=False)
     got, want = sample_both(orc, g, seeds, fanout, 4242)
     assert_same_sample(got, want)
