@@ -149,6 +149,9 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     }
     c->n_tile_status = std::max<int64_t>(nts, 1);
     const int64_t o_tiles = cv.take<uint64_t>(c->n_tile_status);
+    c->n_tile_edges = 0;
+    for (int h = 0; h < a->max_hops; h++) c->n_tile_edges += (c->max_F[h] + kSampleTile - 1) / kSampleTile;
+    const int64_t o_tile_edges = cv.take<unsigned long long>(std::max<int64_t>(c->n_tile_edges, 1));
     const int64_t o_tickets = cv.take<uint32_t>(1 + std::max(1, a->max_hops));
     const int64_t o_ebase = cv.take<uint64_t>(std::max(1, a->max_hops));
     const int64_t o_pad = cv.take<int32_t>(c->max_edges);
@@ -179,6 +182,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     c->newbits = reinterpret_cast<uint32_t*>(w + o_newbits);
     c->visited = reinterpret_cast<uint32_t*>(w + o_visited);
     c->tile_status = reinterpret_cast<uint64_t*>(w + o_tiles);
+    c->tile_edges = reinterpret_cast<unsigned long long*>(w + o_tile_edges);
     c->tickets = reinterpret_cast<uint32_t*>(w + o_tickets);
     c->ebase = reinterpret_cast<uint64_t*>(w + o_ebase);
     c->pad = reinterpret_cast<int32_t*>(w + o_pad);
@@ -257,16 +261,22 @@ extern "C" moment_status moment_ctx_workspace_bytes(moment_ctx_t ctx, int64_t* b
 
 namespace {
 
-__global__ void set_call_kernel(uint64_t* call, uint64_t rng_seed, const int64_t* seeds) {
-    call[0] = rng_seed;
-    call[1] = reinterpret_cast<uint64_t>(seeds);
+__global__ void set_call_kernel(uint64_t* call, uint64_t rng_seed, const int64_t* seeds, unsigned long long* zero,
+                                int64_t n_zero) {
+    if (threadIdx.x == 0) {
+        call[0] = rng_seed;
+        call[1] = reinterpret_cast<uint64_t>(seeds);
+    }
+    for (int64_t j = threadIdx.x; j < n_zero; j += blockDim.x) zero[j] = 0;  // hop 0's compaction tile sums
 }
 
-// Stage the per-call arguments (rng_seed, seeds pointer) into the device call block with a one-thread
+// Stage the per-call arguments (rng_seed, seeds pointer) into the device call block with a one-warp
 // kernel whose parameters carry the values: ordered before the call's kernels on `s`, and safe inside a
-// caller's stream capture (the values are baked into the captured node).
-moment_status write_call(moment_ctx_s* c, uint64_t rng_seed, const int64_t* seeds, cudaStream_t s) {
-    set_call_kernel<<<1, 1, 0, s>>>(c->d_call, rng_seed, seeds);
+// caller's stream capture (the values are baked into the captured node). It also zeroes the first hop's
+// compaction tile sums (the later hops' are zeroed by the scan before them).
+moment_status write_call(moment_ctx_s* c, uint64_t rng_seed, const int64_t* seeds, int64_t n_seeds, cudaStream_t s) {
+    set_call_kernel<<<1, 32, 0, s>>>(c->d_call, rng_seed, seeds, c->tile_edges,
+                                     std::min<int64_t>((n_seeds + kSampleTile - 1) / kSampleTile, c->n_tile_edges));
     return cuda_check(cudaGetLastError(), "call block");
 }
 
@@ -349,7 +359,7 @@ extern "C" moment_status moment_sample(moment_ctx_t ctx, const moment_csr* csr, 
     MOMENT_TRY(check_ctx(ctx, "moment_sample"));
     MOMENT_TRY(check_sample(ctx, csr, seeds, n_seeds, params, out));
     cudaStream_t s = static_cast<cudaStream_t>(stream);
-    MOMENT_TRY(write_call(ctx, params->rng_seed, seeds, s));
+    MOMENT_TRY(write_call(ctx, params->rng_seed, seeds, n_seeds, s));
     return launch_sample(ctx, csr, ctx->d_call, n_seeds, params, out, s);
 }
 
@@ -360,7 +370,7 @@ extern "C" moment_status moment_step(moment_ctx_t ctx, const moment_csr* csr, co
     MOMENT_TRY(check_sample(ctx, csr, seeds, n_seeds, params, out));
     MOMENT_TRY(check_rows(ctx, d_rows, out));
     cudaStream_t s = static_cast<cudaStream_t>(stream);
-    MOMENT_TRY(write_call(ctx, params->rng_seed, seeds, s));
+    MOMENT_TRY(write_call(ctx, params->rng_seed, seeds, n_seeds, s));
     return run_step(ctx, csr, n_seeds, params, out, d_rows, s);
 }
 
@@ -439,7 +449,7 @@ extern "C" moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* cs
     MOMENT_TRY(check_rows(ctx, d_rows, out));
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     MOMENT_TRY(cuda_check(cudaMemcpyAsync(ctx->d_seed_stage, seeds_host, n_seeds * sizeof(int64_t), cudaMemcpyHostToDevice, s), "moment_step_host: H2D"));
-    MOMENT_TRY(write_call(ctx, params->rng_seed, ctx->d_seed_stage, s));
+    MOMENT_TRY(write_call(ctx, params->rng_seed, ctx->d_seed_stage, n_seeds, s));
     MOMENT_TRY(run_step(ctx, csr, n_seeds, params, out, d_rows, s));
     const int H = params->n_hops;
     return cuda_check(cudaMemcpyAsync(counts_host, out->counts, (2 * H + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s),

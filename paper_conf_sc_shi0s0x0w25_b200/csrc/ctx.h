@@ -46,6 +46,8 @@ struct moment_ctx_s {
     uint32_t* newbits = nullptr;    // [n_words]: ids emitted at the current hop
     uint32_t* visited = nullptr;    // [n_words]: F_h membership
     int64_t n_words = 0;
+    unsigned long long* tile_edges = nullptr;  // edges per compaction tile of every hop (bound-numbered)
+    int64_t n_tile_edges = 0;
     uint64_t* tile_status = nullptr;  // decoupled look-back descriptors: compact chain, then bitscan per hop
     int64_t n_tile_status = 0;
     std::vector<int64_t> bitscan_tiles_off;  // per hop offsets into tile_status

@@ -47,6 +47,9 @@ struct HopArgs {
     int32_t h, k;
     int32_t replace;
     int32_t grid_per_sm;   // launch cap: blocks per SM (grid-stride beyond it)
+    // this hop's edges per compaction tile (kSampleTile consecutive nodes), summed here so that the
+    // compaction needs no chained scan; zeroed before the hop (hop 0: set_call, hop h: bitscan h - 1)
+    unsigned long long* tile_edges;
 };
 
 // The per-call initialisation that the first hop's sampler does itself (hop_sample_warp_kernel<Q, true>):
@@ -231,7 +234,11 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_kern
         for (int q = 0; q < Q; q++) {
             const int64_t idx = base + q;
             if (idx >= F) break;
-            if (lane == 0) a.cnt[idx] = a.replace ? (d[q] > 0 ? k : 0) : min(d[q], k);
+            if (lane == 0) {
+                const int32_t c = a.replace ? (d[q] > 0 ? k : 0) : min(d[q], k);
+                a.cnt[idx] = c;
+                if (c) atomicAdd(a.tile_edges + idx / kSampleTile, (unsigned long long)c);
+            }
             if (pos[q] >= 0) {
                 a.pad[idx * k + rnk[q]] = u[q];
                 mark_new(a.newbits, u[q]);
@@ -352,12 +359,18 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp
         for (int q = 0; q < Q; q++) u[q] = pos[q] >= 0 ? dev::ld_rand(a.indices + lo[q] + pos[q]) : 0;
 #pragma unroll
         for (int q = 0; q < Q; q++) {
-            if (!live || idx[q] >= F) continue;
-            if (i == 0) a.cnt[idx[q]] = a.replace ? (d[q] > 0 ? k : 0) : min(d[q], k);
-            if (pos[q] >= 0) {
+            const bool node = live && idx[q] < F;
+            const uint32_t c = node ? (uint32_t)(a.replace ? (d[q] > 0 ? k : 0) : min(d[q], k)) : 0u;
+            if (node && i == 0) a.cnt[idx[q]] = (int32_t)c;
+            if (node && pos[q] >= 0) {
                 a.pad[idx[q] * k + rnk[q]] = u[q];
                 mark_new(a.newbits, u[q]);
             }
+            // the step's NG nodes span at most two compaction tiles: one RED per tile and warp
+            const int64_t tile = idx[q] / kSampleTile;
+            const unsigned peers = __match_any_sync(kFull, (unsigned long long)tile);
+            const uint32_t sum = __reduce_add_sync(peers, i == 0 ? c : 0u);
+            if (lane == __ffs(peers) - 1 && sum) atomicAdd(a.tile_edges + tile, (unsigned long long)sum);
         }
     }
 }
@@ -372,6 +385,8 @@ struct ScanArgs {
     uint32_t* ticket;
     int64_t n_words;
     int32_t h;
+    unsigned long long* zero;  // the next hop's compaction tile sums, zeroed here (before that hop runs)
+    int64_t n_zero;
 };
 
 // F_{h+1} = F_h ++ ascending ids set in (newbits & ~visited).
@@ -381,6 +396,8 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
     __shared__ int s_nearest;
     const int64_t F = a.counts[a.h];
     const int64_t n_tiles = (a.n_words + kScanTileWords - 1) / kScanTileWords;
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < a.n_zero; j += (int64_t)gridDim.x * blockDim.x)
+        a.zero[j] = 0;
     for (;;) {
         if (threadIdx.x == 0) s_tile = atomicAdd(a.ticket, 1u);
         __syncthreads();
@@ -439,24 +456,39 @@ struct CompactArgs {
     const int64_t* nodes;
     const int32_t* lidx;
     uint32_t* visited;
-    uint64_t* tile_status;  // one chain over the tiles of all hops
-    uint64_t* ebase;        // [H]: global edge position of hop h's first edge, kBaseReady-flagged
-    uint32_t* ticket;
+    const unsigned long long* tile_edges;  // edges per tile, tiles of all hops numbered by the bounds tb[]
     int32_t H;
+    int64_t tb[kMaxHops + 1];  // first tile of hop h (sum of ceil(F_bound_h' / kSampleTile), h' < h)
     int32_t k[kMaxHops];
     const int32_t* pad[kMaxHops];
     const int32_t* cnt[kMaxHops];
 };
 
+// Block sum of two int64 per thread (every thread gets both sums).
+__device__ __forceinline__ void block_sum2(int64_t& x, int64_t& y, int64_t (*red)[2]) {
+    for (int d = 16; d > 0; d >>= 1) {
+        x += __shfl_xor_sync(0xffffffffu, x, d);
+        y += __shfl_xor_sync(0xffffffffu, y, d);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        red[threadIdx.x >> 5][0] = x;
+        red[threadIdx.x >> 5][1] = y;
+    }
+    __syncthreads();
+    x = y = 0;
+    for (int w = 0; w < kSampleTile / 32; w++) {
+        x += red[w][0];
+        y += red[w][1];
+    }
+}
+
+// All hops' offsets and src in one wait-free pass: a tile's first edge position is the sum of the edge
+// counts of the tiles before it, which the hop kernels accumulated per tile (no chained scan, no waiting
+// on other blocks); the hop's base is the sum over the earlier hops' tiles.
 __global__ void __launch_bounds__(kSampleTile, MOMENT_SAMPLE_MIN_BLOCKS) compact_kernel(CompactArgs a) {
     __shared__ int64_t s_red[kSampleTile / 32];
-    __shared__ uint32_t s_tile;
-    __shared__ int s_nearest;
-    __shared__ int64_t s_base;
-    int64_t tiles_before[kMaxHops + 1];
-    tiles_before[0] = 0;
-    for (int h = 0; h < a.H; h++) tiles_before[h + 1] = tiles_before[h] + (a.counts[h] + kSampleTile - 1) / kSampleTile;
-    const int64_t n_tiles = tiles_before[a.H];
+    __shared__ int64_t s_red2[kSampleTile / 32][2];
+    const int64_t n_tiles = a.tb[a.H];
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         // hops with an empty frontier have no tile: write their (empty) offsets and E_h here
         int64_t ob = 0;
@@ -468,39 +500,27 @@ __global__ void __launch_bounds__(kSampleTile, MOMENT_SAMPLE_MIN_BLOCKS) compact
             ob += a.counts[h] + 1;
         }
     }
-    for (;;) {
-        if (threadIdx.x == 0) s_tile = atomicAdd(a.ticket, 1u);
-        __syncthreads();
-        const int64_t tile = s_tile;
-        if (tile >= n_tiles) break;
+    for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         int h = 0;
-        while (tile >= tiles_before[h + 1]) h++;
+        while (tile >= a.tb[h + 1]) h++;
         const int64_t F = a.counts[h];
+        const int64_t lt = tile - a.tb[h];
+        if (lt * kSampleTile >= F) continue;  // past this hop's frontier (uniform per block)
         int64_t ob = 0;
         for (int q = 0; q < h; q++) ob += a.counts[q] + 1;
-        const int64_t lt = tile - tiles_before[h];
         const int64_t idx = lt * kSampleTile + threadIdx.x;
         const int32_t c = idx < F ? a.cnt[h][idx] : 0;
+        int64_t before_hop = 0, in_hop = 0;  // edges of the earlier hops' tiles / of this hop's earlier tiles
+        for (int64_t j = threadIdx.x; j < tile; j += kSampleTile) {
+            const int64_t e = (int64_t)__ldcg(a.tile_edges + j);
+            if (j < a.tb[h]) before_hop += e;
+            else in_hop += e;
+        }
+        block_sum2(before_hop, in_hop, s_red2);
         int64_t agg;
         const int64_t excl = dev::block_exclusive_scan<kSampleTile>(c, &agg, s_red);
-        const int64_t prefix = dev::lookback_block<kSampleTile>(a.tile_status, tile, agg, s_red, &s_nearest);
-        if (threadIdx.x == 0) {
-            if (lt == 0) {
-                dev::st_flag(&a.ebase[h], kBaseReady | (uint64_t)prefix);
-                s_base = prefix;
-            } else {
-                uint64_t b;
-                b = dev::ld_flag(&a.ebase[h]);
-                while (!(b & kBaseReady)) {
-                    __nanosleep(64);
-                    b = dev::ld_flag(&a.ebase[h]);
-                }
-                s_base = (int64_t)(b & ~kBaseReady);
-            }
-        }
-        __syncthreads();
-        const int64_t gpos = prefix + excl;  // global position of this node's first edge
-        const int64_t rel = gpos - s_base;
+        const int64_t gpos = before_hop + in_hop + excl;  // global position of this node's first edge
+        const int64_t rel = in_hop + excl;
         if (idx < F) {
             a.offsets[ob + idx] = rel;
             if (idx == F - 1) {
@@ -522,7 +542,7 @@ __global__ void __launch_bounds__(kSampleTile, MOMENT_SAMPLE_MIN_BLOCKS) compact
                     if (r0 + r < c) a.src[gpos + r0 + r] = li[r];
             }
         }
-        __syncthreads();
+        __syncthreads();  // s_red / s_red2 are reused by the next tile
     }
     const int64_t FH = a.counts[a.H];
     for (int64_t i = (int64_t)blockIdx.x * kSampleTile + threadIdx.x; i < FH; i += (int64_t)gridDim.x * kSampleTile)
@@ -655,14 +675,23 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
                                               ctx->tickets, 1 + std::max(1, ctx->max_hops), ctx->ebase,
                                               std::max(1, ctx->max_hops));
     }
-    // per-call bounds on |F_h| for launch sizing and padded-buffer carving (true sizes live in counts)
+    // per-call bounds on |F_h| for launch sizing, padded-buffer carving and compaction tile numbering (the
+    // true sizes live in counts); hop h's tile sums are tile_edges[tb[h] .. tb[h + 1])
     CompactArgs ca{};
-    int64_t F_bound = n_seeds, pad_off = 0, cnt_off = 0, comp_tiles = 0;
+    {
+        int64_t Fb = n_seeds;
+        ca.tb[0] = 0;
+        for (int h = 0; h < H; h++) {
+            ca.tb[h + 1] = ca.tb[h] + (Fb + kSampleTile - 1) / kSampleTile;
+            Fb = std::min(Fb + Fb * (int64_t)p->fanout[h], ctx->n_vertices);
+        }
+    }
+    int64_t F_bound = n_seeds, pad_off = 0, cnt_off = 0;
     const int64_t n_scan_tiles = (ctx->n_words + kScanTileWords - 1) / kScanTileWords;
     for (int h = 0; h < H; h++) {
         const int k = p->fanout[h];
         HopArgs a{csr->indptr, csr->indices, out->nodes, out->counts, ctx->pad + pad_off, ctx->cnt + cnt_off,
-                  ctx->newbits, call, h, k, replace, ctx->hop_grid_per_sm};
+                  ctx->newbits, call, h, k, replace, ctx->hop_grid_per_sm, ctx->tile_edges + ca.tb[h]};
         const int q = ctx->hop_nodes_per_group;
         if (h == 0 && init_in_hop0) launch_sample_warp_q<1, true>(a, F_bound, stream, init);
         else if (ctx->hop_warp_segmented && k <= 32) launch_sample_warp(a, F_bound, q, stream);
@@ -670,15 +699,16 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         else if (k <= 8) launch_sample_hop<8>(a, F_bound, q, stream);
         else if (k <= 16) launch_sample_hop<16>(a, F_bound, q, stream);
         else launch_sample_hop<32>(a, F_bound, q, stream);
+        const int64_t n_zero = h + 1 < H ? ca.tb[h + 2] - ca.tb[h + 1] : 0;  // the next hop's tile sums
         ScanArgs s{out->nodes, out->counts, ctx->lidx, ctx->newbits, ctx->visited,
-                   ctx->tile_status + ctx->bitscan_tiles_off[h], ctx->tickets + 1 + h, ctx->n_words, h};
+                   ctx->tile_status + ctx->bitscan_tiles_off[h], ctx->tickets + 1 + h, ctx->n_words, h,
+                   ctx->tile_edges + ca.tb[h + 1], n_zero};
         bitscan_kernel<<<(int)std::min<int64_t>(n_scan_tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
         ca.k[h] = k;
         ca.pad[h] = ctx->pad + pad_off;
         ca.cnt[h] = ctx->cnt + cnt_off;
         pad_off += F_bound * k;
         cnt_off += F_bound;
-        comp_tiles += (F_bound + kSampleTile - 1) / kSampleTile;
         F_bound = std::min(F_bound + F_bound * (int64_t)k, ctx->n_vertices);
     }
     if (after_hops) MOMENT_TRY(cuda_check(cudaEventRecord(after_hops, stream), "moment_sample: fork event"));
@@ -688,12 +718,10 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
     ca.nodes = out->nodes;
     ca.lidx = ctx->lidx;
     ca.visited = ctx->visited;
-    ca.tile_status = ctx->tile_status;  // the compact chain occupies the first entries
-    ca.ebase = ctx->ebase;
-    ca.ticket = ctx->tickets;
+    ca.tile_edges = ctx->tile_edges;
     ca.H = H;
     const int grid = (int)std::max<int64_t>(
-        1, std::min<int64_t>(std::max(comp_tiles, (F_bound + 1023) / 1024), (int64_t)148 * ctx->compact_grid_per_sm));
+        1, std::min<int64_t>(std::max(ca.tb[H], (F_bound + 1023) / 1024), (int64_t)148 * ctx->compact_grid_per_sm));
     compact_kernel<<<grid, kSampleTile, 0, stream>>>(ca);
     return cuda_check(cudaGetLastError(), "moment_sample: launch");
 }
