@@ -1,17 +1,19 @@
 // sample.cu — H1-H3: multi-hop neighbour sampling with dedup/relabel on sm_100a (R3-R6).
 //
-// One sample call is 2H + 2 kernels and no memsets. No kernel needs the host to know |F_h| or E_h (every
-// size is read from device memory), so the call is CUDA-graph capturable. The critical path per hop is
-// two kernels; offsets, compaction and relabelling of every hop happen once, after the last hop:
-//   init        : F_0 = seeds; lidx / visited of the seeds; zero the tile descriptors and tickets.
-//   sample (h)  : one G-lane group per frontier node v draws min(deg v, k) Floyd (or with-replacement)
+// One sample call is 2H + 1 kernels (2H + 2 with a separate init) and no memsets. No kernel needs the host
+// to know |F_h| or E_h (every size is read from device memory), so the call is CUDA-graph capturable. The
+// critical path per hop is two kernels; offsets, compaction and relabelling of every hop happen once:
+//   init        : F_0 = seeds; lidx / visited of the seeds; zero the tile descriptors and tickets (done by
+//                 the first hop's sampler, or a separate kernel).
+//   sample (h)  : one k-lane group per frontier node v draws min(deg v, k) Floyd (or with-replacement)
 //                 positions from Philox (choices resolved in parallel), writes the neighbour ids to the
-//                 node's k-slot row of a padded buffer, its count to cnt_h, and marks them in `newbits`.
+//                 node's k-slot row of a padded buffer, its count to cnt_h, adds it to its compaction
+//                 tile's edge sum, and marks the ids in `newbits`.
 //   bitscan (h) : F_{h+1} = F_h ++ (newbits & ~visited) in ascending id order: chained scan of bitmap
 //                 popcounts (1024 words per tile) gives each new id its position; lidx[id] = position.
-//   compact     : one chained scan over the counts of all hops (hop-aligned tiles of 256 nodes, block-wide
-//                 decoupled look-back) = global edge positions -> per-hop offsets, E_h, and
-//                 src = lidx[padded id] copied into the packed output; then clears `visited` for F_H.
+//   compact     : every tile's global edge position from the per-tile edge sums (no chaining) -> per-hop
+//                 offsets, E_h, and src = lidx[padded id] copied into the packed output; then clears
+//                 `visited` for F_H.
 #include <cooperative_groups.h>
 
 #include <algorithm>
