@@ -197,15 +197,19 @@ def oracle_baseline(name, budget_s=15.0, seeds_cap=None, state=None):
             "sample": f"{done} seeds of {name} ({i} batch slices of <= {cfg['batch']}), sample + gather, single thread"}
 
 
-def profile_traffic(name):
-    """Per-launch DRAM bytes of the gather kernel from the committed ncu --set full summary, if any."""
+def profile_summary(name):
+    """The committed ncu summary of the gather kernel for `name` (per-launch DRAM bytes, launch shares)."""
     path = os.path.join(ROOT, "profiles", "ncu_gather_summary.json")
     try:
         with open(path) as f:
-            d = json.load(f)
-        return d.get(name, {}).get("dram_bytes_per_launch")
+            return json.load(f).get(name, {})
     except Exception:
-        return None
+        return {}
+
+
+def profile_traffic(name):
+    """Per-launch DRAM bytes of the gather kernel from the committed ncu --set full summary, if any."""
+    return profile_summary(name).get("dram_bytes_per_launch")
 
 
 def run_reference(args, rank, world):
@@ -422,6 +426,8 @@ def main():
             "gather_GBs": gather_gbs,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": profile_traffic(args.config), "kernel": "gather_tma4_kernel",
+                         "launch_shares": profile_summary(args.config).get("launch_shares"),
+                         "why_this_kernel": profile_summary(args.config).get("why_gather"),
                          "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})",
                          "alg_bytes_per_launch": alg_bytes, "launch_ms": gather_ms,
                          "gather_share_of_step": gather_ms / (ms / args.steps),
