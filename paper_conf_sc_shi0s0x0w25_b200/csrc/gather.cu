@@ -139,7 +139,10 @@ template <int N>
 __device__ __forceinline__ void bulk_wait_read() {
     asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
 }
-__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+// Before a block exits only its shared memory must no longer be read by its bulk stores; the writes
+// themselves complete with the grid (as CUTLASS's TMA-store epilogue tail does), so the last tile's write
+// latency is not added to every block.
+__device__ __forceinline__ void bulk_wait_exit() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 
 // Source address of output row i (a row of bin b at slot s, or of the replicated table at slot id).
 __device__ __forceinline__ const char* row_src(const BinTable& bins, const uint64_t* placement, int64_t id,
@@ -210,7 +213,7 @@ __global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const ui
             next_id = load_id(next);
         }
     }
-    if (lane == 0) bulk_wait_all();
+    if (lane == 0) bulk_wait_exit();
 }
 
 // TMA tile::gather4 variant of the bulk gather (sm_100a): one tensor copy fetches FOUR rows of the
@@ -229,13 +232,23 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
     const int lane = threadIdx.x;
     const uint32_t G = (4 * R + 127) & ~127u;
     const uint64_t pol_st = l2_policy(l2_store);
+    const int64_t t0 = blockIdx.x, dt = gridDim.x;
+    if (lane == 0) asm volatile("prefetch.tensormap [%0];" ::"l"(&tmap) : "memory");
+    // the first kStages tiles' ids are loaded speculatively (bounded by max_n, the ids buffer) together with
+    // the count instead of after it: one dependent global round trip fewer before the first row request.
+    // Ids past the count are never used (issue() replaces them by the tile's first row).
+    int32_t pre[kStages];
+#pragma unroll
+    for (int s = 0; s < kStages; s++) {
+        const int64_t r = (t0 + s * dt) * kTma4Rows + lane;
+        pre[s] = r < max_n ? (int32_t)__ldg(ids + r) : -1;
+    }
     const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
     const int64_t n_tiles = (n + kTma4Rows - 1) / kTma4Rows;
     if (lane == 0)
         for (int s = 0; s < kStages; s++) mbar_init(&full[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     __syncwarp();
-    const int64_t t0 = blockIdx.x, dt = gridDim.x;
     auto load_id = [&](int64_t tile) -> int32_t {
         const int64_t r = tile * kTma4Rows + lane;
         return (tile < n_tiles && r < n) ? (int32_t)__ldg(ids + r) : -1;
@@ -257,9 +270,6 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
                 "l"(&tmap), "r"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(&full[s]))
                 : "memory");
     };
-    int32_t pre[kStages];
-#pragma unroll
-    for (int s = 0; s < kStages; s++) pre[s] = load_id(t0 + s * dt);
     int64_t next = t0;
 #pragma unroll
     for (int s = 0; s < kStages; s++, next += dt)
@@ -284,7 +294,7 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
             next_id = load_id(next);
         }
     }
-    bulk_wait_all();
+    bulk_wait_exit();
 }
 
 // Relay service (H7): this rank (server) reads the host rows that `requester` routed through it and

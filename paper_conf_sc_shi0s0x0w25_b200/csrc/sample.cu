@@ -17,6 +17,7 @@
 #include <cooperative_groups.h>
 
 #include <algorithm>
+#include <climits>
 #include <cstdlib>
 
 #include "ctx.h"
@@ -284,6 +285,15 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp
     const bool live = g < NG;
     const int gbase = g * k;
     const unsigned below = (1u << lane) - 1u;
+    // lanes of this lane's group (a 32-bit match keyed by t alone, masked to the group, replaces a 64-bit
+    // match keyed by (group, t)); idle lanes never take part in a Floyd resolution
+    const unsigned gmask = (k >= 32 ? kFull : (1u << k) - 1u) << gbase;
+    // ranks of the chosen positions: every group's k choices go through shared memory (a slot of ks >= k
+    // ints per group, padded with INT_MAX) and each lane counts the smaller ones with 16-byte loads,
+    // ceil(k / 4) loads instead of k shuffles
+    __shared__ __align__(16) int32_t s_rank[8][128];
+    int32_t* const sw = s_rank[threadIdx.x >> 5];
+    const int ks = (k + 3) & ~3;
     const int64_t per_warp = (int64_t)NG * Q;
     const int64_t warps = (int64_t)gridDim.x * 8;
     for (int64_t base = ((int64_t)blockIdx.x * 8 + threadIdx.x / 32) * per_warp; base < F; base += warps * per_warp) {
@@ -338,7 +348,7 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp
             const int32_t jj = dq - k + i;
             const int32_t t = floyd ? (int32_t)dev::uniform(dev::draw(seed, v[q], a.h, i), (uint32_t)(jj + 1))
                                     : -1 - lane;  // unique sentinel: never matches
-            const unsigned same = __match_any_sync(kFull, ((uint64_t)(uint32_t)g << 32) | (uint32_t)t);
+            const unsigned same = __match_any_sync(kFull, (uint32_t)t) & gmask;
             const bool dup_a = floyd && (same & below) != 0;
             const int lstar = gbase + (t - (dq - k));  // the earlier lane of this group whose j equals t
             const bool ref = floyd && !dup_a && t >= dq - k && lstar < lane;
@@ -351,7 +361,21 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp
             }
             const int32_t c = ((dup >> lane) & 1u) ? jj : t;
             int r = 0;
-            for (int l = 0; l < k; l++) r += __shfl_sync(kFull, c, gbase + l) < c;
+            if (k > 1) {
+                if (live) {
+                    sw[g * ks + i] = c;
+                    for (int p = k + i; p < ks; p += k) sw[g * ks + p] = INT_MAX;
+                }
+                __syncwarp();
+                if (live) {
+                    const int4* row = reinterpret_cast<const int4*>(sw + g * ks);
+                    for (int l4 = 0; l4 < ks / 4; l4++) {
+                        const int4 x = row[l4];
+                        r += (x.x < c) + (x.y < c) + (x.z < c) + (x.w < c);
+                    }
+                }
+                __syncwarp();  // the slots are rewritten by the next node step
+            }
             if (floyd) {
                 pos[q] = c;
                 rnk[q] = r;
@@ -359,20 +383,29 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp
         }
 #pragma unroll
         for (int q = 0; q < Q; q++) u[q] = pos[q] >= 0 ? dev::ld_rand(a.indices + lo[q] + pos[q]) : 0;
+        // the warp's step covers nodes [base, base + NG * Q) (<= 128 < kSampleTile), so at most two
+        // compaction tiles: tile_a and the one after it; one warp reduction and RED per tile and step
+        const int64_t tile_a = base / kSampleTile, bound = (tile_a + 1) * kSampleTile;
+        uint32_t sum_a = 0, sum_b = 0;
 #pragma unroll
         for (int q = 0; q < Q; q++) {
             const bool node = live && idx[q] < F;
             const uint32_t c = node ? (uint32_t)(a.replace ? (d[q] > 0 ? k : 0) : min(d[q], k)) : 0u;
-            if (node && i == 0) a.cnt[idx[q]] = (int32_t)c;
+            if (node && i == 0) {
+                a.cnt[idx[q]] = (int32_t)c;
+                if (idx[q] < bound) sum_a += c;
+                else sum_b += c;
+            }
             if (node && pos[q] >= 0) {
                 a.pad[idx[q] * k + rnk[q]] = u[q];
                 mark_new(a.newbits, u[q]);
             }
-            // the step's NG nodes span at most two compaction tiles: one RED per tile and warp
-            const int64_t tile = idx[q] / kSampleTile;
-            const unsigned peers = __match_any_sync(kFull, (unsigned long long)tile);
-            const uint32_t sum = __reduce_add_sync(peers, i == 0 ? c : 0u);
-            if (lane == __ffs(peers) - 1 && sum) atomicAdd(a.tile_edges + tile, (unsigned long long)sum);
+        }
+        sum_a = __reduce_add_sync(kFull, sum_a);
+        sum_b = __reduce_add_sync(kFull, sum_b);
+        if (lane == 0) {
+            if (sum_a) atomicAdd(a.tile_edges + tile_a, (unsigned long long)sum_a);
+            if (sum_b) atomicAdd(a.tile_edges + tile_a + 1, (unsigned long long)sum_b);
         }
     }
 }
@@ -462,6 +495,7 @@ struct CompactArgs {
     int32_t H;
     int64_t tb[kMaxHops + 1];  // first tile of hop h (sum of ceil(F_bound_h' / kSampleTile), h' < h)
     int32_t k[kMaxHops];
+    uint32_t kmagic[kMaxHops];  // ceil(2^32 / k): slot / k = umulhi(slot, kmagic) for slot < 2^18, k <= 1024
     const int32_t* pad[kMaxHops];
     const int32_t* cnt[kMaxHops];
 };
@@ -488,8 +522,10 @@ __device__ __forceinline__ void block_sum2(int64_t& x, int64_t& y, int64_t (*red
 // counts of the tiles before it, which the hop kernels accumulated per tile (no chained scan, no waiting
 // on other blocks); the hop's base is the sum over the earlier hops' tiles.
 __global__ void __launch_bounds__(kSampleTile, MOMENT_SAMPLE_MIN_BLOCKS) compact_kernel(CompactArgs a) {
+    constexpr int kCopyUnroll = 8;  // padded slots per thread in flight (id load -> lidx load -> src store)
     __shared__ int64_t s_red[kSampleTile / 32];
     __shared__ int64_t s_red2[kSampleTile / 32][2];
+    __shared__ int32_t s_excl[kSampleTile], s_cnt[kSampleTile];
     const int64_t n_tiles = a.tb[a.H];
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         // hops with an empty frontier have no tile: write their (empty) offsets and E_h here
@@ -530,21 +566,41 @@ __global__ void __launch_bounds__(kSampleTile, MOMENT_SAMPLE_MIN_BLOCKS) compact
                 a.counts[a.H + 1 + h] = rel + c;
             }
         }
-        // copy + relabel this node's c edges: up to 16 padded ids and their 16 lidx loads in flight at once
-        if (idx < F) {
-            const int32_t* p = a.pad[h] + idx * a.k[h];
-            for (int r0 = 0; r0 < c; r0 += 16) {
-                int32_t id[16], li[16];
+        // copy + relabel the tile's edges slot-parallel: the tile's padded rows (nodes x k ints) are read
+        // coalesced, slot s belongs to node s / k at rank s % k and is an edge iff its rank < the node's
+        // count; kCopyUnroll independent lidx loads in flight per thread
+        s_excl[threadIdx.x] = (int32_t)excl;
+        s_cnt[threadIdx.x] = c;
+        __syncthreads();
+        {
+            const int k = a.k[h];
+            const uint32_t km = a.kmagic[h];
+            const int32_t* p = a.pad[h] + lt * kSampleTile * k;
+            int32_t* out = a.src + (gpos - excl);  // the tile's first edge
+            const int slots = (int)min((int64_t)kSampleTile, F - lt * kSampleTile) * k;
+            for (int s0 = threadIdx.x; s0 < slots; s0 += kSampleTile * kCopyUnroll) {
+                int32_t id[kCopyUnroll], at[kCopyUnroll];
 #pragma unroll
-                for (int r = 0; r < 16; r++) id[r] = r0 + r < c ? __ldg(p + r0 + r) : 0;
+                for (int u = 0; u < kCopyUnroll; u++) {
+                    const int sl = s0 + u * kSampleTile;
+                    at[u] = -1;
+                    if (sl < slots) {
+                        const int node = k == 1 ? sl : (int)__umulhi((uint32_t)sl, km);
+                        const int r = sl - node * k;
+                        if (r < s_cnt[node]) {
+                            at[u] = s_excl[node] + r;
+                            id[u] = __ldg(p + sl);
+                        }
+                    }
+                }
 #pragma unroll
-                for (int r = 0; r < 16; r++) li[r] = r0 + r < c ? dev::ld_rand(a.lidx + id[r]) : 0;
+                for (int u = 0; u < kCopyUnroll; u++) id[u] = at[u] >= 0 ? dev::ld_rand(a.lidx + id[u]) : 0;
 #pragma unroll
-                for (int r = 0; r < 16; r++)
-                    if (r0 + r < c) a.src[gpos + r0 + r] = li[r];
+                for (int u = 0; u < kCopyUnroll; u++)
+                    if (at[u] >= 0) out[at[u]] = id[u];
             }
         }
-        __syncthreads();  // s_red / s_red2 are reused by the next tile
+        __syncthreads();  // s_red / s_red2 / s_excl / s_cnt are reused by the next tile
     }
     const int64_t FH = a.counts[a.H];
     for (int64_t i = (int64_t)blockIdx.x * kSampleTile + threadIdx.x; i < FH; i += (int64_t)gridDim.x * kSampleTile)
@@ -707,6 +763,7 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
                    ctx->tile_edges + ca.tb[h + 1], n_zero};
         bitscan_kernel<<<(int)std::min<int64_t>(n_scan_tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
         ca.k[h] = k;
+        ca.kmagic[h] = k == 1 ? 0u : (uint32_t)(((uint64_t(1) << 32) + (uint64_t)k - 1) / (uint64_t)k);
         ca.pad[h] = ctx->pad + pad_off;
         ca.cnt[h] = ctx->cnt + cnt_off;
         pad_off += F_bound * k;

@@ -42,10 +42,12 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", default="C2")
     ap.add_argument("--steps", type=int, default=400)
+    ap.add_argument("--lanes", default="1,2,4,8,16")
     args = ap.parse_args()
-    st = bench.build_state(args.config, "cuda:0", 0, 1, inflight=8)
+    lanes = [int(x) for x in args.lanes.split(",")]
+    st = bench.build_state(args.config, "cuda:0", 0, 1, inflight=max(lanes))
     batches = [st.batch(i) for i in range(args.steps)]
-    for P in (1, 2, 4, 8):
+    for P in lanes:
         for L, b in zip(st.lanes[:P], batches):  # lanes hold a real F_H for gather-only
             L.ctx.step(st.graph.indptr, st.graph.indices, b[0], st.fanout, b[1], L.bufs, L.rows, stream=L.stream)
         torch.cuda.synchronize()
