@@ -108,6 +108,8 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     if (const char* v = std::getenv("MOMENT_STEP_FORK")) c->step_fork = std::atoi(v) != 0;
     if (const char* v = std::getenv("MOMENT_INIT_KERNEL")) c->init_in_hop0 = std::atoi(v) == 0;
     if (const char* v = std::getenv("MOMENT_COMPACT_GRID")) c->compact_grid_per_sm = std::max(1, std::atoi(v));
+    c->sparse_scan = (a->n_vertices + 31) / 32 > kSparseScanMinWords;
+    if (const char* v = std::getenv("MOMENT_SPARSE_SCAN")) c->sparse_scan = std::atoi(v) != 0;
     if (const char* l2 = std::getenv("MOMENT_GATHER_L2")) {  // "<load><store>" digits, e.g. "01"
         if (std::strlen(l2) == 2) {
             c->l2_load_policy = l2[0] - '0';
@@ -136,6 +138,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     const int64_t n_words_pad = (c->n_words + kBitscanTileWords - 1) / kBitscanTileWords * kBitscanTileWords;
     const int64_t o_newbits = cv.take<uint32_t>(n_words_pad);
     const int64_t o_visited = cv.take<uint32_t>(n_words_pad);
+    const int64_t o_summary = cv.take<uint32_t>(n_words_pad / 32);
     const int64_t scan_tiles = n_words_pad / kBitscanTileWords;
     c->bitscan_tiles_off.resize(a->max_hops);
     int64_t nts = 0, cnt_total = 0;
@@ -181,6 +184,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     c->lidx = reinterpret_cast<int32_t*>(w + o_lidx);
     c->newbits = reinterpret_cast<uint32_t*>(w + o_newbits);
     c->visited = reinterpret_cast<uint32_t*>(w + o_visited);
+    c->summary = reinterpret_cast<uint32_t*>(w + o_summary);
     c->tile_status = reinterpret_cast<uint64_t*>(w + o_tiles);
     c->tile_edges = reinterpret_cast<unsigned long long*>(w + o_tile_edges);
     c->tickets = reinterpret_cast<uint32_t*>(w + o_tickets);

@@ -45,7 +45,11 @@ struct moment_ctx_s {
     int32_t* lidx = nullptr;        // [n_vertices]: local index of v in the current batch (valid for F_H)
     uint32_t* newbits = nullptr;    // [n_words]: ids emitted at the current hop
     uint32_t* visited = nullptr;    // [n_words]: F_h membership
+    uint32_t* summary = nullptr;    // [n_words / 32]: newbits words marked at the current hop (sparse scan)
     int64_t n_words = 0;
+    // sparse scan (summary bitmap, scan cost proportional to the touched words) for large graphs: auto when
+    // n_words > kSparseScanMinWords (MOMENT_SPARSE_SCAN=0/1 forces it off/on)
+    int32_t sparse_scan = 0;
     unsigned long long* tile_edges = nullptr;  // edges per compaction tile of every hop (bound-numbered)
     int64_t n_tile_edges = 0;
     uint64_t* tile_status = nullptr;  // decoupled look-back descriptors: compact chain, then bitscan per hop
@@ -99,6 +103,7 @@ constexpr int kSampleTile = 256;     // frontier nodes per sampler tile
 constexpr int kBitscanWordsPerThread = 4;  // one uint4 per thread (16 measured slower: 13.1 vs 7.6 us/launch)
 constexpr int kBitscanThreads = 256;
 constexpr int kBitscanTileWords = kBitscanWordsPerThread * kBitscanThreads;  // 1024 words = 32768 ids
+constexpr int64_t kSparseScanMinWords = 1 << 18;  // > 8.4 M vertices: C3-C5 scan sparsely, C1/C2 densely
 constexpr int kBucketTile = 1024;    // requests per bucketing tile
 constexpr int kMaxFanout = 1024;
 

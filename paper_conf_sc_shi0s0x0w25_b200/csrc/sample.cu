@@ -46,6 +46,7 @@ struct HopArgs {
     int32_t* pad;      // [F_bound_h * k]: node idx's samples at pad[idx * k + r]
     int32_t* cnt;      // [F_bound_h]: samples of node idx
     uint32_t* newbits;
+    uint32_t* summary;     // sparse scan only (else null): bit w of summary = newbits word w was marked
     const uint64_t* call;  // device call block: [0] = rng_seed, [1] = seeds pointer (written per call)
     int32_t h, k;
     int32_t replace;
@@ -75,8 +76,11 @@ struct InitArgs {
 };
 
 // Fire-and-forget: the result is unused, so this is a RED.OR the issuing warp never waits on.
-__device__ __forceinline__ void mark_new(uint32_t* newbits, int32_t u) {
-    atomicOr(newbits + (u >> 5), 1u << (u & 31));
+// Sparse scan (large graphs): the newbits word's bit in `summary` is marked too, so that the bitscan reads
+// only the words a hop touched instead of the whole n-bit bitmap.
+__device__ __forceinline__ void mark_new(const HopArgs& a, int32_t u) {
+    atomicOr(a.newbits + (u >> 5), 1u << (u & 31));
+    if (a.summary) atomicOr(a.summary + (u >> 10), 1u << ((u >> 5) & 31));
 }
 
 // Floyd's k choices for node v at hop h, lane i < k owning choice i (k <= G): t_i = uniform(draw(i),
@@ -148,7 +152,7 @@ __device__ void sample_node_wide(const cg::thread_block_tile<32>& grp, const Hop
         if (i < k) {
             const int32_t u = __ldg(a.indices + lo + mine[q]);
             out[rk[q]] = u;
-            mark_new(a.newbits, u);
+            mark_new(a, u);
         }
     }
 }
@@ -163,13 +167,13 @@ __device__ __forceinline__ void sample_node_slow(const cg::thread_block_tile<G>&
         for (int i = lane; i < k; i += G) {
             const int32_t u = __ldg(a.indices + lo + dev::uniform(dev::draw(seed, v, a.h, i), (uint32_t)d));
             out[i] = u;
-            mark_new(a.newbits, u);
+            mark_new(a, u);
         }
     } else if (d <= k) {
         for (int p = lane; p < d; p += G) {
             const int32_t u = __ldg(a.indices + lo + p);
             out[p] = u;
-            mark_new(a.newbits, u);
+            mark_new(a, u);
         }
     } else {
         if constexpr (G == 32) sample_node_wide(grp, a, seed, v, lo, d, out);
@@ -244,7 +248,7 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_kern
             }
             if (pos[q] >= 0) {
                 a.pad[idx * k + rnk[q]] = u[q];
-                mark_new(a.newbits, u[q]);
+                mark_new(a, u[q]);
             }
         }
         if (k > G) {
@@ -398,7 +402,7 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp
             }
             if (node && pos[q] >= 0) {
                 a.pad[idx[q] * k + rnk[q]] = u[q];
-                mark_new(a.newbits, u[q]);
+                mark_new(a, u[q]);
             }
         }
         sum_a = __reduce_add_sync(kFull, sum_a);
@@ -416,6 +420,7 @@ struct ScanArgs {
     int32_t* lidx;
     uint32_t* newbits;
     uint32_t* visited;
+    uint32_t* summary;  // sparse scan: touched-word bitmap of newbits (cleared here)
     uint64_t* tile_status;
     uint32_t* ticket;
     int64_t n_words;
@@ -480,6 +485,79 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
             if (nb[q]) a.newbits[w] = 0u;
             if (nw) a.visited[w] = vs[q] | nw;  // no re-read: the tile owns its words
         }
+        __syncthreads();
+    }
+}
+
+// Sparse variant for large graphs (n_words >> touched words): a tile is kSparseTileWords newbits words =
+// one summary word per thread; a thread reads only the newbits / visited words whose summary bit is set
+// (the words the hop marked), 4 at a time, so the scan costs O(touched words + n / 1024) instead of
+// O(n / 32). Same result and order as bitscan_kernel: a thread's words are consecutive and its ids
+// ascending, threads of a tile and tiles are in id order.
+constexpr int kSparseTileWords = 32 * kBitscanThreads;
+
+template <typename Fn>
+__device__ __forceinline__ void for_touched_words(uint32_t sm, const uint32_t* newbits, const uint32_t* visited,
+                                                  int64_t w_base, Fn fn) {
+    while (sm) {
+        int wi[4];
+        uint32_t nb[4], vs[4];
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            wi[j] = sm ? __ffs(sm) - 1 : -1;
+            sm &= sm - 1;
+        }
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            nb[j] = wi[j] >= 0 ? __ldcg(newbits + w_base + wi[j]) : 0u;
+            vs[j] = wi[j] >= 0 ? __ldcg(visited + w_base + wi[j]) : 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < 4; j++)
+            if (wi[j] >= 0) fn(w_base + wi[j], nb[j], vs[j]);
+    }
+}
+
+__global__ void __launch_bounds__(kBitscanThreads) bitscan_sparse_kernel(ScanArgs a) {
+    __shared__ int64_t s_red[kBitscanThreads / 32];
+    __shared__ uint32_t s_tile;
+    __shared__ int s_nearest;
+    const int64_t F = a.counts[a.h];
+    const int64_t n_tiles = (a.n_words + kSparseTileWords - 1) / kSparseTileWords;
+    const int64_t n_summary = (a.n_words + 31) / 32;
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < a.n_zero; j += (int64_t)gridDim.x * blockDim.x)
+        a.zero[j] = 0;
+    for (;;) {
+        if (threadIdx.x == 0) s_tile = atomicAdd(a.ticket, 1u);
+        __syncthreads();
+        const int64_t tile = s_tile;
+        if (tile >= n_tiles) break;
+        const int64_t sw = tile * kBitscanThreads + threadIdx.x;  // this thread's summary word
+        const uint32_t sm = sw < n_summary ? __ldcg(a.summary + sw) : 0u;
+        const int64_t w_base = sw * 32;
+        int cnt = 0;
+        for_touched_words(sm, a.newbits, a.visited, w_base,
+                          [&](int64_t, uint32_t nb, uint32_t vs) { cnt += __popc(nb & ~vs); });
+        int64_t agg;
+        const int64_t excl = dev::block_exclusive_scan<kBitscanThreads>(cnt, &agg, s_red);
+        const int64_t prefix = dev::lookback_block<kBitscanThreads>(a.tile_status, tile, agg, s_red, &s_nearest);
+        int64_t pos = F + prefix + excl;
+        if (tile == n_tiles - 1 && threadIdx.x == 0) a.counts[a.h + 1] = F + prefix + agg;
+        for_touched_words(sm, a.newbits, a.visited, w_base, [&](int64_t w, uint32_t nb, uint32_t vs) {
+            const uint32_t nw = nb & ~vs;
+            uint32_t bits = nw;
+            while (bits) {
+                const int b = __ffs(bits) - 1;
+                bits &= bits - 1;
+                const int64_t id = w * 32 + b;
+                a.nodes[pos] = id;
+                a.lidx[id] = (int32_t)pos;
+                pos++;
+            }
+            a.newbits[w] = 0u;
+            if (nw) a.visited[w] = vs | nw;
+        });
+        if (sm) a.summary[sw] = 0u;
         __syncthreads();
     }
 }
@@ -668,7 +746,8 @@ void launch_sample_warp(const HopArgs& a, int64_t max_F, int big_q, cudaStream_t
 // Same shared-memory carveout for every kernel of the library (see configure_gather_kernels).
 moment_status configure_sample_kernels(int carveout) {
     if (carveout < 0) return MOMENT_OK;
-    const void* fns[] = {(const void*)init_kernel, (const void*)bitscan_kernel, (const void*)compact_kernel,
+    const void* fns[] = {(const void*)init_kernel, (const void*)bitscan_kernel, (const void*)bitscan_sparse_kernel,
+                         (const void*)compact_kernel,
                          (const void*)hop_sample_kernel<4, 1>, (const void*)hop_sample_kernel<8, 1>,
                          (const void*)hop_sample_kernel<16, 1>, (const void*)hop_sample_kernel<32, 1>,
                          (const void*)hop_sample_kernel<4, 2>, (const void*)hop_sample_kernel<8, 2>,
@@ -749,7 +828,8 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
     for (int h = 0; h < H; h++) {
         const int k = p->fanout[h];
         HopArgs a{csr->indptr, csr->indices, out->nodes, out->counts, ctx->pad + pad_off, ctx->cnt + cnt_off,
-                  ctx->newbits, call, h, k, replace, ctx->hop_grid_per_sm, ctx->tile_edges + ca.tb[h]};
+                  ctx->newbits, ctx->sparse_scan ? ctx->summary : nullptr, call, h, k, replace,
+                  ctx->hop_grid_per_sm, ctx->tile_edges + ca.tb[h]};
         const int q = ctx->hop_nodes_per_group;
         if (h == 0 && init_in_hop0) launch_sample_warp_q<1, true>(a, F_bound, stream, init);
         else if (ctx->hop_warp_segmented && k <= 32) launch_sample_warp(a, F_bound, q, stream);
@@ -758,10 +838,15 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         else if (k <= 16) launch_sample_hop<16>(a, F_bound, q, stream);
         else launch_sample_hop<32>(a, F_bound, q, stream);
         const int64_t n_zero = h + 1 < H ? ca.tb[h + 2] - ca.tb[h + 1] : 0;  // the next hop's tile sums
-        ScanArgs s{out->nodes, out->counts, ctx->lidx, ctx->newbits, ctx->visited,
+        ScanArgs s{out->nodes, out->counts, ctx->lidx, ctx->newbits, ctx->visited, ctx->summary,
                    ctx->tile_status + ctx->bitscan_tiles_off[h], ctx->tickets + 1 + h, ctx->n_words, h,
                    ctx->tile_edges + ca.tb[h + 1], n_zero};
-        bitscan_kernel<<<(int)std::min<int64_t>(n_scan_tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
+        if (ctx->sparse_scan) {
+            const int64_t tiles = (ctx->n_words + kSparseTileWords - 1) / kSparseTileWords;
+            bitscan_sparse_kernel<<<(int)std::min<int64_t>(tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
+        } else {
+            bitscan_kernel<<<(int)std::min<int64_t>(n_scan_tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
+        }
         ca.k[h] = k;
         ca.kmagic[h] = k == 1 ? 0u : (uint32_t)(((uint64_t(1) << 32) + (uint64_t)k - 1) / (uint64_t)k);
         ca.pad[h] = ctx->pad + pad_off;

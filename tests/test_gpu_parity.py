@@ -68,12 +68,13 @@ def test_sample_fanouts_and_ragged(orc, c1, fanout, n_seeds):
     assert_same_sample(got, want)
 
 
-@pytest.mark.parametrize("knob", [("MOMENT_HOP_WARP", "0"), ("MOMENT_INIT_KERNEL", "1")])
-@pytest.mark.parametrize("fanout", [[15, 10, 5], [7, 3], [20]])
+@pytest.mark.parametrize("knob", [("MOMENT_HOP_WARP", "0"), ("MOMENT_INIT_KERNEL", "1"), ("MOMENT_SPARSE_SCAN", "1")])
+@pytest.mark.parametrize("fanout", [[15, 10, 5], [7, 3], [20], [40, 2]])
 def test_sample_kernel_variants(orc, c1, fanout, knob, monkeypatch):
     """The other sampler kernels give the same result as the default: MOMENT_HOP_WARP=0 selects the
     power-of-two lane tiles (always used for k > 32), MOMENT_INIT_KERNEL=1 a separate init kernel instead of
-    the first hop's sampler initialising the call."""
+    the first hop's sampler initialising the call, MOMENT_SPARSE_SCAN=1 the summary-bitmap bitscan that
+    graphs above 8.4 M vertices use (C3-C5)."""
     _, g = c1
     monkeypatch.setenv(*knob)
     seeds = np.random.default_rng(5).choice(g.n, 1000, replace=False)
@@ -135,9 +136,12 @@ def test_sample_check_flags_bad_seeds(c1):
     assert e.value.status == M.EINVAL
 
 
-def test_sample_reused_ctx_many_batches(orc, c1):
-    """The workspace (lidx, bitmaps, tile descriptors) is reset correctly between calls."""
+@pytest.mark.parametrize("sparse", ["0", "1"])
+def test_sample_reused_ctx_many_batches(orc, c1, sparse, monkeypatch):
+    """The workspace (lidx, bitmaps, summary bitmap, tile descriptors) is reset correctly between calls,
+    for the dense and the sparse (summary-bitmap) bitscan."""
     cfg, g = c1
+    monkeypatch.setenv("MOMENT_SPARSE_SCAN", sparse)
     ctx = M.Ctx(n_vertices=g.n, max_seeds=1024, max_fanout=[10, 5], device=0)
     rng = np.random.default_rng(0)
     for b in range(4):

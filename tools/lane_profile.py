@@ -41,8 +41,9 @@ def main():
     ap.add_argument("--lanes", type=int, default=8)
     ap.add_argument("--mode", default="full")
     ap.add_argument("--steps", type=int, default=64)
+    ap.add_argument("--config", default="C2")
     a = ap.parse_args()
-    st = bench.build_state("C2", "cuda:0", 0, 1, inflight=a.lanes)
+    st = bench.build_state(a.config, "cuda:0", 0, 1, inflight=a.lanes)
     batches = [st.batch(i) for i in range(a.steps)]
     profile(st, batches[:16], a.lanes, a.mode)
     w1, d1 = profile(st, batches, 1, a.mode)
