@@ -110,6 +110,10 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     if (const char* v = std::getenv("MOMENT_COMPACT_GRID")) c->compact_grid_per_sm = std::max(1, std::atoi(v));
     c->sparse_scan = (a->n_vertices + 31) / 32 > kSparseScanMinWords;
     if (const char* v = std::getenv("MOMENT_SPARSE_SCAN")) c->sparse_scan = std::atoi(v) != 0;
+    if (const char* v = std::getenv("MOMENT_SPARSE_NT")) {
+        const int nt = std::atoi(v);
+        c->sparse_threads = nt >= 1024 ? 1024 : nt >= 512 ? 512 : 256;
+    }
     if (const char* l2 = std::getenv("MOMENT_GATHER_L2")) {  // "<load><store>" digits, e.g. "01"
         if (std::strlen(l2) == 2) {
             c->l2_load_policy = l2[0] - '0';

@@ -50,6 +50,7 @@ struct moment_ctx_s {
     // sparse scan (summary bitmap, scan cost proportional to the touched words) for large graphs: auto when
     // n_words > kSparseScanMinWords (MOMENT_SPARSE_SCAN=0/1 forces it off/on)
     int32_t sparse_scan = 0;
+    int32_t sparse_threads = 1024;  // threads (= summary words) per sparse scan tile (MOMENT_SPARSE_NT: 256/512/1024)
     unsigned long long* tile_edges = nullptr;  // edges per compaction tile of every hop (bound-numbered)
     int64_t n_tile_edges = 0;
     uint64_t* tile_status = nullptr;  // decoupled look-back descriptors: compact chain, then bitscan per hop

@@ -494,7 +494,6 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
 // (the words the hop marked), 4 at a time, so the scan costs O(touched words + n / 1024) instead of
 // O(n / 32). Same result and order as bitscan_kernel: a thread's words are consecutive and its ids
 // ascending, threads of a tile and tiles are in id order.
-constexpr int kSparseTileWords = 32 * kBitscanThreads;
 
 template <typename Fn>
 __device__ __forceinline__ void for_touched_words(uint32_t sm, const uint32_t* newbits, const uint32_t* visited,
@@ -518,8 +517,10 @@ __device__ __forceinline__ void for_touched_words(uint32_t sm, const uint32_t* n
     }
 }
 
-__global__ void __launch_bounds__(kBitscanThreads) bitscan_sparse_kernel(ScanArgs a) {
-    __shared__ int64_t s_red[kBitscanThreads / 32];
+template <int NT>
+__global__ void __launch_bounds__(NT) bitscan_sparse_kernel(ScanArgs a) {
+    constexpr int kSparseTileWords = 32 * NT;
+    __shared__ int64_t s_red[NT / 32];
     __shared__ uint32_t s_tile;
     __shared__ int s_nearest;
     const int64_t F = a.counts[a.h];
@@ -532,15 +533,15 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_sparse_kernel(ScanArg
         __syncthreads();
         const int64_t tile = s_tile;
         if (tile >= n_tiles) break;
-        const int64_t sw = tile * kBitscanThreads + threadIdx.x;  // this thread's summary word
+        const int64_t sw = tile * NT + threadIdx.x;  // this thread's summary word
         const uint32_t sm = sw < n_summary ? __ldcg(a.summary + sw) : 0u;
         const int64_t w_base = sw * 32;
         int cnt = 0;
         for_touched_words(sm, a.newbits, a.visited, w_base,
                           [&](int64_t, uint32_t nb, uint32_t vs) { cnt += __popc(nb & ~vs); });
         int64_t agg;
-        const int64_t excl = dev::block_exclusive_scan<kBitscanThreads>(cnt, &agg, s_red);
-        const int64_t prefix = dev::lookback_block<kBitscanThreads>(a.tile_status, tile, agg, s_red, &s_nearest);
+        const int64_t excl = dev::block_exclusive_scan<NT>(cnt, &agg, s_red);
+        const int64_t prefix = dev::lookback_block<NT>(a.tile_status, tile, agg, s_red, &s_nearest);
         int64_t pos = F + prefix + excl;
         if (tile == n_tiles - 1 && threadIdx.x == 0) a.counts[a.h + 1] = F + prefix + agg;
         for_touched_words(sm, a.newbits, a.visited, w_base, [&](int64_t w, uint32_t nb, uint32_t vs) {
@@ -746,7 +747,8 @@ void launch_sample_warp(const HopArgs& a, int64_t max_F, int big_q, cudaStream_t
 // Same shared-memory carveout for every kernel of the library (see configure_gather_kernels).
 moment_status configure_sample_kernels(int carveout) {
     if (carveout < 0) return MOMENT_OK;
-    const void* fns[] = {(const void*)init_kernel, (const void*)bitscan_kernel, (const void*)bitscan_sparse_kernel,
+    const void* fns[] = {(const void*)init_kernel, (const void*)bitscan_kernel, (const void*)bitscan_sparse_kernel<256>,
+                         (const void*)bitscan_sparse_kernel<512>, (const void*)bitscan_sparse_kernel<1024>,
                          (const void*)compact_kernel,
                          (const void*)hop_sample_kernel<4, 1>, (const void*)hop_sample_kernel<8, 1>,
                          (const void*)hop_sample_kernel<16, 1>, (const void*)hop_sample_kernel<32, 1>,
@@ -841,9 +843,13 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         ScanArgs s{out->nodes, out->counts, ctx->lidx, ctx->newbits, ctx->visited, ctx->summary,
                    ctx->tile_status + ctx->bitscan_tiles_off[h], ctx->tickets + 1 + h, ctx->n_words, h,
                    ctx->tile_edges + ca.tb[h + 1], n_zero};
-        if (ctx->sparse_scan) {
-            const int64_t tiles = (ctx->n_words + kSparseTileWords - 1) / kSparseTileWords;
-            bitscan_sparse_kernel<<<(int)std::min<int64_t>(tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
+        if (ctx->sparse_scan) {  // one summary word (32 newbits words) per thread
+            const int nt = ctx->sparse_threads;
+            const int64_t tiles = (ctx->n_words + 32 * nt - 1) / (32 * nt);
+            const int grid = (int)std::min<int64_t>(tiles, 148 * (1024 / nt) * 2);
+            if (nt == 1024) bitscan_sparse_kernel<1024><<<grid, 1024, 0, stream>>>(s);
+            else if (nt == 512) bitscan_sparse_kernel<512><<<grid, 512, 0, stream>>>(s);
+            else bitscan_sparse_kernel<256><<<grid, 256, 0, stream>>>(s);
         } else {
             bitscan_kernel<<<(int)std::min<int64_t>(n_scan_tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
         }

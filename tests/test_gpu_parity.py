@@ -68,7 +68,9 @@ def test_sample_fanouts_and_ragged(orc, c1, fanout, n_seeds):
     assert_same_sample(got, want)
 
 
-@pytest.mark.parametrize("knob", [("MOMENT_HOP_WARP", "0"), ("MOMENT_INIT_KERNEL", "1"), ("MOMENT_SPARSE_SCAN", "1")])
+@pytest.mark.parametrize("knob", [(("MOMENT_HOP_WARP", "0"),), (("MOMENT_INIT_KERNEL", "1"),),
+                                  (("MOMENT_SPARSE_SCAN", "1"),),
+                                  (("MOMENT_SPARSE_SCAN", "1"), ("MOMENT_SPARSE_NT", "1024"))])
 @pytest.mark.parametrize("fanout", [[15, 10, 5], [7, 3], [20], [40, 2]])
 def test_sample_kernel_variants(orc, c1, fanout, knob, monkeypatch):
     """The other sampler kernels give the same result as the default: MOMENT_HOP_WARP=0 selects the
@@ -76,7 +78,8 @@ def test_sample_kernel_variants(orc, c1, fanout, knob, monkeypatch):
     the first hop's sampler initialising the call, MOMENT_SPARSE_SCAN=1 the summary-bitmap bitscan that
     graphs above 8.4 M vertices use (C3-C5)."""
     _, g = c1
-    monkeypatch.setenv(*knob)
+    for k, v in knob:
+        monkeypatch.setenv(k, v)
     seeds = np.random.default_rng(5).choice(g.n, 1000, replace=False)
     got, want = sample_both(orc, g, seeds, fanout, 4242)
     assert_same_sample(got, want)
