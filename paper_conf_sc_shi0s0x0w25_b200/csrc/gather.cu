@@ -226,12 +226,13 @@ constexpr int kTma4Rows = 32;  // rows per tile = 8 groups of 4
 template <int kStages>
 __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__ CUtensorMap tmap,
                                                          const int64_t* __restrict__ ids, const int64_t* n_dev,
-                                                         int64_t max_n, uint32_t R, int l2_store, char* __restrict__ out) {
+                                                         int64_t max_n, uint32_t R, int l2_load, int l2_store,
+                                                         char* __restrict__ out) {
     extern __shared__ __align__(128) char stage[];  // kStages * 8 * G
     __shared__ __align__(8) uint64_t full[kStages];
     const int lane = threadIdx.x;
     const uint32_t G = (4 * R + 127) & ~127u;
-    const uint64_t pol_st = l2_policy(l2_store);
+    const uint64_t pol_st = l2_policy(l2_store), pol_ld = l2_policy(l2_load);
     const int64_t t0 = blockIdx.x, dt = gridDim.x;
     if (lane == 0) asm volatile("prefetch.tensormap [%0];" ::"l"(&tmap) : "memory");
     // the first kStages tiles' ids are loaded speculatively (bounded by max_n, the ids buffer) together with
@@ -263,12 +264,20 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
         const int32_t r2 = __shfl_sync(0xffffffffu, rid, 4 * g + 2), r3 = __shfl_sync(0xffffffffu, rid, 4 * g + 3);
         if (lane == 0) mbar_expect_tx(&full[s], (uint32_t)groups * 4u * R);
         __syncwarp();
-        if (lane < groups)
-            asm volatile(
-                "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes [%0], [%1, {%2, "
-                "%3, %4, %5, %6}], [%7];" ::"r"(smem_u32(stage + ((size_t)s * 8 + lane) * G)),
-                "l"(&tmap), "r"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(&full[s]))
-                : "memory");
+        if (lane < groups) {
+            if (l2_load)  // L2 eviction priority of the fetched rows (MOMENT_GATHER_L2 first digit)
+                asm volatile(
+                    "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes.L2::cache_hint "
+                    "[%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(smem_u32(stage + ((size_t)s * 8 + lane) * G)),
+                    "l"(&tmap), "r"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(&full[s])), "l"(pol_ld)
+                    : "memory");
+            else
+                asm volatile(
+                    "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes [%0], [%1, {%2, "
+                    "%3, %4, %5, %6}], [%7];" ::"r"(smem_u32(stage + ((size_t)s * 8 + lane) * G)),
+                    "l"(&tmap), "r"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(&full[s]))
+                    : "memory");
+        }
     };
     int64_t next = t0;
 #pragma unroll
@@ -555,7 +564,8 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
         const int64_t tiles = (max_n + kTma4Rows - 1) / kTma4Rows;
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)148 * bps));
         gather_tma4_kernel<4><<<grid, 32, smem, stream>>>(ctx->tma_map, ids, n_dev, max_n, (uint32_t)ctx->row_bytes,
-                                                          ctx->l2_store_policy, reinterpret_cast<char*>(out));
+                                                          ctx->l2_load_policy, ctx->l2_store_policy,
+                                                          reinterpret_cast<char*>(out));
         return cuda_check(cudaGetLastError(), "moment_gather: tma4 launch");
     }
     if (bulk && route == nullptr) {
