@@ -121,7 +121,16 @@ typedef struct {
                                          max-flow of topo ("modeled by maximum flow", R7) */
     int64_t pool;                     /* vertices per decision; <= 0 means 100 */
     int32_t mode;                     /* MOMENT_PLACE_DDAK, or MOMENT_PLACE_HASH (uniform baseline) */
+    int64_t replicate_rows;           /* r >= 0 (DDAK mode only; R25): the r first vertices
+                                         of the DDAK order are copied into EVERY GPU_HBM bin at slots 0..r-1
+                                         (bin_of = MOMENT_BIN_REPLICA, slot_of = position in the order); the
+                                         other vertices are placed by DDAK over the GPU bins' capacities minus
+                                         r (their slots start at r) and the other bins unchanged. Requires
+                                         r <= every GPU bin's capacity. 0 = plain DDAK (bit-identical). */
 } moment_place_args;
+
+/* bin_of value of a vertex replicated in every GPU_HBM bin (replicate_rows > 0). */
+#define MOMENT_BIN_REPLICA (-2)
 
 typedef struct {
     int32_t* bin_of;           /* host [n_vertices] */
@@ -129,6 +138,7 @@ typedef struct {
     uint64_t* bin_access;      /* host [n_bins] or NULL: final Bin_access (sum of hotness) */
     int64_t* bin_rows_used;    /* host [n_bins] or NULL: final Bin_currentCapacity */
     int64_t* bin_traffic_used; /* host [n_bins] or NULL: the Bin_traffic the decision used */
+    uint64_t* replica_access;  /* host [1] or NULL: sum of the hotness of the replicated vertices */
 } moment_place_out;
 
 /* topo may be NULL when bin_tier and bin_traffic are given. Errors: EINVAL, EINFEASIBLE (sum of
@@ -137,6 +147,11 @@ moment_status moment_place(moment_topo_t topo, const moment_place_args* args, mo
 /* packed[v] = ((uint64)bin_of[v] << 40) | slot_of[v] — the device placement map layout (D3). */
 moment_status moment_place_pack(int64_t n_vertices, const int32_t* bin_of, const int64_t* slot_of,
                                 uint64_t* packed);
+/* The device map of ONE rank when replicas exist: a MOMENT_BIN_REPLICA vertex maps to
+ * (replica_bin << 40) | slot — replica_bin = that rank's own GPU_HBM bin, so every rank reads its
+ * replicas locally; other vertices as moment_place_pack. Errors: EINVAL (replica_bin out of range). */
+moment_status moment_place_pack_rank(int64_t n_vertices, const int32_t* bin_of, const int64_t* slot_of,
+                                     int32_t replica_bin, uint64_t* packed);
 
 /* ================================================================================================
  * P5 — time-bisection plan + quotas (ingest model R10-R12)
@@ -156,6 +171,9 @@ typedef struct {
                                         (bytes one GPU reads from b per batch); other entries ignored */
     int64_t nvlink_cap;              /* bytes/us per GPU per direction; 0 = no NVLink (no relay) */
     int64_t hbm_cap;                 /* bytes/us per GPU, read + write */
+    int64_t replica_demand_bytes;    /* bytes one GPU reads per batch from rows replicated in every active
+                                        GPU's HBM (R25): a local read plus the write of the same bytes into
+                                        its batch, so it adds 2x to T_hbm and nothing to NVLink or ingest */
 } moment_plan_args;
 
 moment_status moment_plan(moment_topo_t topo, const moment_plan_args* args, moment_plan_t* out);
@@ -164,6 +182,39 @@ moment_status moment_plan(moment_topo_t topo, const moment_plan_args* args, mome
 moment_status moment_plan_info(moment_plan_t plan, int64_t* t_star, int64_t* t_ingest, int64_t* t_nvlink,
                                int64_t* t_hbm, int64_t* link_flow, int64_t* quota);
 moment_status moment_plan_free(moment_plan_t plan);
+
+/* ================================================================================================
+ * Replication search (R25): the plan's predicted per-batch time T* as a function
+ * of how many hot rows are replicated in every GPU's HBM — the paper evaluates candidate layouts by the
+ * time-bisection model instead of by running them. For each candidate r:
+ *   moment_place(topo, place with replicate_rows = r)                                   (P4 + R25)
+ *   d_b = floor(R * A'_b / demand_batches) for every bin b (its topology node), replica demand
+ *   d_rep = floor(R * A'_rep / demand_batches)   (A' = demand_counts summed over the bin's vertices: counts
+ *                                                 of appearances in F_H over demand_batches batches summed
+ *                                                 over all ranks; NULL = the placement's own hotness over
+ *                                                 hot_batches, an in-sample estimate that over-states the
+ *                                                 hit rate of the hot bins — pass held-out batches' counts)
+ *   T*(r) = moment_plan(topo, k, gpu_node, d, nvlink_cap, hbm_cap, d_rep).t_star         (P5 + R25)
+ * t_star[i] = T*(candidates[i]), or -1 if candidate i is infeasible (r above a GPU bin's capacity or
+ * n_vertices, the rest not fitting, or the plan having no finite time). Errors: EINVAL (null or negative
+ * arguments, mode not DDAK, a bin that is not a storage node). *best = the first index with the least T*, or -1 if none is feasible.
+ * ================================================================================================ */
+typedef struct {
+    const moment_place_args* place;  /* mode must be DDAK; its replicate_rows is ignored; bin_node or the
+                                        topology maps bins to storage nodes */
+    int32_t k;                       /* as moment_plan_args */
+    const int32_t* gpu_node;
+    int64_t nvlink_cap, hbm_cap;
+    int64_t row_bytes;               /* R */
+    int64_t hot_batches;             /* > 0: batches place->hotness was counted over */
+    const uint64_t* demand_counts;   /* host [n_vertices] or NULL (= place->hotness, hot_batches) */
+    int64_t demand_batches;          /* > 0 when demand_counts is given */
+    int32_t n_candidates;
+    const int64_t* candidates;       /* host [n_candidates]: replicate_rows values */
+} moment_replicate_args;
+
+moment_status moment_replicate_search(moment_topo_t topo, const moment_replicate_args* args, int64_t* t_star,
+                                      int32_t* best);
 
 /* ================================================================================================
  * Device context: one per GPU rank; owns all device workspaces (no allocation on the hot path).

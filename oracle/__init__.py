@@ -71,12 +71,14 @@ def _setup(L):
     L.orc_maxflow.restype = C.c_int
     L.orc_time_bisect.argtypes = [I32, I32, P, P, P, P, I32, I32, P, P]
     L.orc_time_bisect.restype = C.c_int
-    L.orc_plan_closed_forms.argtypes = [I32, I32, P, P, P, I64, I64, P, P]
+    L.orc_plan_closed_forms.argtypes = [I32, I32, P, P, P, I64, I64, I64, P, P]
     L.orc_plan_closed_forms.restype = C.c_int
     L.orc_bucket.argtypes = [I32, I32, I32, P, P, P, I64, P, P, P]
     L.orc_bucket.restype = C.c_int
     L.orc_ddak.argtypes = [I64, P, I32, P, P, P, I64, P, P, P, P]
     L.orc_ddak.restype = C.c_int
+    L.orc_ddak_replicate.argtypes = [I64, P, I32, P, P, P, I64, I64, P, P, P, P, P]
+    L.orc_ddak_replicate.restype = C.c_int
 
 
 def _p(a: np.ndarray):
@@ -195,13 +197,14 @@ def time_bisect(n_nodes: int, links, is_supply, s: int, t: int):
     return int(ts[0]), flow[: len(links)]
 
 
-def plan_closed_forms(k: int, hbm_owner, d, x, nvlink_cap: int, hbm_cap: int):
+def plan_closed_forms(k: int, hbm_owner, d, x, nvlink_cap: int, hbm_cap: int, replica_d: int = 0):
     own = _c(hbm_owner, np.int32)
     dd = _c(d, np.int64)
     xx = _c(x, np.int64).reshape(-1)
     tn = np.zeros(1, np.int64)
     th = np.zeros(1, np.int64)
-    st = lib().orc_plan_closed_forms(k, len(own), _p(own), _p(dd), _p(xx), nvlink_cap, hbm_cap, _p(tn), _p(th))
+    st = lib().orc_plan_closed_forms(k, len(own), _p(own), _p(dd), _p(xx), nvlink_cap, hbm_cap, replica_d, _p(tn),
+                                     _p(th))
     if st != OK:
         raise OracleError(st, "plan_closed_forms")
     return int(tn[0]), int(th[0])
@@ -237,3 +240,23 @@ def ddak(hotness, tier_rank, cap_rows, traffic, pool: int = 100):
     if st != OK:
         raise OracleError(st, "ddak")
     return bin_of[:n], slot_of[:n], A, U
+
+
+def ddak_replicate(hotness, tier_rank, cap_rows, traffic, r: int, pool: int = 100):
+    """R25: (bin_of with -2 = replica, slot_of, A, U, replica_access)."""
+    hot = _c(hotness, np.uint64)
+    tr = _c(tier_rank, np.int32)
+    cap = _c(cap_rows, np.int64)
+    traf = _c(traffic, np.int64)
+    n = len(hot)
+    nb = len(tr)
+    bin_of = np.full(max(n, 1), -1, np.int32)
+    slot_of = np.full(max(n, 1), -1, np.int64)
+    A = np.zeros(nb, np.uint64)
+    U = np.zeros(nb, np.int64)
+    rep = np.zeros(1, np.uint64)
+    st = lib().orc_ddak_replicate(n, _p(hot), nb, _p(tr), _p(cap), _p(traf), pool, r, _p(bin_of), _p(slot_of), _p(A),
+                                  _p(U), _p(rep))
+    if st != OK:
+        raise OracleError(st, "ddak_replicate")
+    return bin_of[:n], slot_of[:n], A, U, int(rep[0])

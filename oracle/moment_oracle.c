@@ -20,6 +20,7 @@
  *   orc_plan_closed_forms .... NVLink / HBM closed-form times of the ingest plan (R11)
  *   orc_bucket ............... per-request routing by placement + quota (R12)
  *   orc_ddak ................. data-distribution-aware knapsack, Eq. 2 (R13-R17)
+ *   orc_ddak_replicate ....... the same with the r hottest rows replicated in every GPU bin (R25)
  *
  * Parity status of every function is listed in DESIGN.md §4 with its pins (tests/test_oracle_*.py).
  */
@@ -379,8 +380,10 @@ int orc_time_bisect(int32_t n_nodes, int32_t n_links, const int32_t* from, const
  * in_g  = sum_{b HBM, o != g} d_b + sum_j ceil(d_j * (W_j - x[j][g]) / W_j)
  * out_h = sum_{b HBM owned by h} (k-1) d_b + sum_j ceil((k-1) * d_j * x[j][h] / W_j)
  * T_nvlink = ceil(max_g max(in_g, out_g) / nvlink_cap) (0 if no NVLink bytes);
- * T_hbm = ceil(max_g (k d_{HBM_g} + sum_b d_b) / hbm_cap)   (reads of g's HBM bin by all k GPUs plus
- *         the writes of g's own batch buffer). Each relay term is rounded up to whole bytes (R11).
+ * T_hbm = ceil(max_g (k d_{HBM_g} + sum_b d_b + 2 d_rep) / hbm_cap)   (reads of g's HBM bin by all k GPUs
+ *         plus the writes of g's own batch buffer; d_rep = bytes g reads from rows replicated in every
+ *         GPU's HBM, read locally and written into its batch, R25). Each relay term is rounded up to
+ *         whole bytes (R11).
  * Inputs are indexed by rank 0..k-1: hbm_owner[b] = owning rank, or -1 for host bins; x is [n_bins][k].
  * ------------------------------------------------------------------------------------------------ */
 static int64_t ceil_div_u128(unsigned __int128 a, unsigned __int128 b) {
@@ -388,10 +391,12 @@ static int64_t ceil_div_u128(unsigned __int128 a, unsigned __int128 b) {
 }
 
 int orc_plan_closed_forms(int32_t k, int32_t n_bins, const int32_t* hbm_owner, const int64_t* d,
-                          const int64_t* x, int64_t nvlink_cap, int64_t hbm_cap, int64_t* t_nvlink,
-                          int64_t* t_hbm) {
+                          const int64_t* x, int64_t nvlink_cap, int64_t hbm_cap, int64_t replica_d,
+                          int64_t* t_nvlink, int64_t* t_hbm) {
     int64_t max_link = 0, max_hbm = 0;
-    int64_t total_d = 0;
+    /* R25: replicated rows are read from g's own HBM and written into its batch: 2 replica_d on g's
+     * HBM, nothing on NVLink */
+    int64_t total_d = 2 * replica_d;
     for (int32_t b = 0; b < n_bins; b++) total_d += d[b];
     for (int32_t g = 0; g < k; g++) {
         int64_t in_g = 0, out_g = 0, hbm_g = total_d;
@@ -593,4 +598,56 @@ int orc_ddak(int64_t n, const uint64_t* hotness, int32_t n_bins, const int32_t* 
     }
     free(order); free(A); free(U);
     return status;
+}
+
+/* ------------------------------------------------------------------------------------------------
+ * Replication-aware DDAK (R25; an extension of Eq. 2):
+ *   order = vertices by (hotness desc, id asc)                                            (as orc_ddak)
+ *   the first r vertices of order are replicas: bin_of = -2, slot_of = position in order; each sits at
+ *     that slot in EVERY GPU-tier bin (tier_rank 0), so every GPU bin needs capacity >= r
+ *   the remaining vertices are placed by orc_ddak with GPU bins' capacities reduced by r; their slots in
+ *     GPU bins are shifted by r (the bin holds [replicas | partition])
+ * rep_access = sum of the replicas' hotness. A and U count the partition only.
+ * ------------------------------------------------------------------------------------------------ */
+int orc_ddak_replicate(int64_t n, const uint64_t* hotness, int32_t n_bins, const int32_t* tier_rank,
+                       const int64_t* cap_rows, const int64_t* traffic, int64_t pool, int64_t r, int32_t* bin_of,
+                       int64_t* slot_of, uint64_t* access_out, int64_t* used_out, uint64_t* rep_access) {
+    if (n < 0 || n_bins <= 0 || pool <= 0 || r < 0 || r > n) return ORC_EINVAL;
+    for (int32_t b = 0; b < n_bins; b++)
+        if (tier_rank[b] == 0 && cap_rows[b] < r) return ORC_EINFEASIBLE;
+    int64_t* order = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+    if (!order) return ORC_ENOMEM;
+    for (int64_t v = 0; v < n; v++) order[v] = v;
+    g_hot_for_sort = hotness;
+    qsort(order, (size_t)n, sizeof(int64_t), cmp_hot_desc);
+    char* is_rep = (char*)calloc((size_t)(n > 0 ? n : 1), 1);
+    uint64_t rep = 0;
+    for (int64_t i = 0; i < r; i++) {
+        is_rep[order[i]] = 1;
+        bin_of[order[i]] = -2;
+        slot_of[order[i]] = i;
+        rep += hotness[order[i]];
+    }
+    free(order);
+    /* the remaining vertices, in ascending id order (keeps orc_ddak's id tie-break) */
+    int64_t m = n - r;
+    int64_t* ids = (int64_t*)malloc(sizeof(int64_t) * (size_t)(m > 0 ? m : 1));
+    uint64_t* sub_hot = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)(m > 0 ? m : 1));
+    int32_t* sub_bin = (int32_t*)malloc(sizeof(int32_t) * (size_t)(m > 0 ? m : 1));
+    int64_t* sub_slot = (int64_t*)malloc(sizeof(int64_t) * (size_t)(m > 0 ? m : 1));
+    int64_t* cap2 = (int64_t*)malloc(sizeof(int64_t) * (size_t)n_bins);
+    int64_t j = 0;
+    for (int64_t v = 0; v < n; v++)
+        if (!is_rep[v]) { ids[j] = v; sub_hot[j] = hotness[v]; j++; }
+    for (int32_t b = 0; b < n_bins; b++) cap2[b] = tier_rank[b] == 0 ? cap_rows[b] - r : cap_rows[b];
+    int st = orc_ddak(m, sub_hot, n_bins, tier_rank, cap2, traffic, pool, sub_bin, sub_slot, access_out, used_out);
+    if (st == ORC_OK) {
+        for (int64_t q = 0; q < m; q++) {
+            bin_of[ids[q]] = sub_bin[q];
+            slot_of[ids[q]] = sub_slot[q] + (tier_rank[sub_bin[q]] == 0 ? r : 0);
+        }
+        if (rep_access) *rep_access = rep;
+    }
+    free(is_rep); free(ids); free(sub_hot); free(sub_bin); free(sub_slot); free(cap2);
+    return st;
 }

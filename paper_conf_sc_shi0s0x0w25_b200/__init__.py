@@ -5,3 +5,4 @@ The Python layer is argument marshalling only (`moment.py`); see DESIGN.md.
 """
 from . import moment  # noqa: F401
 from .moment import *  # noqa: F401,F403
+from . import boxes  # noqa: F401,E402

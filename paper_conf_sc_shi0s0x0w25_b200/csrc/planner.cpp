@@ -327,6 +327,7 @@ int cmp_frac(u128 p1, u128 q1, u128 p2, u128 q2) {
 
 struct Bin {
     uint64_t access = 0;  // A: cumulative hotness
+    uint64_t demand = 0;  // A': cumulative demand counts (replication search only)
     int64_t used = 0;     // U: rows placed
     int64_t cap = 0;      // C
     int64_t traffic = 0;  // T
@@ -404,17 +405,13 @@ uint64_t mix64(uint64_t x) {
     return x ^ (x >> 31);
 }
 
-}  // namespace
-
-extern "C" moment_status moment_place(moment_topo_t T, const moment_place_args* a, moment_place_out* o) {
-    if (!a || !o || !o->bin_of || !o->slot_of) return fail(MOMENT_EINVAL, "moment_place: null argument");
-    const int64_t n = a->n_vertices;
+// Bins of a placement call: node, tier rank, capacity and Bin_traffic resolved from args/topology.
+moment_status resolve_bins(moment_topo_t T, const moment_place_args* a, std::vector<Bin>& bins,
+                           std::vector<int32_t>& bin_node) {
     const int32_t nb = a->n_bins;
-    if (n < 0 || n >= (int64_t(1) << 32)) return fail(MOMENT_EINVAL, "moment_place: n_vertices %lld out of range", (long long)n);
     if (nb <= 0 || nb > MOMENT_MAX_BINS) return fail(MOMENT_EINVAL, "moment_place: n_bins %d out of range", nb);
-    if (n > 0 && !a->hotness && a->mode == MOMENT_PLACE_DDAK) return fail(MOMENT_EINVAL, "moment_place: hotness is null");
     if (!a->bin_capacity_rows) return fail(MOMENT_EINVAL, "moment_place: bin_capacity_rows is null");
-    std::vector<int32_t> bin_node(nb, -1);
+    bin_node.assign(nb, -1);
     if (a->bin_node) {
         for (int b = 0; b < nb; b++) bin_node[b] = a->bin_node[b];
     } else if (T) {
@@ -423,7 +420,7 @@ extern "C" moment_status moment_place(moment_topo_t T, const moment_place_args* 
             if (T->nodes[v].kind == MOMENT_NODE_STORAGE) bin_node[b++] = v;
         if (b != nb) return fail(MOMENT_EINVAL, "moment_place: topology has %d storage nodes, n_bins = %d", b, nb);
     }
-    std::vector<Bin> bins(nb);
+    bins.assign(nb, Bin{});
     std::vector<int64_t> traffic(nb, 0);
     if (a->bin_traffic) {
         for (int b = 0; b < nb; b++) traffic[b] = a->bin_traffic[b];
@@ -451,11 +448,90 @@ extern "C" moment_status moment_place(moment_topo_t T, const moment_place_args* 
         bins[b].cap = a->bin_capacity_rows[b];
         bins[b].traffic = traffic[b];
     }
-    int64_t total_cap = 0;
-    for (auto& b : bins) total_cap += b.cap;
-    if (total_cap < n) return fail(MOMENT_EINFEASIBLE, "moment_place: capacity %lld rows < %lld vertices", (long long)total_cap, (long long)n);
+    return MOMENT_OK;
+}
 
+// DDAK over `order` (hotness desc, id asc) with the first r vertices replicated in every GPU bin (R25;
+// r = 0: plain DDAK, R13-R17). bin_of/slot_of may be null (the search needs only A, U per bin).
+moment_status ddak_core(int64_t n, const uint64_t* hot, const std::vector<uint32_t>& order, int64_t r, int64_t pool,
+                        std::vector<Bin>& bins, uint64_t* replica_access, int32_t* bin_of, int64_t* slot_of,
+                        const uint64_t* dem = nullptr, uint64_t* replica_demand = nullptr) {
+    const int nb = (int)bins.size();
+    if (r < 0 || r > n) return fail(MOMENT_EINVAL, "moment_place: replicate_rows %lld out of [0, %lld]", (long long)r, (long long)n);
+    std::vector<int64_t> slot0(nb, 0);
+    int64_t total_cap = 0;
+    for (int b = 0; b < nb; b++) {
+        if (r > 0 && bins[b].rank == MOMENT_TIER_GPU_HBM - 1) {
+            if (bins[b].cap < r)
+                return fail(MOMENT_EINFEASIBLE, "moment_place: replicate_rows %lld exceeds GPU bin %d capacity %lld",
+                            (long long)r, b, (long long)bins[b].cap);
+            bins[b].cap -= r;  // Eq. 2 runs on the residual capacity; the partition's slots start at r
+            slot0[b] = r;
+        }
+        total_cap += bins[b].cap;
+    }
+    if (total_cap < n - r)
+        return fail(MOMENT_EINFEASIBLE, "moment_place: capacity %lld rows < %lld vertices", (long long)total_cap, (long long)(n - r));
+    uint64_t rep = 0, rep_dem = 0;
+    for (int64_t i = 0; i < r; i++) {
+        const uint32_t v = order[i];
+        if (bin_of) { bin_of[v] = MOMENT_BIN_REPLICA; slot_of[v] = i; }
+        rep += hot[v];
+        if (dem) rep_dem += dem[v];
+    }
+    if (replica_access) *replica_access = rep;
+    if (replica_demand) *replica_demand = rep_dem;
+    for (int64_t g0 = r; g0 < n; g0 += pool) {
+        int64_t next = g0, g1 = std::min(n, g0 + pool);
+        while (next < g1) {
+            int best_rank = std::numeric_limits<int>::max();
+            for (auto& b : bins)
+                if (b.used < b.cap && b.traffic > 0) best_rank = std::min(best_rank, b.rank);
+            int pick = -1;
+            for (int b = 0; b < nb; b++) {
+                const Bin& B = bins[b];
+                if (B.used >= B.cap) continue;
+                if (best_rank != std::numeric_limits<int>::max() && B.rank != best_rank) continue;
+                if (pick < 0) { pick = b; continue; }
+                int c = priority_cmp(B, bins[pick]);
+                if (c < 0 || (c == 0 && B.rank < bins[pick].rank)) pick = b;
+            }
+            if (pick < 0) return fail(MOMENT_EINFEASIBLE, "moment_place: no bin has room");
+            Bin& B = bins[pick];
+            int64_t m = std::min(g1 - next, B.cap - B.used);
+            uint64_t acc = 0, dacc = 0;
+            for (int64_t q = 0; q < m; q++) {
+                uint32_t v = order[next + q];
+                if (bin_of) { bin_of[v] = pick; slot_of[v] = slot0[pick] + B.used + q; }
+                acc += hot[v];
+                if (dem) dacc += dem[v];
+            }
+            B.access += acc;
+            B.demand += dacc;
+            B.used += m;
+            next += m;
+        }
+    }
+    return MOMENT_OK;
+}
+
+}  // namespace
+
+extern "C" moment_status moment_place(moment_topo_t T, const moment_place_args* a, moment_place_out* o) {
+    if (!a || !o || !o->bin_of || !o->slot_of) return fail(MOMENT_EINVAL, "moment_place: null argument");
+    const int64_t n = a->n_vertices;
+    const int32_t nb = a->n_bins;
+    if (n < 0 || n >= (int64_t(1) << 32)) return fail(MOMENT_EINVAL, "moment_place: n_vertices %lld out of range", (long long)n);
+    if (n > 0 && !a->hotness && a->mode == MOMENT_PLACE_DDAK) return fail(MOMENT_EINVAL, "moment_place: hotness is null");
+    std::vector<Bin> bins;
+    std::vector<int32_t> bin_node;
+    MOMENT_TRY(resolve_bins(T, a, bins, bin_node));
+    if (o->replica_access) *o->replica_access = 0;
     if (a->mode == MOMENT_PLACE_HASH) {
+        if (a->replicate_rows != 0) return fail(MOMENT_EINVAL, "moment_place: replicate_rows needs DDAK mode");
+        int64_t total_cap = 0;
+        for (auto& b : bins) total_cap += b.cap;
+        if (total_cap < n) return fail(MOMENT_EINFEASIBLE, "moment_place: capacity %lld rows < %lld vertices", (long long)total_cap, (long long)n);
         // Uniform baseline ("hash-based partitioning"): bin = hash(v) mod n_bins, next non-full
         // bin on overflow; slots in id order.
         for (int64_t v = 0; v < n; v++) {
@@ -469,34 +545,8 @@ extern "C" moment_status moment_place(moment_topo_t T, const moment_place_args* 
         std::vector<uint32_t> order;
         order_by_hotness(n, a->hotness, order);
         const int64_t pool = a->pool > 0 ? a->pool : 100;
-        for (int64_t g0 = 0; g0 < n; g0 += pool) {
-            int64_t next = g0, g1 = std::min(n, g0 + pool);
-            while (next < g1) {
-                int best_rank = std::numeric_limits<int>::max();
-                for (auto& b : bins)
-                    if (b.used < b.cap && b.traffic > 0) best_rank = std::min(best_rank, b.rank);
-                int pick = -1;
-                for (int b = 0; b < nb; b++) {
-                    const Bin& B = bins[b];
-                    if (B.used >= B.cap) continue;
-                    if (best_rank != std::numeric_limits<int>::max() && B.rank != best_rank) continue;
-                    if (pick < 0) { pick = b; continue; }
-                    int c = priority_cmp(B, bins[pick]);
-                    if (c < 0 || (c == 0 && B.rank < bins[pick].rank)) pick = b;
-                }
-                if (pick < 0) return fail(MOMENT_EINFEASIBLE, "moment_place: no bin has room");
-                Bin& B = bins[pick];
-                int64_t m = std::min(g1 - next, B.cap - B.used);
-                for (int64_t q = 0; q < m; q++) {
-                    uint32_t v = order[next + q];
-                    o->bin_of[v] = pick;
-                    o->slot_of[v] = B.used + q;
-                    B.access += a->hotness[v];
-                }
-                B.used += m;
-                next += m;
-            }
-        }
+        MOMENT_TRY(ddak_core(n, a->hotness, order, a->replicate_rows, pool, bins, o->replica_access, o->bin_of,
+                             o->slot_of));
     } else {
         return fail(MOMENT_EINVAL, "moment_place: unknown mode %d", a->mode);
     }
@@ -504,6 +554,21 @@ extern "C" moment_status moment_place(moment_topo_t T, const moment_place_args* 
         if (o->bin_access) o->bin_access[b] = bins[b].access;
         if (o->bin_rows_used) o->bin_rows_used[b] = bins[b].used;
         if (o->bin_traffic_used) o->bin_traffic_used[b] = bins[b].traffic;
+    }
+    return MOMENT_OK;
+}
+
+extern "C" moment_status moment_place_pack_rank(int64_t n, const int32_t* bin_of, const int64_t* slot_of,
+                                               int32_t replica_bin, uint64_t* packed) {
+    if (n < 0 || (n > 0 && (!bin_of || !slot_of || !packed))) return fail(MOMENT_EINVAL, "moment_place_pack_rank: null argument");
+    if (replica_bin < 0 || replica_bin >= MOMENT_MAX_BINS)
+        return fail(MOMENT_EINVAL, "moment_place_pack_rank: replica_bin %d out of range", replica_bin);
+    for (int64_t v = 0; v < n; v++) {
+        const int32_t b = bin_of[v] == MOMENT_BIN_REPLICA ? replica_bin : bin_of[v];
+        if (b < 0 || b >= MOMENT_MAX_BINS || slot_of[v] < 0 || slot_of[v] >= (int64_t(1) << 40))
+            return fail(MOMENT_EINVAL, "moment_place_pack_rank: vertex %lld has bin %d slot %lld out of range", (long long)v,
+                        bin_of[v], (long long)slot_of[v]);
+        packed[v] = ((uint64_t)b << 40) | (uint64_t)slot_of[v];
     }
     return MOMENT_OK;
 }
@@ -680,7 +745,10 @@ extern "C" moment_status moment_plan(moment_topo_t T, const moment_plan_args* a,
         }
     }
     // Closed forms (R11).
-    int64_t total_d = 0;
+    if (a->replica_demand_bytes < 0) { delete P; return fail(MOMENT_EINVAL, "moment_plan: negative replica demand"); }
+    // every GPU writes its whole batch: partitioned demand + the replicated rows, which it also reads
+    // from its own HBM (R25)
+    int64_t total_d = 2 * a->replica_demand_bytes;
     for (int b = 0; b < N; b++)
         if (T->nodes[b].kind == MOMENT_NODE_STORAGE) total_d += a->bin_demand_bytes[b];
     int64_t max_link = 0, max_hbm = 0;
@@ -719,6 +787,63 @@ extern "C" moment_status moment_plan(moment_topo_t T, const moment_plan_args* a,
     return MOMENT_OK;
 }
 
+extern "C" moment_status moment_replicate_search(moment_topo_t T, const moment_replicate_args* a, int64_t* t_star,
+                                                int32_t* best) {
+    if (!T || !a || !a->place || !t_star || !best || (a->n_candidates > 0 && !a->candidates))
+        return fail(MOMENT_EINVAL, "moment_replicate_search: null argument");
+    const moment_place_args* pa = a->place;
+    const int64_t n = pa->n_vertices;
+    if (pa->mode != MOMENT_PLACE_DDAK) return fail(MOMENT_EINVAL, "moment_replicate_search: place mode must be DDAK");
+    if (n < 0 || n >= (int64_t(1) << 32)) return fail(MOMENT_EINVAL, "moment_replicate_search: n_vertices out of range");
+    if (n > 0 && !pa->hotness) return fail(MOMENT_EINVAL, "moment_replicate_search: hotness is null");
+    if (a->row_bytes <= 0 || a->hot_batches <= 0 || a->n_candidates < 0 || (a->demand_counts && a->demand_batches <= 0))
+        return fail(MOMENT_EINVAL, "moment_replicate_search: row_bytes, hot_batches, demand_batches must be > 0");
+    const uint64_t* dem = a->demand_counts ? a->demand_counts : pa->hotness;
+    const int64_t dem_batches = a->demand_counts ? a->demand_batches : a->hot_batches;
+    std::vector<Bin> bins0;
+    std::vector<int32_t> bin_node;
+    MOMENT_TRY(resolve_bins(T, pa, bins0, bin_node));
+    const int N = (int)T->nodes.size();
+    for (size_t b = 0; b < bin_node.size(); b++)
+        if (bin_node[b] < 0 || bin_node[b] >= N || T->nodes[bin_node[b]].kind != MOMENT_NODE_STORAGE)
+            return fail(MOMENT_EINVAL, "moment_replicate_search: bin %zu is not a storage node", b);
+    std::vector<uint32_t> order;
+    order_by_hotness(n, pa->hotness, order);
+    const int64_t pool = pa->pool > 0 ? pa->pool : 100;
+    *best = -1;
+    auto demand = [&](uint64_t acc) -> int64_t {
+        return (int64_t)(((u128)acc * (u128)(uint64_t)a->row_bytes) / (u128)(uint64_t)dem_batches);
+    };
+    for (int32_t i = 0; i < a->n_candidates; i++) {
+        t_star[i] = -1;
+        if (a->candidates[i] < 0) return fail(MOMENT_EINVAL, "moment_replicate_search: candidate %d is negative", i);
+        if (a->candidates[i] > n) continue;  // more replicas than vertices: infeasible
+        std::vector<Bin> bins = bins0;
+        uint64_t rep = 0;
+        moment_status st = ddak_core(n, pa->hotness, order, a->candidates[i], pool, bins, nullptr, nullptr, nullptr,
+                                     dem, &rep);
+        if (st == MOMENT_EINFEASIBLE) continue;
+        if (st != MOMENT_OK) return st;
+        std::vector<int64_t> d(N, 0);
+        for (size_t b = 0; b < bins.size(); b++) d[bin_node[b]] += demand(bins[b].demand);
+        moment_plan_args pl{};
+        pl.k = a->k;
+        pl.gpu_node = a->gpu_node;
+        pl.bin_demand_bytes = d.data();
+        pl.nvlink_cap = a->nvlink_cap;
+        pl.hbm_cap = a->hbm_cap;
+        pl.replica_demand_bytes = demand(rep);
+        moment_plan_t P = nullptr;
+        st = moment_plan(T, &pl, &P);
+        if (st == MOMENT_EINFEASIBLE) continue;
+        if (st != MOMENT_OK) return st;
+        t_star[i] = P->t_star;
+        moment_plan_free(P);
+        if (*best < 0 || t_star[i] < t_star[*best]) *best = i;
+    }
+    return MOMENT_OK;
+}
+
 extern "C" moment_status moment_plan_info(moment_plan_t P, int64_t* t_star, int64_t* t_ingest, int64_t* t_nvlink,
                                           int64_t* t_hbm, int64_t* link_flow, int64_t* quota) {
     if (!P) return fail(MOMENT_EINVAL, "moment_plan_info: null plan");
@@ -737,4 +862,4 @@ extern "C" moment_status moment_plan_free(moment_plan_t P) {
 }
 
 extern "C" const char* moment_last_error(void) { return moment::last_error(); }
-extern "C" int32_t moment_version(void) { return (0 << 16) | 1; }
+extern "C" int32_t moment_version(void) { return (0 << 16) | 2; }

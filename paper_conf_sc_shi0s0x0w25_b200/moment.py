@@ -20,13 +20,14 @@ CAP_INF = np.iinfo(np.int64).max
 NODE_SOURCE, NODE_SINK, NODE_STORAGE, NODE_INTERCONNECT, NODE_COMPUTE = range(5)
 TIER_NONE, TIER_GPU_HBM, TIER_HOST_DRAM, TIER_SSD = range(4)
 PLACE_DDAK, PLACE_HASH = 0, 1
+BIN_REPLICA = -2
 SAMPLE_REPLACE, SAMPLE_CHECK = 1, 2
 MAX_BINS = 64
 
 EXPORTED = [
     "moment_last_error", "moment_version", "moment_topology", "moment_topology_info", "moment_topology_export",
-    "moment_topology_free", "moment_maxflow", "moment_place", "moment_place_pack", "moment_plan", "moment_plan_info",
-    "moment_plan_free", "moment_ctx_create", "moment_ctx_free", "moment_ctx_workspace_bytes", "moment_sample_bounds",
+    "moment_topology_free", "moment_maxflow", "moment_place", "moment_place_pack", "moment_place_pack_rank", "moment_plan",
+    "moment_plan_info", "moment_plan_free", "moment_replicate_search", "moment_ctx_create", "moment_ctx_free", "moment_ctx_workspace_bytes", "moment_sample_bounds",
     "moment_sample", "moment_sample_check", "moment_hotness", "moment_bucket", "moment_gather", "moment_gather_group",
     "moment_step", "moment_step_host", "moment_gather_routed", "moment_relay_pack", "moment_relay_serve",
     "moment_relay_scatter", "moment_relay_push", "moment_relay_serve_push", "moment_ipc_export", "moment_ipc_import",
@@ -52,17 +53,24 @@ class Link(C.Structure):
 class PlaceArgs(C.Structure):
     _fields_ = [("n_vertices", C.c_int64), ("hotness", C.c_void_p), ("n_bins", C.c_int32), ("bin_node", C.c_void_p),
                 ("bin_tier", C.c_void_p), ("bin_capacity_rows", C.c_void_p), ("bin_traffic", C.c_void_p),
-                ("pool", C.c_int64), ("mode", C.c_int32)]
+                ("pool", C.c_int64), ("mode", C.c_int32), ("replicate_rows", C.c_int64)]
 
 
 class PlaceOut(C.Structure):
     _fields_ = [("bin_of", C.c_void_p), ("slot_of", C.c_void_p), ("bin_access", C.c_void_p),
-                ("bin_rows_used", C.c_void_p), ("bin_traffic_used", C.c_void_p)]
+                ("bin_rows_used", C.c_void_p), ("bin_traffic_used", C.c_void_p), ("replica_access", C.c_void_p)]
 
 
 class PlanArgs(C.Structure):
     _fields_ = [("k", C.c_int32), ("gpu_node", C.c_void_p), ("bin_demand_bytes", C.c_void_p),
-                ("nvlink_cap", C.c_int64), ("hbm_cap", C.c_int64)]
+                ("nvlink_cap", C.c_int64), ("hbm_cap", C.c_int64), ("replica_demand_bytes", C.c_int64)]
+
+
+class ReplicateArgs(C.Structure):
+    _fields_ = [("place", C.c_void_p), ("k", C.c_int32), ("gpu_node", C.c_void_p), ("nvlink_cap", C.c_int64),
+                ("hbm_cap", C.c_int64), ("row_bytes", C.c_int64), ("hot_batches", C.c_int64),
+                ("demand_counts", C.c_void_p), ("demand_batches", C.c_int64),
+                ("n_candidates", C.c_int32), ("candidates", C.c_void_p)]
 
 
 class CtxArgs(C.Structure):
@@ -107,6 +115,8 @@ def lib():
             "moment_maxflow": ([P, P, P], I32),
             "moment_place": ([P, P, P], I32),
             "moment_place_pack": ([I64, P, P, P], I32),
+            "moment_place_pack_rank": ([I64, P, P, I32, P], I32),
+            "moment_replicate_search": ([P, P, P, P], I32),
             "moment_plan": ([P, P, P], I32),
             "moment_plan_info": ([P, P, P, P, P, P, P], I32),
             "moment_plan_free": ([P], I32),
@@ -212,9 +222,10 @@ def topology(nodes, links) -> Topology:
 
 # ---------------------------------------------------------------------------------------------- P4
 def place(topo: Topology | None, hotness, capacity_rows, *, bin_node=None, bin_tier=None, bin_traffic=None,
-          pool: int = 100, mode: int = PLACE_DDAK):
+          pool: int = 100, mode: int = PLACE_DDAK, replicate_rows: int = 0, return_replica_access: bool = False):
     """DDAK placement. Returns (bin_of int32[n], slot_of int64[n], access uint64[nb], used int64[nb],
-    traffic int64[nb])."""
+    traffic int64[nb]) [+ replica_access]. replicate_rows > 0: the hottest rows are copied into every GPU bin
+    (bin_of = BIN_REPLICA, R25)."""
     hot = _np(hotness, np.uint64)
     cap = _np(capacity_rows, np.int64)
     nb = len(cap)
@@ -229,14 +240,18 @@ def place(topo: Topology | None, hotness, capacity_rows, *, bin_node=None, bin_t
         return arr.ctypes.data
 
     args = PlaceArgs(n, hot.ctypes.data, nb, opt(bin_node, np.int32), opt(bin_tier, np.int32), cap.ctypes.data,
-                     opt(bin_traffic, np.int64), pool, mode)
+                     opt(bin_traffic, np.int64), pool, mode, replicate_rows)
     bin_of = np.zeros(max(n, 1), np.int32)
     slot_of = np.zeros(max(n, 1), np.int64)
     acc = np.zeros(nb, np.uint64)
     used = np.zeros(nb, np.int64)
     traf = np.zeros(nb, np.int64)
-    out = PlaceOut(bin_of.ctypes.data, slot_of.ctypes.data, acc.ctypes.data, used.ctypes.data, traf.ctypes.data)
+    rep = np.zeros(1, np.uint64)
+    out = PlaceOut(bin_of.ctypes.data, slot_of.ctypes.data, acc.ctypes.data, used.ctypes.data, traf.ctypes.data,
+                   rep.ctypes.data)
     _check(lib().moment_place(topo.handle if topo is not None else None, C.byref(args), C.byref(out)))
+    if return_replica_access:
+        return bin_of[:n], slot_of[:n], acc, used, traf, int(rep[0])
     return bin_of[:n], slot_of[:n], acc, used, traf
 
 
@@ -248,16 +263,25 @@ def place_pack(bin_of, slot_of) -> np.ndarray:
     return out[: len(b)]
 
 
+def place_pack_rank(bin_of, slot_of, replica_bin: int) -> np.ndarray:
+    """One rank's device map: replicated vertices point at that rank's own HBM bin `replica_bin`."""
+    b = _np(bin_of, np.int32)
+    s = _np(slot_of, np.int64)
+    out = np.zeros(max(len(b), 1), np.uint64)
+    _check(lib().moment_place_pack_rank(len(b), b.ctypes.data, s.ctypes.data, replica_bin, out.ctypes.data))
+    return out[: len(b)]
+
+
 # ---------------------------------------------------------------------------------------------- P5
 class Plan:
-    def __init__(self, topo: Topology, gpu_node, demand_bytes, nvlink_cap: int, hbm_cap: int):
+    def __init__(self, topo: Topology, gpu_node, demand_bytes, nvlink_cap: int, hbm_cap: int, replica_demand: int = 0):
         g = _np(gpu_node, np.int32)
         d = _np(demand_bytes, np.int64)
         n, m, _, _ = topo.info()
         if len(d) != n:
             raise MomentError(EINVAL, f"demand has {len(d)} entries, topology has {n} nodes")
         self.k, self.n_nodes, self.n_links = len(g), n, m
-        args = PlanArgs(len(g), g.ctypes.data, d.ctypes.data, nvlink_cap, hbm_cap)
+        args = PlanArgs(len(g), g.ctypes.data, d.ctypes.data, nvlink_cap, hbm_cap, replica_demand)
         h = C.c_void_p()
         _check(lib().moment_plan(topo.handle, C.byref(args), C.byref(h)))
         self.handle = h
@@ -277,8 +301,38 @@ class Plan:
                 "link_flow": flow[: self.n_links], "quota": quota.reshape(self.n_nodes, self.k)}
 
 
-def plan(topo, gpu_node, demand_bytes, nvlink_cap, hbm_cap) -> Plan:
-    return Plan(topo, gpu_node, demand_bytes, nvlink_cap, hbm_cap)
+def plan(topo, gpu_node, demand_bytes, nvlink_cap, hbm_cap, replica_demand: int = 0) -> Plan:
+    return Plan(topo, gpu_node, demand_bytes, nvlink_cap, hbm_cap, replica_demand)
+
+
+def replicate_search(topo: Topology, hotness, capacity_rows, candidates, *, gpu_node, nvlink_cap: int, hbm_cap: int,
+                     row_bytes: int, hot_batches: int, bin_node=None, bin_tier=None, bin_traffic=None, pool: int = 100,
+                     demand_counts=None, demand_batches: int = 0):
+    """T*(r) of the plan for every candidate replicate_rows r (R25). Returns (t_star int64[n_cand] with -1 =
+    infeasible, best index or -1). demand_counts / demand_batches: held-out F_H counts for the per-bin demand
+    (default: the placement's own hotness)."""
+    hot = _np(hotness, np.uint64)
+    cap = _np(capacity_rows, np.int64)
+    keep = []
+
+    def opt(a, dt):
+        if a is None:
+            return None
+        arr = _np(a, dt)
+        keep.append(arr)
+        return arr.ctypes.data
+
+    pa = PlaceArgs(len(hot), hot.ctypes.data, len(cap), opt(bin_node, np.int32), opt(bin_tier, np.int32),
+                   cap.ctypes.data, opt(bin_traffic, np.int64), pool, PLACE_DDAK, 0)
+    g = _np(gpu_node, np.int32)
+    cand = _np(candidates, np.int64)
+    ts = np.zeros(max(len(cand), 1), np.int64)
+    best = C.c_int32()
+    dem = opt(demand_counts, np.uint64)
+    args = ReplicateArgs(C.addressof(pa), len(g), g.ctypes.data, nvlink_cap, hbm_cap, row_bytes, hot_batches,
+                         dem, demand_batches, len(cand), cand.ctypes.data)
+    _check(lib().moment_replicate_search(topo.handle, C.byref(args), ts.ctypes.data, C.byref(best)))
+    return ts[: len(cand)], best.value
 
 
 # ---------------------------------------------------------------------------------------------- ctx

@@ -478,3 +478,75 @@ def test_full_size_tiered_gather(orc, name, cache_gib):
         assert 0.0 < frac_hbm < 1.0  # both tiers exercised
     del hbm, ring, g, rows
     torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_gather_replicated_hot_rows_per_rank_maps(orc, c1, world):
+    """R25: the hottest rows replicated in every rank's HBM bin, the rest DDAK-partitioned over the HBM bins
+    and a pinned host bin. Each rank's device map (moment_place_pack_rank) points replicas at its OWN bin:
+    byte-exact rows, replicas routed to the local queue, and the replica regions of every other bin
+    poisoned while a rank gathers (a replica read from a peer bin would show)."""
+    cfg, g = c1
+    n = g.n
+    table = W.feature_table(n, 32, torch.float32, device=DEV)  # 128-byte rows
+    R = table.shape[1]
+    rng = np.random.default_rng(7 + world)
+    hot = (rng.pareto(0.9, n) * 4).astype(np.uint64)
+    r = n // 16
+    owners = list(range(world)) + [-1]
+    tiers = [M.TIER_GPU_HBM] * world + [M.TIER_HOST_DRAM]
+    caps = [r + n // (4 * world)] * world + [n]
+    bin_of, slot_of, A, U, T = M.place(None, hot, caps, bin_tier=tiers, bin_traffic=[100] * world + [10],
+                                       replicate_rows=r)
+    ob, os_, *_ = orc.ddak_replicate(hot, np.array(tiers) - 1, caps, [100] * world + [10], r, 100)
+    assert np.array_equal(bin_of, ob) and np.array_equal(slot_of, os_)
+    t_cpu = table.cpu()
+    rep = np.where(bin_of == M.BIN_REPLICA)[0]
+    bins = []
+    for b in range(world + 1):
+        sel = np.where(bin_of == b)[0]
+        rows = r + int(U[b]) if b < world else max(1, int(U[b]))
+        buf = torch.zeros((rows, R), dtype=torch.uint8)
+        buf[torch.as_tensor(slot_of[sel])] = t_cpu[torch.as_tensor(sel)]
+        if b < world:
+            buf[torch.as_tensor(slot_of[rep])] = t_cpu[torch.as_tensor(rep)]
+            bins.append(buf.to(DEV))
+        else:
+            bins.append(buf.pin_memory())
+    train = W.training_set(g, min_count=1024 * world)
+    tab = table.cpu().numpy()
+    n_rep_seen = 0
+    for rank in range(world):
+        placement = torch.as_tensor(M.place_pack_rank(bin_of, slot_of, rank).view(np.int64), device=DEV)
+        ctx = M.Ctx(n_vertices=n, max_seeds=1024, max_fanout=[10, 5], rank=rank, world=world, device=0,
+                    row_bytes=R, bin_owner=owners, bin_ptr=[b.data_ptr() for b in bins], placement=placement)
+        seeds = W.epoch_batches(train, 1024, 0, rank=rank, world=world)[0]
+        bufs = M.SampleBuffers.allocate(1024, [10, 5], n, DEV)
+        ctx.sample(g.indptr, g.indices, seeds, [10, 5], 90 + rank, bufs)
+        nF = int(bufs.counts[2])
+        ids = bufs.nodes[:nF].clone()
+        ids_np = ids.cpu().numpy()
+        # routing: replicas to this rank's own bin queue, everything else as the oracle routes it
+        route = torch.empty(nF, dtype=torch.int32, device=DEV)
+        qoff = torch.empty((world + 1) * world + 1, dtype=torch.int64, device=DEV)
+        qpos = torch.empty(nF, dtype=torch.int64, device=DEV)
+        ctx.bucket(ids, route, qoff, qpos)
+        eff_bin = np.where(bin_of[ids_np] == M.BIN_REPLICA, rank, bin_of[ids_np])
+        o_route, o_qoff, o_qpos = orc.bucket(rank, world, owners, np.zeros((world + 1, world), np.int64), eff_bin)
+        assert np.array_equal(route.cpu().numpy(), o_route)
+        is_rep = bin_of[ids_np] == M.BIN_REPLICA
+        n_rep_seen += int(is_rep.sum())
+        assert (route.cpu().numpy()[is_rep] == rank * world + rank).all()
+        # poison the replica region of every other rank's bin
+        for b in range(world):
+            if b != rank:
+                bins[b][:r].fill_(0xAB)
+        out = torch.zeros((nF, R), dtype=torch.uint8, device=DEV)
+        ctx.gather(ids, out)
+        torch.cuda.synchronize()
+        assert np.array_equal(out.cpu().numpy(), orc.gather(tab, ids_np)), rank
+        for b in range(world):
+            if b != rank:
+                bins[b][:r] = t_cpu[torch.as_tensor(rep)].to(DEV)[torch.as_tensor(np.argsort(slot_of[rep]))]
+        del ctx
+    assert n_rep_seen > 0

@@ -330,3 +330,77 @@ def test_ddak_single_bin_and_pool_semantics(orc):
     bin_of, _, _, U = orc.ddak(hot, [0, 1], [2, 10], [1, 100], 1)
     assert list(U) == [2, 4]
     assert set(np.where(bin_of == 0)[0].tolist()) == {1, 3}
+
+
+# ------------------------------------------------------------------------------------------------
+# Replication-aware DDAK (R25) and the replica term of the closed forms
+# ------------------------------------------------------------------------------------------------
+def hot_order(hot):
+    """(hotness desc, id asc) — written out independently of the oracle's qsort comparator."""
+    return sorted(range(len(hot)), key=lambda v: (-int(hot[v]), v))
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_ddak_replicate_exhaustive_small(orc, seed):
+    rng = np.random.default_rng(100 + seed)
+    nv = int(rng.integers(1, 8))
+    nb = int(rng.integers(1, 4))
+    hot = rng.integers(0, 20, nv)
+    tier = sorted(rng.integers(0, 2, nb).tolist())
+    caps = rng.integers(0, nv + 1, nb)
+    traffic = rng.integers(0, 10, nb)
+    gpu = [b for b in range(nb) if tier[b] == 0]
+    for r in range(0, nv + 1):
+        if any(caps[b] < r for b in gpu):
+            with pytest.raises(orc.OracleError) as e:
+                orc.ddak_replicate(hot, tier, caps, traffic, r, 1)
+            assert e.value.status == orc.EINFEASIBLE
+            continue
+        red = [int(caps[b]) - (r if tier[b] == 0 else 0) for b in range(nb)]
+        if sum(red) < nv - r:
+            continue
+        for pool in (1, 3):
+            bin_of, slot_of, A, U, rep = orc.ddak_replicate(hot, tier, caps, traffic, r, pool)
+            top = hot_order(hot)[:r]
+            # replicas: exactly the r first vertices of the order, slot = position in the order
+            assert sorted(np.where(bin_of == -2)[0].tolist()) == sorted(top)
+            assert [int(slot_of[v]) for v in top] == list(range(r))
+            assert rep == int(sum(int(hot[v]) for v in top))
+            # the rest: a feasible assignment under the reduced capacities (brute force), slots after the
+            # replica region in GPU bins, dense from 0 in the others
+            rest = [v for v in range(nv) if v not in top]
+            sols = set(brute_ddak_feasible([hot[v] for v in rest], red))
+            assert tuple(int(bin_of[v]) for v in rest) in sols
+            for b in range(nb):
+                mine = [v for v in rest if bin_of[v] == b]
+                base = r if tier[b] == 0 else 0
+                assert U[b] == len(mine) <= red[b]
+                assert sorted(int(slot_of[v]) for v in mine) == list(range(base, base + len(mine)))
+                assert A[b] == sum(int(hot[v]) for v in mine)
+            # r = 0 is plain DDAK
+            if r == 0:
+                b0, s0, A0, U0 = orc.ddak(hot, tier, caps, traffic, pool)
+                assert np.array_equal(b0, bin_of) and np.array_equal(s0, slot_of)
+
+
+def test_ddak_replicate_closed_form_split(orc):
+    # uniform hotness, GPU bins with traffic (4, 1) and ample capacity: after the r replicas the
+    # partition still splits 2:1 (the closed form of test_ddak_closed_form_ratio on n - r vertices)
+    n, r = 3300, 300
+    bin_of, slot_of, A, U, rep = orc.ddak_replicate(np.ones(n, np.uint64), [0, 0], [10**6, 10**6], [4, 1], r, 1)
+    assert rep == r and U.sum() == n - r
+    assert abs(U[0] - 2 * U[1]) <= 2
+    # replicas are the r lowest ids (all hotness equal: id order)
+    assert np.array_equal(np.where(bin_of == -2)[0], np.arange(r))
+
+
+def test_plan_closed_forms_replica_hand_worked(orc):
+    # the k = 2 example of test_plan_closed_forms_hand_worked plus d_rep = 50 bytes per GPU from replicas:
+    # NVLink unchanged (19); HBM GPU0 = 2*100 + (200 + 2*50) = 500 -> ceil(500/9) = 56
+    own = [0, 1, -1]
+    d = [100, 60, 40]
+    x = [[0, 0], [0, 0], [30, 10]]
+    assert orc.plan_closed_forms(2, own, d, x, 7, 9, 50) == (19, 56)
+    # everything replicated (d_b = 0, k = 8): no NVLink bytes, T_hbm = ceil(2 d_rep / hbm)
+    assert orc.plan_closed_forms(8, list(range(8)), [0] * 8, [[0] * 8] * 8, 900, 6500, 1000) == (0, 1)
+    assert orc.plan_closed_forms(8, list(range(8)), [0] * 8, [[0] * 8] * 8, 0, 6500, 6500) == (0, 2)

@@ -294,3 +294,149 @@ def test_plan_infeasible_and_zero():
     d[:] = 0
     info = M.plan(topo, [3], d, 0, 100).info()
     assert info["t_ingest"] == 0 and info["t_star"] == 0
+
+
+# ------------------------------------------------------------------------------------------------
+# Replication-aware placement and search (R25)
+# ------------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("seed", range(16))
+def test_ddak_replicate_bit_exact_vs_oracle(orc, seed):
+    rng = np.random.default_rng(1000 + seed)
+    n = int(rng.integers(1, 4000))
+    n_gpu = int(rng.integers(1, 5))
+    n_host = int(rng.integers(0, 3))
+    nb = n_gpu + n_host
+    hot = (rng.pareto(1.1, n) * 10).astype(np.uint64)
+    if seed % 3 == 0:
+        hot[:] = rng.integers(0, 3, n)  # many ties
+    tier = np.array([1] * n_gpu + [2] * n_host, np.int32)
+    caps = rng.integers(n // 8, n // 2 + 2, nb).astype(np.int64)
+    r_max = int(caps[:n_gpu].min())
+    for r in sorted({0, 1, r_max // 2, r_max}):
+        need = n - r - int((caps - np.where(tier == 1, r, 0)).sum())
+        caps_r = caps.copy()
+        if need > 0:
+            caps_r[-1] += need
+        traffic = rng.integers(1, 1000, nb).astype(np.int64)
+        for pool in (1, 100):
+            b, s, A, U, T, rep = M.place(None, hot, caps_r, bin_tier=tier, bin_traffic=traffic, pool=pool,
+                                         replicate_rows=r, return_replica_access=True)
+            ob, os_, oA, oU, orep = orc.ddak_replicate(hot, tier - 1, caps_r, traffic, r, pool)
+            assert np.array_equal(b, ob) and np.array_equal(s, os_), (r, pool)
+            assert np.array_equal(A, oA) and np.array_equal(U, oU) and rep == orep
+            # one rank's device map: replicas point at that rank's own bin
+            g = int(rng.integers(0, n_gpu))
+            packed = M.place_pack_rank(b, s, g)
+            want = np.where(b == M.BIN_REPLICA, g, b).astype(np.uint64) << np.uint64(40) | s.astype(np.uint64)
+            assert np.array_equal(packed, want)
+            if r > 0:
+                with pytest.raises(M.MomentError):
+                    M.place_pack(b, s)  # a replica has no single bin
+
+
+def test_ddak_replicate_errors():
+    hot = np.arange(10, dtype=np.uint64)
+    with pytest.raises(M.MomentError) as e:  # r above a GPU bin's capacity
+        M.place(None, hot, [4, 8, 20], bin_tier=[1, 1, 2], bin_traffic=[1, 1, 1], replicate_rows=5)
+    assert e.value.status == M.EINFEASIBLE
+    with pytest.raises(M.MomentError) as e:  # hash placement has no replicas
+        M.place(None, hot, [10, 10], bin_tier=[1, 2], bin_traffic=[1, 1], replicate_rows=1, mode=M.PLACE_HASH)
+    assert e.value.status == M.EINVAL
+    with pytest.raises(M.MomentError):
+        M.place_pack_rank([M.BIN_REPLICA], [0], 64)
+    # r = n with room: everything replicated, nothing partitioned
+    b, s, A, U, T = M.place(None, hot, [10, 10, 0], bin_tier=[1, 1, 2], bin_traffic=[1, 1, 1], replicate_rows=10)
+    assert (b == M.BIN_REPLICA).all() and list(U) == [0, 0, 0]
+    assert list(s[np.argsort(-hot.astype(np.int64), kind="stable")]) == list(range(10))
+
+
+@pytest.mark.parametrize("k,d_host0,d_hbm,d_rep", [(8, 4000, 500, 700), (2, 0, 300, 10**6), (1, 500, 500, 1)])
+def test_plan_replica_demand_vs_oracle(orc, k, d_host0, d_hbm, d_rep):
+    nodes, links, host, hbm_nodes, gpu_nodes = two_socket_box(k=8)
+    topo = M.topology(nodes, links)
+    N, _, s, t = topo.info()
+    allnodes, _, _, _ = topo.export()
+    demand = np.zeros(N, np.int64)
+    demand[host[0]] = d_host0
+    for g in range(k):
+        demand[hbm_nodes[g]] = d_hbm
+    p0 = M.plan(topo, gpu_nodes[:k], demand, 770, 6000).info()
+    p = M.plan(topo, gpu_nodes[:k], demand, 770, 6000, replica_demand=d_rep).info()
+    assert p["t_ingest"] == p0["t_ingest"] and p["t_nvlink"] == p0["t_nvlink"]  # replicas: HBM only
+    bins = [v for v in range(N) if allnodes[v][0] == M.NODE_STORAGE]
+    owner = [allnodes[v][2] if allnodes[v][1] == M.TIER_GPU_HBM and allnodes[v][2] < k else -1 for v in bins]
+    d = [demand[v] for v in bins]
+    tn, th = orc.plan_closed_forms(k, owner, d, [p["quota"][v] for v in bins], 770, 6000, d_rep)
+    assert (p["t_nvlink"], p["t_hbm"]) == (tn, th)
+    assert p["t_star"] == max(p["t_ingest"], tn, th)
+    with pytest.raises(M.MomentError):
+        M.plan(topo, gpu_nodes[:k], demand, 770, 6000, replica_demand=-1)
+
+
+def _search_setup(k, n, cap_gpu, host_cap, hot, port=55, nv=900, hbm=6500):
+    nodes, links, host, hbm_nodes, gpu_nodes = two_socket_box(k=k, port=port, nv=nv, hbm=hbm)
+    topo = M.topology(nodes, links)
+    bin_node = hbm_nodes + host
+    tier = [M.TIER_GPU_HBM] * k + [M.TIER_HOST_DRAM] * 2
+    caps = [cap_gpu] * k + [host_cap, host_cap]
+    traffic = [hbm] * k + [10, 10]
+    return topo, bin_node, tier, caps, traffic, gpu_nodes, host, hbm_nodes
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_replicate_search_vs_oracle_composition(orc, seed):
+    """Every candidate's T* = the plan (checked against the oracle above) of the demands that the ORACLE's
+    replicated placement implies: d_b = floor(R A_b / batches), d_rep = floor(R A_rep / batches)."""
+    rng = np.random.default_rng(seed)
+    k, n, R, batches = [2, 4, 8, 8][seed], 5000, 512, 64
+    hot = (rng.pareto(0.8, n) * 5).astype(np.uint64)
+    cap_gpu = [n // k, n // (2 * k), n, n // 3][seed]
+    topo, bin_node, tier, caps, traffic, gpu_nodes, host, hbm_nodes = _search_setup(k, n, cap_gpu, n, hot)
+    cand = [0, cap_gpu // 4, cap_gpu // 2, cap_gpu, cap_gpu + 1]
+    held = (rng.pareto(0.8, n) * 3).astype(np.uint64)  # held-out batches' counts (demand estimate)
+    for dem, dem_batches in ((None, 0), (held, 32)):
+        ts, best = M.replicate_search(topo, hot, caps, cand, gpu_node=gpu_nodes, nvlink_cap=900, hbm_cap=6500,
+                                      row_bytes=R, hot_batches=batches, bin_node=bin_node, bin_tier=tier,
+                                      bin_traffic=traffic, demand_counts=dem, demand_batches=dem_batches)
+        cnt, nb_ = (hot, batches) if dem is None else (dem, dem_batches)
+        N = topo.info()[0]
+        for r, t_got in zip(cand, ts):
+            if r > cap_gpu:
+                assert t_got == -1
+                continue
+            b, s, A, U, rep = orc.ddak_replicate(hot, np.array(tier) - 1, caps, traffic, r, 100)
+            demand = np.zeros(N, np.int64)
+            for i, v in enumerate(bin_node):
+                demand[v] += int(cnt[b == i].sum()) * R // nb_
+            rep_d = int(cnt[b == -2].sum()) * R // nb_
+            want = M.plan(topo, gpu_nodes, demand, 900, 6500, replica_demand=rep_d).info()["t_star"]
+            assert t_got == want, r
+        feas = [i for i, x in enumerate(ts) if x >= 0]
+        assert best == min(feas, key=lambda i: (ts[i], i))
+
+
+def test_replicate_search_closed_forms():
+    """Uniform hotness, all rows fit in every GPU (no host rows): replicating everything removes the
+    NVLink term; with k = 1 replication changes nothing; with tight GPU capacity, replication pushes rows
+    to the host tier and T* grows."""
+    n, R, batches, k = 8000, 512, 1, 8
+    hot = np.ones(n, np.uint64)
+    topo, bin_node, tier, caps, traffic, gpu_nodes, host, hbm_nodes = _search_setup(k, n, n, n, hot, nv=900,
+                                                                                      hbm=6500)
+    cand = [0, n // 4, n // 2, n]
+    ts, best = M.replicate_search(topo, hot, caps, cand, gpu_node=gpu_nodes, nvlink_cap=900, hbm_cap=6500,
+                                  row_bytes=R, hot_batches=batches, bin_node=bin_node, bin_tier=tier,
+                                  bin_traffic=traffic)
+    # per GPU per batch: D = n R bytes. r = 0: DDAK splits evenly (equal traffic), each GPU reads
+    # (k-1)/k D over NVLink in and serves the same out: T_nvlink = ceil(7/8 D / 900); r = n: T = ceil(2D/6500)
+    D = n * R
+    assert ts[0] == max(-(-(D * 7 // 8) // 900), -(-(D + k * D // 8) // 6500))
+    assert ts[-1] == -(-(2 * D) // 6500)
+    assert list(ts) == sorted(ts, reverse=True) and best == 3
+    # tight GPU capacity (n/8 per GPU = the whole table exactly once): every replica forces n/8 rows
+    # (spread over 8 bins) to host DRAM over 55 bytes/us ports
+    topo, bin_node, tier, caps, traffic, gpu_nodes, host, hbm_nodes = _search_setup(k, n, n // k, n, hot)
+    ts, best = M.replicate_search(topo, hot, caps, [0, 100, 500], gpu_node=gpu_nodes, nvlink_cap=900,
+                                  hbm_cap=6500, row_bytes=R, hot_batches=batches, bin_node=bin_node, bin_tier=tier,
+                                  bin_traffic=traffic)
+    assert best == 0 and ts[0] < ts[1] < ts[2]
