@@ -127,7 +127,14 @@ typedef struct {
                                          other vertices are placed by DDAK over the GPU bins' capacities minus
                                          r (their slots start at r) and the other bins unchanged. Requires
                                          r <= every GPU bin's capacity. 0 = plain DDAK (bit-identical). */
+    int32_t traffic_mode;             /* when bin_traffic is NULL: MOMENT_TRAFFIC_RATE_FLOW (0) = f(s, b) of
+                                         one rate max-flow (non-unique, R7: a symmetric box can give
+                                         one of two equal host bins all the flow and the other none), or
+                                         MOMENT_TRAFFIC_STANDALONE (1) = the max-flow from b alone to t with
+                                         every other supply link cut (unique, R7's canonical mode) */
 } moment_place_args;
+
+enum { MOMENT_TRAFFIC_RATE_FLOW = 0, MOMENT_TRAFFIC_STANDALONE = 1 };
 
 /* bin_of value of a vertex replicated in every GPU_HBM bin (replicate_rows > 0). */
 #define MOMENT_BIN_REPLICA (-2)

@@ -488,7 +488,7 @@ int orc_bucket(int32_t g, int32_t k, int32_t n_bins, const int32_t* hbm_owner, c
  *       cand = non-full bins of the best tier that has a non-full bin with traffic > 0;
  *              if none: all non-full bins; if none: EINFEASIBLE
  *       b* = argmin over cand of priority_b = (A_b / T_b) * (U_b / C_b)           (Eq. 2; R13 argmin)
- *            T_b = 0 => +inf; ties -> better tier, then lower index                 (R16)
+ *            T_b = 0 => +inf; ties -> less filled (U_b / C_b), then better tier, then lower index (R16)
  *       take m = min(|group|, C_b* - U_b*) vertices in order; slot_of = U_b*, U_b*+1, ...
  *       A_b* += their hotness; U_b* += m                                            (P:L252 re-evaluate)
  * A = Bin_access (cumulative hotness), T = Bin_traffic, U = Bin_currentCapacity (rows), C = Bin_Capacity.
@@ -576,8 +576,14 @@ int orc_ddak(int64_t n, const uint64_t* hotness, int32_t n_bins, const int32_t* 
                 if (bstar < 0) { bstar = b; continue; }
                 int c = priority_cmp(A[b], U[b], traffic[b], cap_rows[b], A[bstar], U[bstar], traffic[bstar],
                                      cap_rows[bstar]);
+                if (c == 0) {
+                    /* R16: equal priority -> the less-filled bin, U_b / C_b < U_b* / C_b* */
+                    unsigned __int128 fb = (unsigned __int128)(uint64_t)U[b] * (uint64_t)cap_rows[bstar];
+                    unsigned __int128 fs = (unsigned __int128)(uint64_t)U[bstar] * (uint64_t)cap_rows[b];
+                    c = fb < fs ? -1 : (fb > fs ? 1 : 0);
+                }
                 if (c < 0 || (c == 0 && tier_rank[b] < tier_rank[bstar])) bstar = b;
-                /* equal priority and tier: keep the lower index (bstar < b) */
+                /* equal priority, fill and tier: keep the lower index (bstar < b) */
             }
             if (bstar < 0) { status = ORC_EINFEASIBLE; break; }
             int64_t room = cap_rows[bstar] - U[bstar];

@@ -343,6 +343,12 @@ int priority_cmp(const Bin& a, const Bin& b) {
     return cmp_frac(pa, qa, pb, qb);
 }
 
+// -1 if a is less filled than b (U_a / C_a < U_b / C_b), exactly; C > 0 for non-full bins.
+int fill_cmp(const Bin& a, const Bin& b) {
+    const u128 l = (u128)(uint64_t)a.used * (u128)(uint64_t)b.cap, r = (u128)(uint64_t)b.used * (u128)(uint64_t)a.cap;
+    return l < r ? -1 : (l > r ? 1 : 0);
+}
+
 // Stable LSD radix sort of vertex ids by descending hotness (ties: ascending id, from stability).
 void order_by_hotness(int64_t n, const uint64_t* hot, std::vector<uint32_t>& order) {
     order.resize(n);
@@ -426,15 +432,27 @@ moment_status resolve_bins(moment_topo_t T, const moment_place_args* a, std::vec
         for (int b = 0; b < nb; b++) traffic[b] = a->bin_traffic[b];
     } else {
         if (!T) return fail(MOMENT_EINVAL, "moment_place: bin_traffic is null and no topology given");
+        if (a->traffic_mode != MOMENT_TRAFFIC_RATE_FLOW && a->traffic_mode != MOMENT_TRAFFIC_STANDALONE)
+            return fail(MOMENT_EINVAL, "moment_place: unknown traffic_mode %d", a->traffic_mode);
         std::vector<int32_t> from, to;
         std::vector<int64_t> cap, flow;
         split_links(T, from, to, cap);
-        int64_t F = 0;
-        MOMENT_TRY(run_flow((int)T->nodes.size(), from, to, cap, T->s, T->t, &F, &flow));
-        for (int b = 0; b < nb; b++) {
+        for (int b = 0; b < nb; b++)
             if (bin_node[b] < 0) return fail(MOMENT_EINVAL, "moment_place: bin %d has no topology node", b);
-            for (size_t i = 0; i < T->links.size(); i++)
-                if (T->links[i].from == T->s && T->links[i].to == bin_node[b]) traffic[b] += flow[i];
+        int64_t F = 0;
+        if (a->traffic_mode == MOMENT_TRAFFIC_RATE_FLOW) {
+            MOMENT_TRY(run_flow((int)T->nodes.size(), from, to, cap, T->s, T->t, &F, &flow));
+            for (int b = 0; b < nb; b++)
+                for (size_t i = 0; i < T->links.size(); i++)
+                    if (T->links[i].from == T->s && T->links[i].to == bin_node[b]) traffic[b] += flow[i];
+        } else {
+            for (int b = 0; b < nb; b++) {
+                std::vector<int64_t> c = cap;
+                for (size_t i = 0; i < T->links.size(); i++)
+                    if (T->links[i].from == T->s && T->links[i].to != bin_node[b]) c[i] = 0;
+                MOMENT_TRY(run_flow((int)T->nodes.size(), from, to, c, T->s, T->t, &F, nullptr));
+                traffic[b] = F;
+            }
         }
     }
     for (int b = 0; b < nb; b++) {
@@ -494,6 +512,7 @@ moment_status ddak_core(int64_t n, const uint64_t* hot, const std::vector<uint32
                 if (best_rank != std::numeric_limits<int>::max() && B.rank != best_rank) continue;
                 if (pick < 0) { pick = b; continue; }
                 int c = priority_cmp(B, bins[pick]);
+                if (c == 0) c = fill_cmp(B, bins[pick]);  // R16: equal priority -> the less-filled bin
                 if (c < 0 || (c == 0 && B.rank < bins[pick].rank)) pick = b;
             }
             if (pick < 0) return fail(MOMENT_EINFEASIBLE, "moment_place: no bin has room");

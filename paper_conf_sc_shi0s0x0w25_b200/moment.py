@@ -21,6 +21,7 @@ NODE_SOURCE, NODE_SINK, NODE_STORAGE, NODE_INTERCONNECT, NODE_COMPUTE = range(5)
 TIER_NONE, TIER_GPU_HBM, TIER_HOST_DRAM, TIER_SSD = range(4)
 PLACE_DDAK, PLACE_HASH = 0, 1
 BIN_REPLICA = -2
+TRAFFIC_RATE_FLOW, TRAFFIC_STANDALONE = 0, 1
 SAMPLE_REPLACE, SAMPLE_CHECK = 1, 2
 MAX_BINS = 64
 
@@ -53,7 +54,8 @@ class Link(C.Structure):
 class PlaceArgs(C.Structure):
     _fields_ = [("n_vertices", C.c_int64), ("hotness", C.c_void_p), ("n_bins", C.c_int32), ("bin_node", C.c_void_p),
                 ("bin_tier", C.c_void_p), ("bin_capacity_rows", C.c_void_p), ("bin_traffic", C.c_void_p),
-                ("pool", C.c_int64), ("mode", C.c_int32), ("replicate_rows", C.c_int64)]
+                ("pool", C.c_int64), ("mode", C.c_int32), ("replicate_rows", C.c_int64),
+                ("traffic_mode", C.c_int32)]
 
 
 class PlaceOut(C.Structure):
@@ -222,7 +224,8 @@ def topology(nodes, links) -> Topology:
 
 # ---------------------------------------------------------------------------------------------- P4
 def place(topo: Topology | None, hotness, capacity_rows, *, bin_node=None, bin_tier=None, bin_traffic=None,
-          pool: int = 100, mode: int = PLACE_DDAK, replicate_rows: int = 0, return_replica_access: bool = False):
+          pool: int = 100, mode: int = PLACE_DDAK, replicate_rows: int = 0, return_replica_access: bool = False,
+          traffic_mode: int = TRAFFIC_RATE_FLOW):
     """DDAK placement. Returns (bin_of int32[n], slot_of int64[n], access uint64[nb], used int64[nb],
     traffic int64[nb]) [+ replica_access]. replicate_rows > 0: the hottest rows are copied into every GPU bin
     (bin_of = BIN_REPLICA, R25)."""
@@ -240,7 +243,7 @@ def place(topo: Topology | None, hotness, capacity_rows, *, bin_node=None, bin_t
         return arr.ctypes.data
 
     args = PlaceArgs(n, hot.ctypes.data, nb, opt(bin_node, np.int32), opt(bin_tier, np.int32), cap.ctypes.data,
-                     opt(bin_traffic, np.int64), pool, mode, replicate_rows)
+                     opt(bin_traffic, np.int64), pool, mode, replicate_rows, traffic_mode)
     bin_of = np.zeros(max(n, 1), np.int32)
     slot_of = np.zeros(max(n, 1), np.int64)
     acc = np.zeros(nb, np.uint64)
@@ -307,7 +310,7 @@ def plan(topo, gpu_node, demand_bytes, nvlink_cap, hbm_cap, replica_demand: int 
 
 def replicate_search(topo: Topology, hotness, capacity_rows, candidates, *, gpu_node, nvlink_cap: int, hbm_cap: int,
                      row_bytes: int, hot_batches: int, bin_node=None, bin_tier=None, bin_traffic=None, pool: int = 100,
-                     demand_counts=None, demand_batches: int = 0):
+                     demand_counts=None, demand_batches: int = 0, traffic_mode: int = TRAFFIC_RATE_FLOW):
     """T*(r) of the plan for every candidate replicate_rows r (R25). Returns (t_star int64[n_cand] with -1 =
     infeasible, best index or -1). demand_counts / demand_batches: held-out F_H counts for the per-bin demand
     (default: the placement's own hotness)."""
@@ -323,7 +326,7 @@ def replicate_search(topo: Topology, hotness, capacity_rows, candidates, *, gpu_
         return arr.ctypes.data
 
     pa = PlaceArgs(len(hot), hot.ctypes.data, len(cap), opt(bin_node, np.int32), opt(bin_tier, np.int32),
-                   cap.ctypes.data, opt(bin_traffic, np.int64), pool, PLACE_DDAK, 0)
+                   cap.ctypes.data, opt(bin_traffic, np.int64), pool, PLACE_DDAK, 0, traffic_mode)
     g = _np(gpu_node, np.int32)
     cand = _np(candidates, np.int64)
     ts = np.zeros(max(len(cand), 1), np.int64)

@@ -404,3 +404,18 @@ def test_plan_closed_forms_replica_hand_worked(orc):
     # everything replicated (d_b = 0, k = 8): no NVLink bytes, T_hbm = ceil(2 d_rep / hbm)
     assert orc.plan_closed_forms(8, list(range(8)), [0] * 8, [[0] * 8] * 8, 900, 6500, 1000) == (0, 1)
     assert orc.plan_closed_forms(8, list(range(8)), [0] * 8, [[0] * 8] * 8, 0, 6500, 6500) == (0, 2)
+
+
+def test_ddak_zero_hotness_spreads_by_fill(orc):
+    # R16 tie-break: vertices pre-sampling never saw (hotness 0) keep every bin's priority at 0; they go to
+    # the less-filled bin, so equal bins split them evenly and unequal ones in proportion to capacity
+    hot = np.zeros(1000, np.uint64)
+    _, _, _, U = orc.ddak(hot, [1, 1], [600, 600], [5, 5], 1)
+    assert list(U) == [500, 500]
+    _, _, _, U = orc.ddak(hot, [1, 1], [300, 900], [5, 7], 1)
+    assert abs(3 * U[0] - U[1]) <= 3 and U.sum() == 1000
+    # hot vertices first by Eq. 2, the cold tail then balances the fill
+    hot = np.zeros(1000, np.uint64)
+    hot[:10] = 100
+    bin_of, _, A, U = orc.ddak(hot, [1, 1], [600, 600], [5, 5], 1)
+    assert abs(int(U[0]) - int(U[1])) <= 1 and A[0] > 0 and A[1] > 0

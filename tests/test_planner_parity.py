@@ -440,3 +440,25 @@ def test_replicate_search_closed_forms():
                                   hbm_cap=6500, row_bytes=R, hot_batches=batches, bin_node=bin_node, bin_tier=tier,
                                   bin_traffic=traffic)
     assert best == 0 and ts[0] < ts[1] < ts[2]
+
+
+def test_standalone_traffic_vs_oracle(orc):
+    """R7 canonical Bin_traffic: each bin's own max-flow to t (every other supply cut) = the oracle's
+    Edmonds-Karp on the same graph; on the symmetric box both host bins get equal traffic, where the rate
+    max-flow may give one of them none."""
+    for act in ([0], [0, 4], [0, 1, 4, 5], list(range(8))):
+        box = M.boxes.hgx_b200(8, active=act)
+        topo = box.topology()
+        N, L, s, t = topo.info()
+        nodes, links, _, _ = topo.export()
+        bins = [box.hbm_bin[g] for g in act] + box.host_bin
+        hot = np.arange(1000, dtype=np.uint64)
+        *_, T = M.place(topo, hot, [10] * len(act) + [1000, 1000], bin_node=bins,
+                        traffic_mode=M.TRAFFIC_STANDALONE)
+        for i, b in enumerate(bins):
+            cut = [(u, v, 0 if (u == s and v != b) else c) for (u, v, c) in links]
+            assert T[i] == orc.maxflow(N, cut, s, t)[0]
+        if len(act) > 1:
+            assert T[-1] == T[-2]
+    with pytest.raises(M.MomentError):
+        M.place(topo, hot, [10] * 8 + [1000, 1000], bin_node=bins, traffic_mode=7)

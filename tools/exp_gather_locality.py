@@ -18,7 +18,8 @@ import paper_conf_sc_shi0s0x0w25_b200 as M  # noqa: E402
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--rows", type=int, default=120000)
+    ap.add_argument("--rows", default="120000", help="comma-separated row counts")
+    ap.add_argument("--orders", default="sequential,sorted random,unsorted random")
     ap.add_argument("--reps", type=int, default=40)
     a = ap.parse_args()
     cfg = W.CONFIGS["C2"]
@@ -32,7 +33,11 @@ def main():
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     g = torch.Generator(device="cuda")
     g.manual_seed(7)
-    m = a.rows
+    for m in [int(x) for x in a.rows.split(",")]:
+        run(a, ctx, table, flush, g, n, R, stride, m)
+
+
+def run(a, ctx, table, flush, g, n, R, stride, m):
     outs = [torch.empty((m, R), dtype=torch.uint8, device="cuda") for _ in range(4)]
     peak = 6543.4
     orders = {
@@ -45,6 +50,8 @@ def main():
     print(f"{'order':>16s} {'warm b2b us':>12s} {'frac':>6s} {'flushed us':>11s} {'frac':>6s} {'index_select b2b us':>20s}")
     tab_view = table[:, :R]
     for name, ids in orders.items():
+        if name not in a.orders.split(","):
+            continue
         for _ in range(3):
             ctx.gather(ids, outs[0])
         torch.cuda.synchronize()

@@ -69,7 +69,7 @@ def counts(cfg, batches, held):
 
 
 def breakdown(topo, box, active, hot, dem, caps, bin_node, R, held, r, nv, hbm):
-    b, s, A, U, T = M.place(topo, hot, caps, bin_node=bin_node, replicate_rows=r)
+    b, s, A, U, T = M.place(topo, hot, caps, bin_node=bin_node, replicate_rows=r, traffic_mode=M.TRAFFIC_STANDALONE)
     N = topo.info()[0]
     per_bin = np.bincount(b.astype(np.int64) + 2, weights=dem.astype(np.float64), minlength=len(bin_node) + 2)
     d = np.zeros(N, np.int64)
@@ -96,7 +96,7 @@ def evaluate(name, cfg, hot, dem, R, k, active, cap_gpu, a, hbm_gbs, nv_gbs, mea
     ts, best = M.replicate_search(topo, hot, caps, cand, gpu_node=[box.gpu[g] for g in active],
                                   nvlink_cap=int(nv_gbs * 1000), hbm_cap=int(hbm_gbs * 1000), row_bytes=R,
                                   hot_batches=a.batches, bin_node=bin_node, demand_counts=dem,
-                                  demand_batches=a.held)
+                                  demand_batches=a.held, traffic_mode=M.TRAFFIC_STANDALONE)
     t_search = time.perf_counter() - t1
     nv, hb = int(nv_gbs * 1000), int(hbm_gbs * 1000)
     b0 = breakdown(topo, box, active, hot, dem, caps, bin_node, R, a.held, 0, nv, hb)
