@@ -65,20 +65,30 @@ def one_gpu_topology(h2d_gbs, hbm_gbs):
                       [(0, 3, int(hbm_gbs * 1000)), (1, 2, 400_000), (2, 3, int(h2d_gbs * 1000))])
 
 
-def build_tiers(name, cfg, g, R, batches, h2d, hbm_gbs, fan):
-    """P2 hotness (64 pre-sample batches), P3/P4 DDAK placement, HBM cache + pinned ring host tier."""
+def build_tiers(name, cfg, g, R, batches, h2d, hbm_gbs, fan, presample=64, held=64):
+    """P2 hotness (`presample` pre-sample batches: seeds of later epochs than the timed ones, rng epoch
+    2^32 - 1), P3/P4 DDAK placement, HBM cache + pinned ring host tier. Also counts F_H over `held` held-out
+    batches (other seeds, other rng stream) for the planner's demand estimate (as tools/sim_plan.py)."""
     n, B = g.n, cfg["batch"]
     ctx0 = M.Ctx(n_vertices=n, max_seeds=B, max_fanout=fan, device=0)
     bufs = M.SampleBuffers.allocate(B, fan, n, DEV)
     hot = torch.zeros(n, dtype=torch.int64, device=DEV)
+    dem = torch.zeros(n, dtype=torch.int64, device=DEV)
     H = len(fan)
-    for i in range(64):
-        ctx0.step(g.indptr, g.indices, batches[i % len(batches)], fan, W.batch_rng_seed(5, 2**32 - 1, 0, i), bufs,
-                  None)
-        ctx0.hotness(bufs.nodes, hot, n_dev=bufs.counts[H:H + 1], max_n=bufs.nodes.numel())
+    pre = []
+    e = 2
+    while len(pre) < presample + held:
+        pre += W.epoch_batches(batches["train"], B, e)
+        e += 1
+    for i in range(presample + held):
+        p = i < presample
+        ctx0.step(g.indptr, g.indices, pre[i], fan,
+                  W.batch_rng_seed(5, 2**32 - 1, 0, i) if p else W.batch_rng_seed(7, 0, 0, i), bufs, None)
+        ctx0.hotness(bufs.nodes, hot if p else dem, n_dev=bufs.counts[H:H + 1], max_n=bufs.nodes.numel())
     torch.cuda.synchronize()
     hot_np = hot.cpu().numpy().astype(np.uint64)
-    del hot, ctx0, bufs
+    dem_np = dem.cpu().numpy()
+    del hot, dem, ctx0, bufs
     cap_hbm = (CACHE_GIB[name] << 30) // R
     topo = one_gpu_topology(h2d, hbm_gbs)
     t0 = time.perf_counter()
@@ -101,7 +111,10 @@ def build_tiers(name, cfg, g, R, batches, h2d, hbm_gbs, fan):
         ids = torch.arange(c0, min(R_PHYS, c0 + chunk), device=DEV)
         ring[c0:c0 + len(ids)] = W.feature_rows(ids, cfg["dim"], cfg["dtype"]).cpu()
     torch.cuda.empty_cache()
+    held_rows = np.bincount(bin_of, weights=dem_np.astype(np.float64), minlength=2) / held
     info = {"hbm_cache_gib": CACHE_GIB[name], "hbm_rows": int(used[0]), "host_rows": int(used[1]),
+            "presample_batches": presample, "held_out_batches": held,
+            "held_out_rows_per_batch": [float(x) for x in held_rows],
             "host_tier": f"pinned ring of {R_PHYS} rows ({R_PHYS * R / 2**30:.1f} GiB), row(v) = feature(v mod R_phys)",
             "ddak_place_s": t_place, "bin_traffic": [int(x) for x in traffic]}
     return dict(bin_ptr=[hbm.data_ptr(), ring.data_ptr()], bin_owner=[0, -1], placement=placement,
@@ -127,7 +140,7 @@ def run_config(name, args, hbm_gbs, h2d):
            "fanout": fan, "batch": B, "graph_gen_s": t_graph}
     tiered = name in CACHE_GIB
     if tiered:
-        tiers = build_tiers(name, cfg, g, R, [b for b, _ in batches], h2d, hbm_gbs, fan)
+        tiers = build_tiers(name, cfg, g, R, {"train": train}, h2d, hbm_gbs, fan, presample=args.presample)
         res.update(tiers["info"])
         kw = dict(bin_owner=tiers["bin_owner"], bin_ptr=tiers["bin_ptr"], placement=tiers["placement"])
         stride = R
@@ -224,6 +237,12 @@ def run_config(name, args, hbm_gbs, h2d):
         res["plan_s"] = time.perf_counter() - t0
         res["plan_t_star_us"] = pl["t_star"]
         res["plan_prediction_error"] = abs(pl["t_star"] - gather_us) / gather_us
+        # the simulation's estimate: demand from held-out batches' counts, not from the measured batches
+        hr = tiers["info"]["held_out_rows_per_batch"]
+        demand[0], demand[1] = int(hr[0] * R), int(hr[1] * R)
+        ph = M.plan(tiers["topo"], [3], demand, 0, int(hbm_gbs * 1000) // 2).info()
+        res["plan_t_star_heldout_us"] = ph["t_star"]
+        res["plan_heldout_prediction_error"] = abs(ph["t_star"] - gather_us) / gather_us
     # CPU oracle (single thread) on a bounded slice of the same workload: sample + gather (C4/C5 from the ring)
     oracle.build()
     ip, ix = g.indptr.cpu().numpy(), g.indices.cpu().numpy()
@@ -263,6 +282,7 @@ def main():
     ap.add_argument("--batches", type=int, default=200)
     ap.add_argument("--lanes", type=int, default=8)
     ap.add_argument("--oracle-s", type=float, default=8.0)
+    ap.add_argument("--presample", type=int, default=64, help="pre-sample batches for the DDAK hotness (P2)")
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
     torch.cuda.set_device(0)
