@@ -416,6 +416,27 @@ moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* csr, const in
                                int64_t n_seeds, const moment_sample_params* params,
                                const moment_sample_out* out, void* d_rows, int64_t* counts_host, void* stream);
 
+/* ================================================================================================
+ * Consumer: GraphSAGE mean aggregation over one sampled block — the sparse part of a
+ * layer of the model the paper trains (Eq. 1; GraphSAGE, hidden 256). The weight GEMMs,
+ * activation and loss are the caller's (plain library GEMMs).
+ *   out[i, :] = (1 / deg_i) * sum_{e = offsets[i]}^{offsets[i+1]-1} x[src[e], :]      (deg_i = 0 -> 0)
+ * x: device [n_src][ld_x] of `dtype` (row = dim elements, dim * size a multiple of 16 bytes, <= 2048 bytes,
+ * 16-byte aligned); offsets: device int64 [n_dst + 1] relative to the block (moment_sample's per-hop
+ * offsets); src: device int32 [offsets[n_dst]] (< n_src, not checked); out: device [n_dst][ld_out] of
+ * `dtype`. Accumulates in fp32. Enqueued on `stream`. Errors: EINVAL (shape, dtype, alignment),
+ * EUNSUPPORTED (rows above 2048 bytes).
+ * Backward: grad_x[src[e], :] += grad_out[i, :] / deg_i (fp32 atomics; grad_x is caller-zeroed fp32
+ * [n_src][ld_gx]); the order of the additions is not fixed, so results agree to rounding, not bitwise.
+ * ================================================================================================ */
+enum { MOMENT_DTYPE_F32 = 0, MOMENT_DTYPE_BF16 = 1 };
+
+moment_status moment_sage_mean(const void* x, int64_t ld_x, int32_t dtype, int64_t dim, const int64_t* offsets,
+                               const int32_t* src, int64_t n_dst, void* out, int64_t ld_out, void* stream);
+moment_status moment_sage_mean_backward(const void* grad_out, int64_t ld_g, int32_t dtype, int64_t dim,
+                                        const int64_t* offsets, const int32_t* src, int64_t n_dst, float* grad_x,
+                                        int64_t ld_gx, void* stream);
+
 #ifdef __cplusplus
 }
 #endif

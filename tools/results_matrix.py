@@ -282,7 +282,8 @@ def main():
     ap.add_argument("--batches", type=int, default=200)
     ap.add_argument("--lanes", type=int, default=8)
     ap.add_argument("--oracle-s", type=float, default=8.0)
-    ap.add_argument("--presample", type=int, default=64, help="pre-sample batches for the DDAK hotness (P2)")
+    ap.add_argument("--presample", type=int, default=512,
+                    help="pre-sample batches for the DDAK hotness (P2); 512 = SURVEY 8(d)'s 64 per rank summed over 8 ranks")
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
     torch.cuda.set_device(0)
