@@ -79,6 +79,10 @@ def _setup(L):
     L.orc_ddak.restype = C.c_int
     L.orc_ddak_replicate.argtypes = [I64, P, I32, P, P, P, I64, I64, P, P, P, P, P]
     L.orc_ddak_replicate.restype = C.c_int
+    L.orc_sage_mean.argtypes = [P, I64, P, P, I64, P]
+    L.orc_sage_mean.restype = None
+    L.orc_sage_mean_backward.argtypes = [P, I64, P, P, I64, P]
+    L.orc_sage_mean_backward.restype = None
 
 
 def _p(a: np.ndarray):
@@ -260,3 +264,27 @@ def ddak_replicate(hotness, tier_rank, cap_rows, traffic, r: int, pool: int = 10
     if st != OK:
         raise OracleError(st, "ddak_replicate")
     return bin_of[:n], slot_of[:n], A, U, int(rep[0])
+
+
+def sage_mean(x, offsets, src):
+    """fp64 mean aggregation over a block (Eq. 1): out[i] = mean of x[src[e]], e in [offsets[i], offsets[i+1])."""
+    x = _c(x, np.float64)
+    off = _c(offsets, np.int64)
+    sr = _c(src, np.int32)
+    n_dst = len(off) - 1
+    dim = x.shape[1]
+    out = np.zeros((max(n_dst, 1), dim), np.float64)
+    lib().orc_sage_mean(_p(x), dim, _p(off), _p(sr), n_dst, _p(out))
+    return out[:n_dst]
+
+
+def sage_mean_backward(g, offsets, src, n_src: int):
+    """fp64 adjoint of sage_mean: gx[src[e]] += g[i] / deg_i."""
+    g = _c(g, np.float64)
+    off = _c(offsets, np.int64)
+    sr = _c(src, np.int32)
+    n_dst = len(off) - 1
+    dim = g.shape[1]
+    gx = np.zeros((max(n_src, 1), dim), np.float64)
+    lib().orc_sage_mean_backward(_p(g), dim, _p(off), _p(sr), n_dst, _p(gx))
+    return gx[:n_src]

@@ -21,6 +21,7 @@
  *   orc_bucket ............... per-request routing by placement + quota (R12)
  *   orc_ddak ................. data-distribution-aware knapsack, Eq. 2 (R13-R17)
  *   orc_ddak_replicate ....... the same with the r hottest rows replicated in every GPU bin (R25)
+ *   orc_sage_mean(_backward) . GraphSAGE mean aggregation over a sampled block and its adjoint (Eq. 1)
  *
  * Parity status of every function is listed in DESIGN.md §4 with its pins (tests/test_oracle_*.py).
  */
@@ -656,4 +657,32 @@ int orc_ddak_replicate(int64_t n, const uint64_t* hotness, int32_t n_bins, const
     }
     free(is_rep); free(ids); free(sub_hot); free(sub_bin); free(sub_slot); free(cap2);
     return st;
+}
+
+/* ------------------------------------------------------------------------------------------------
+ * GraphSAGE mean aggregation over one sampled block (Eq. 1: the aggregate of the neighbours'
+ * h_u^{l-1}; the paper's model is GraphSAGE), in fp64:
+ *   out[i][c] = (1 / deg_i) * sum_{e = offsets[i]}^{offsets[i+1]-1} x[src[e]][c],  deg_i = 0 -> 0
+ * and its adjoint (the backward of the same linear map):
+ *   gx[src[e]][c] += g[i][c] / deg_i   for every edge e of row i
+ * ------------------------------------------------------------------------------------------------ */
+void orc_sage_mean(const double* x, int64_t dim, const int64_t* offsets, const int32_t* src, int64_t n_dst,
+                   double* out) {
+    for (int64_t i = 0; i < n_dst; i++) {
+        int64_t deg = offsets[i + 1] - offsets[i];
+        for (int64_t c = 0; c < dim; c++) {
+            double acc = 0.0;
+            for (int64_t e = offsets[i]; e < offsets[i + 1]; e++) acc += x[(int64_t)src[e] * dim + c];
+            out[i * dim + c] = deg > 0 ? acc / (double)deg : 0.0;
+        }
+    }
+}
+
+void orc_sage_mean_backward(const double* g, int64_t dim, const int64_t* offsets, const int32_t* src, int64_t n_dst,
+                            double* gx) {
+    for (int64_t i = 0; i < n_dst; i++) {
+        int64_t deg = offsets[i + 1] - offsets[i];
+        for (int64_t e = offsets[i]; e < offsets[i + 1]; e++)
+            for (int64_t c = 0; c < dim; c++) gx[(int64_t)src[e] * dim + c] += g[i * dim + c] / (double)deg;
+    }
 }

@@ -22,6 +22,7 @@ TIER_NONE, TIER_GPU_HBM, TIER_HOST_DRAM, TIER_SSD = range(4)
 PLACE_DDAK, PLACE_HASH = 0, 1
 BIN_REPLICA = -2
 TRAFFIC_RATE_FLOW, TRAFFIC_STANDALONE = 0, 1
+DTYPE_F32, DTYPE_BF16 = 0, 1
 SAMPLE_REPLACE, SAMPLE_CHECK = 1, 2
 MAX_BINS = 64
 
@@ -32,7 +33,7 @@ EXPORTED = [
     "moment_sample", "moment_sample_check", "moment_hotness", "moment_bucket", "moment_gather", "moment_gather_group",
     "moment_step", "moment_step_host", "moment_gather_routed", "moment_relay_pack", "moment_relay_serve",
     "moment_relay_scatter", "moment_relay_push", "moment_relay_serve_push", "moment_ipc_export", "moment_ipc_import",
-    "moment_ipc_close",
+    "moment_ipc_close", "moment_sage_mean", "moment_sage_mean_backward",
 ]
 MAX_WORLD = 64
 
@@ -143,6 +144,8 @@ def lib():
             "moment_ipc_export": ([P, P, P], I32),
             "moment_ipc_import": ([P, P], I32),
             "moment_ipc_close": ([P], I32),
+            "moment_sage_mean": ([P, I64, I32, I64, P, P, I64, P, I64, P], I32),
+            "moment_sage_mean_backward": ([P, I64, I32, I64, P, P, I64, P, I64, P], I32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -546,3 +549,34 @@ def gather_group(ctxs, ids, out, *, n_dev=None, max_n: int, stream=None):
     nd = (C.c_void_p * k)(*[t.data_ptr() for t in n_dev]) if n_dev is not None else None
     _check(lib().moment_gather_group(C.cast(hs, P), k, C.cast(ip, P), C.cast(nd, P) if nd is not None else None,
                                      max_n, C.cast(op, P), _stream(stream)))
+
+
+# ---------------------------------------------------------------------------------------------- consumer
+def _dtype_code(t) -> int:
+    import torch
+
+    if t.dtype == torch.float32:
+        return DTYPE_F32
+    if t.dtype == torch.bfloat16:
+        return DTYPE_BF16
+    raise MomentError(EINVAL, f"unsupported dtype {t.dtype}")
+
+
+def sage_mean(x, offsets, src, n_dst: int, out, *, stream=None):
+    """out[i] = mean of x[src[e]] over the block's edges of row i (moment_sage_mean). x, out: 2-D tensors of the
+    same dtype (fp32 / bf16) with unit column stride."""
+    if x.stride(1) != 1 or out.stride(1) != 1 or out.dtype != x.dtype:
+        raise MomentError(EINVAL, "sage_mean: x and out need unit column stride and one dtype")
+    _check(lib().moment_sage_mean(x.data_ptr(), x.stride(0), _dtype_code(x), x.shape[1], offsets.data_ptr(),
+                                  src.data_ptr(), n_dst, out.data_ptr(), out.stride(0), _stream(stream)))
+    return out
+
+
+def sage_mean_backward(grad_out, offsets, src, n_dst: int, grad_x, *, stream=None):
+    """grad_x[src[e]] += grad_out[i] / deg_i (fp32 grad_x, caller-zeroed)."""
+    if grad_out.stride(1) != 1 or grad_x.stride(1) != 1:
+        raise MomentError(EINVAL, "sage_mean_backward: unit column stride needed")
+    _check(lib().moment_sage_mean_backward(grad_out.data_ptr(), grad_out.stride(0), _dtype_code(grad_out),
+                                           grad_out.shape[1], offsets.data_ptr(), src.data_ptr(), n_dst,
+                                           grad_x.data_ptr(), grad_x.stride(0), _stream(stream)))
+    return grad_x
