@@ -27,7 +27,6 @@ struct moment_ctx_s {
     // L2 promotion of the gathered rows: 64 B (measured: a 400-byte row then costs 448 B of DRAM reads instead
     // of the 512 B whole 128-byte lines the default fetches; MOMENT_TMA_PROMO: 0 none, 1 64B, 2 128B, 3 256B)
     int32_t tma_promo = 1;
-    int32_t tma4_balance = 0;        // balanced last round of the gather4 kernel (MOMENT_TMA4_BALANCE)
     int32_t tma4_blocks_per_sm = 3;  // 1-warp gather4 blocks per SM, 4 stages of 8 x 4 rows (MOMENT_TMA4_BLOCKS)
     int32_t l2_load_policy = 0, l2_store_policy = 1;  // bulk gather L2 hints: 0 normal, 1 evict_first, 2 evict_last
     int32_t hop_grid_per_sm = 4, compact_grid_per_sm = 1;  // launch caps (MOMENT_HOP_GRID / MOMENT_COMPACT_GRID)

@@ -223,47 +223,11 @@ __global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const ui
 // own bulk copy (per-lane bulk groups). Rows past the end of a tile repeat the tile's first row and are
 // not stored.
 constexpr int kTma4Rows = 32;  // rows per tile = 8 groups of 4
-// Work items of block b (t0 = b, dt = grid): tile t0 + i dt (32 rows) for i < rounds. balance = 0: every
-// tile of the batch that way (the last round leaves grid - (n_tiles mod grid) blocks idle). balance = 1:
-// rounds = floor(n_tiles / grid) full rounds, then the remaining rows (< 32 grid) are split evenly, one
-// chunk of <= 32 rows (a multiple of 4) per block, so every block ends after the same number of rows
-// (+-4) instead of one block in (n_tiles mod grid) / grid doing a whole extra tile.
-struct Tma4Items {
-    int64_t n, rounds, base, chunk, n_items;
-    int64_t t0, dt;
-    bool balance;
-    __device__ Tma4Items(int64_t n_, int64_t t0_, int64_t dt_, bool bal) : n(n_), t0(t0_), dt(dt_), balance(bal) {
-        const int64_t n_tiles = (n + kTma4Rows - 1) / kTma4Rows;
-        if (!balance || n_tiles % dt == 0) {
-            balance = false;
-            rounds = t0 < n_tiles ? (n_tiles - t0 + dt - 1) / dt : 0;
-            base = chunk = 0;
-            n_items = rounds;
-        } else {
-            rounds = n_tiles / dt;
-            base = rounds * dt * kTma4Rows;
-            const int64_t rem = n - base;  // < 32 dt
-            chunk = (((rem + dt - 1) / dt) + 3) & ~int64_t(3);
-            n_items = rounds + (base + t0 * chunk < n ? 1 : 0);
-        }
-    }
-    // first row and row count of item i (< n_items)
-    __device__ void at(int64_t i, int64_t& row0, int& rows) const {
-        if (i < rounds) {
-            row0 = (t0 + i * dt) * kTma4Rows;
-            rows = (int)min((int64_t)kTma4Rows, n - row0);
-        } else {
-            row0 = base + t0 * chunk;
-            rows = (int)min(chunk, n - row0);
-        }
-    }
-};
-
 template <int kStages>
 __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__ CUtensorMap tmap,
                                                          const int64_t* __restrict__ ids, const int64_t* n_dev,
                                                          int64_t max_n, uint32_t R, int l2_load, int l2_store,
-                                                         int balance, char* __restrict__ out) {
+                                                         char* __restrict__ out) {
     extern __shared__ __align__(128) char stage[];  // kStages * 8 * G
     __shared__ __align__(8) uint64_t full[kStages];
     const int lane = threadIdx.x;
@@ -273,8 +237,7 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
     if (lane == 0) asm volatile("prefetch.tensormap [%0];" ::"l"(&tmap) : "memory");
     // the first kStages tiles' ids are loaded speculatively (bounded by max_n, the ids buffer) together with
     // the count instead of after it: one dependent global round trip fewer before the first row request.
-    // Ids past the count are never used (issue() replaces them by the tile's first row); a speculative id of
-    // an item that turns out to be a balanced tail chunk is reloaded.
+    // Ids past the count are never used (issue() replaces them by the tile's first row).
     int32_t pre[kStages];
 #pragma unroll
     for (int s = 0; s < kStages; s++) {
@@ -282,22 +245,17 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
         pre[s] = r < max_n ? (int32_t)__ldg(ids + r) : -1;
     }
     const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
-    const Tma4Items items(n, t0, dt, balance != 0);
+    const int64_t n_tiles = (n + kTma4Rows - 1) / kTma4Rows;
     if (lane == 0)
         for (int s = 0; s < kStages; s++) mbar_init(&full[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     __syncwarp();
-    auto load_id = [&](int64_t i) -> int32_t {
-        if (i >= items.n_items) return -1;
-        int64_t row0;
-        int rows;
-        items.at(i, row0, rows);
-        return lane < rows ? (int32_t)__ldg(ids + row0 + lane) : -1;
+    auto load_id = [&](int64_t tile) -> int32_t {
+        const int64_t r = tile * kTma4Rows + lane;
+        return (tile < n_tiles && r < n) ? (int32_t)__ldg(ids + r) : -1;
     };
-    auto issue = [&](int64_t i, int s, int32_t id) {
-        int64_t row0;
-        int rows;
-        items.at(i, row0, rows);
+    auto issue = [&](int64_t tile, int s, int32_t id) {
+        const int rows = (int)min((int64_t)kTma4Rows, n - tile * kTma4Rows);
         const int groups = (rows + 3) >> 2;
         const int32_t first = __shfl_sync(0xffffffffu, id, 0);
         const int32_t rid = lane < rows ? id : first;
@@ -321,18 +279,17 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
                     : "memory");
         }
     };
-    int64_t next = 0;
+    int64_t next = t0;
 #pragma unroll
-    for (int s = 0; s < kStages; s++, next++)
-        if (next < items.n_items) issue(next, s, next < items.rounds ? pre[s] : load_id(next));
+    for (int s = 0; s < kStages; s++, next += dt)
+        if (next < n_tiles) issue(next, s, pre[s]);
     int32_t next_id = load_id(next);
     int it = 0;
-    for (int64_t i = 0; i < items.n_items; i++, it++) {
+    for (int64_t tile = t0; tile < n_tiles; tile += dt, it++) {
         const int s = it % kStages;
         mbar_wait(&full[s], (uint32_t)((it / kStages) & 1));
-        int64_t row0;
-        int rows;
-        items.at(i, row0, rows);
+        const int64_t row0 = tile * kTma4Rows;
+        const int rows = (int)min((int64_t)kTma4Rows, n - row0);
         const int groups = (rows + 3) >> 2;
         if (lane < groups) {
             bulk_store(out + (row0 + 4 * lane) * (int64_t)R, stage + ((size_t)s * 8 + lane) * G,
@@ -340,9 +297,9 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
         }
         if (it > 0) bulk_wait_read<1>();  // this lane's store of the previous tile has read its slot
         __syncwarp();
-        if (it > 0 && next < items.n_items) {
+        if (it > 0 && next < n_tiles) {
             issue(next, (it - 1) % kStages, next_id);
-            next++;
+            next += dt;
             next_id = load_id(next);
         }
     }
@@ -608,7 +565,7 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)148 * bps));
         gather_tma4_kernel<4><<<grid, 32, smem, stream>>>(ctx->tma_map, ids, n_dev, max_n, (uint32_t)ctx->row_bytes,
                                                           ctx->l2_load_policy, ctx->l2_store_policy,
-                                                          ctx->tma4_balance, reinterpret_cast<char*>(out));
+                                                          reinterpret_cast<char*>(out));
         return cuda_check(cudaGetLastError(), "moment_gather: tma4 launch");
     }
     if (bulk && route == nullptr) {

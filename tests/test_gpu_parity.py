@@ -153,19 +153,18 @@ def test_sample_reused_ctx_many_batches(orc, c1, sparse, monkeypatch):
         assert_same_sample(got, want)
 
 
-@pytest.mark.parametrize("path", ["auto", "ldg", "bulk", "tma4", "tma4b"])
+@pytest.mark.parametrize("path", ["auto", "ldg", "bulk", "tma4"])
 @pytest.mark.parametrize("dim,dtype", [(4, torch.float32), (12, torch.float32), (100, torch.float32),
                                        (128, torch.float32), (768, torch.float16), (1024, torch.float32)])
 def test_gather_replicated(orc, dim, dtype, path, monkeypatch):
     _need_gpu()
-    monkeypatch.setenv("MOMENT_GATHER_PATH", "tma4" if path == "tma4b" else path)
-    monkeypatch.setenv("MOMENT_TMA4_BALANCE", "1" if path == "tma4b" else "0")
+    monkeypatch.setenv("MOMENT_GATHER_PATH", path)
     n = 5000
     table = W.feature_table(n, dim, dtype, device=DEV)
     R = table.shape[1]
     rng = np.random.default_rng(dim)
-    # counts past one round of tiles (148 SMs x 3 blocks x 32 rows) exercise the balanced tail chunks
-    for count in [1, 31, 1000, 4099] + ([15000, 50001] if path.startswith("tma4") else []):
+    # counts past one round of tiles (148 SMs x 3 blocks x 32 rows) exercise the ragged last round
+    for count in [1, 31, 1000, 4099] + ([15000, 50001] if path == "tma4" else []):
         ids = torch.as_tensor(rng.integers(0, n, count), device=DEV)
         ctx = M.Ctx(n_vertices=n, max_seeds=1, max_fanout=[1], device=0, row_bytes=R, bin_owner=[0],
                     bin_ptr=[table.data_ptr()])
