@@ -551,3 +551,48 @@ def test_gather_replicated_hot_rows_per_rank_maps(orc, c1, world):
                 bins[b][:r] = t_cpu[torch.as_tensor(rep)].to(DEV)[torch.as_tensor(np.argsort(slot_of[rep]))]
         del ctx
     assert n_rep_seen > 0
+
+
+def test_near_maximum_frontier_uniform_graph(orc):
+    """Workspace bounds at (nearly) their maximum: a uniform random graph with 2^24 vertices and 16 distinct-ish
+    out-neighbours each has almost no overlap between frontiers, so one batch of the bench's shape (1024 seeds,
+    [15, 10, 5]) reaches |F_H| close to the no-dedup bound 1 081 344 (R-MAT batches stay near 121 k): whole-sample
+    parity with the oracle, the padded sampler buffers and the compaction tiles at their largest, the gather of
+    ~1 M rows (432 MB) checked on a sample of rows, in both bitscan modes."""
+    _need_gpu()
+    n, deg = 1 << 24, 16
+    gen = torch.Generator(device=DEV)
+    gen.manual_seed(2024)
+    indices = torch.randint(0, n, (n * deg,), device=DEV, generator=gen, dtype=torch.int64)
+    indices = indices.view(n, deg).sort(dim=1).values.reshape(-1).to(torch.int32)
+    indptr = torch.arange(0, n * deg + 1, deg, device=DEV, dtype=torch.int64)
+    fan = [15, 10, 5]
+    seeds = torch.randperm(n, device=DEV, generator=gen)[:1024]
+    dim = 100
+    rows_needed = 1024 * 16 * 11 * 6
+    table = W.feature_table(n, dim, torch.float32, device=DEV)
+    R = table.shape[1]
+    ip, ix = indptr.cpu().numpy(), indices.cpu().numpy()
+    want = orc.sample(ip, ix, seeds.cpu().numpy(), fan, 4242)
+    nF = int(want["counts"][3])
+    assert nF > 1_000_000 and nF <= rows_needed
+    for sparse in ("0", "1"):
+        import os
+        os.environ["MOMENT_SPARSE_SCAN"] = sparse
+        try:
+            ctx = M.Ctx(n_vertices=n, max_seeds=1024, max_fanout=fan, device=0, row_bytes=R, bin_owner=[0],
+                        bin_ptr=[table.data_ptr()])
+        finally:
+            del os.environ["MOMENT_SPARSE_SCAN"]
+        bufs = M.SampleBuffers.allocate(1024, fan, n, DEV)
+        rows = torch.empty((bufs.nodes.numel(), R), dtype=torch.uint8, device=DEV)
+        ctx.step(indptr, indices, seeds, fan, 4242, bufs, rows)
+        torch.cuda.synchronize()
+        assert_same_sample(bufs.result(), want)
+        pick = np.random.default_rng(1).integers(0, nF, 8192)
+        ids = torch.as_tensor(want["nodes"][pick])
+        assert np.array_equal(rows[torch.as_tensor(pick, device=DEV)].cpu().numpy(),
+                              W.feature_rows(ids, dim, torch.float32).numpy())
+        del ctx, bufs, rows
+    del table, indices
+    torch.cuda.empty_cache()
