@@ -556,9 +556,9 @@ def test_gather_replicated_hot_rows_per_rank_maps(orc, c1, world):
 def test_near_maximum_frontier_uniform_graph(orc):
     """Workspace bounds at (nearly) their maximum: a uniform random graph with 2^24 vertices and 16 distinct-ish
     out-neighbours each has almost no overlap between frontiers, so one batch of the bench's shape (1024 seeds,
-    [15, 10, 5]) reaches |F_H| close to the no-dedup bound 1 081 344 (R-MAT batches stay near 121 k): whole-sample
+    [15, 10, 5]) comes close to the no-dedup bound 1 081 344 (R-MAT batches stay near 121 k): whole-sample
     parity with the oracle, the padded sampler buffers and the compaction tiles at their largest, the gather of
-    ~1 M rows (432 MB) checked on a sample of rows, in both bitscan modes."""
+    ~0.94 M rows (375 MB) checked on a sample of rows, in both bitscan modes."""
     _need_gpu()
     n, deg = 1 << 24, 16
     gen = torch.Generator(device=DEV)
@@ -575,7 +575,9 @@ def test_near_maximum_frontier_uniform_graph(orc):
     ip, ix = indptr.cpu().numpy(), indices.cpu().numpy()
     want = orc.sample(ip, ix, seeds.cpu().numpy(), fan, 4242)
     nF = int(want["counts"][3])
-    assert nF > 1_000_000 and nF <= rows_needed
+    # every node of F_h is resampled at hop h (R4), so earlier nodes mostly re-pick neighbours already in the
+    # batch: ~0.94 M here, 7.8x an R-MAT batch, 87 % of the no-dedup bound
+    assert nF > 900_000 and nF <= rows_needed
     for sparse in ("0", "1"):
         import os
         os.environ["MOMENT_SPARSE_SCAN"] = sparse
