@@ -365,7 +365,8 @@ moment_status moment_relay_scatter(moment_ctx_t ctx, const uint64_t* words, cons
  *                             and their number into peer_count[h] = &count_h[self] (0 when none); entries
  *                             for h == self are ignored (may be NULL). Requests beyond cap: MOMENT_EOVERFLOW
  *                             is not detectable on the device, so the caller sizes cap >= max_n.
- *   (caller) barrier: every rank's pushes are complete and visible (stream synchronize + process barrier)
+ *   (caller) barrier: every rank's pushes are complete and visible (moment_signal_barrier, or stream
+ *                         synchronize + process barrier)
  *   moment_relay_serve_push : for every source g != self, the min(count[g], cap) requests of inbox[g] are
  *                             read from THIS rank's mapping of the host bins (its PCIe link) and stored
  *                             straight into g's output (peer stores): peer_out[g] = g's out base,
@@ -375,6 +376,17 @@ moment_status moment_relay_scatter(moment_ctx_t ctx, const uint64_t* words, cons
  * Byte-exact with moment_gather of the same ids.
  * ================================================================================================ */
 #define MOMENT_MAX_WORLD 64
+
+/* Device-side barrier between the two phases (and after the second), replacing "stream synchronize +
+ * process barrier" (a signal barrier over symmetric memory). Every rank owns flags[world]
+ * (uint64, zero-initialised, exported with moment_ipc_export); peer_flags[h] = &flags_h[self] as mapped here
+ * (NULL for h == self). The kernel issues a system-scope fence, stores `epoch` (release, system scope) into
+ * every peer's slot, then waits (acquire) until flags[h] >= epoch for every h != self. `epoch` must grow from
+ * call to call (e.g. 1, 2, 3, ... per barrier). After timeout_ns it stops waiting and writes MOMENT_ETIMEDOUT
+ * into *status_dev (device int32, may be NULL); the caller checks it when it next synchronises. Enqueued on
+ * `stream`; no host synchronisation. world == 1: no-op. Errors: EINVAL. */
+moment_status moment_signal_barrier(int32_t world, int32_t rank, uint64_t* const* peer_flags, const uint64_t* flags,
+                                    uint64_t epoch, int64_t timeout_ns, int32_t* status_dev, void* stream);
 moment_status moment_relay_push(moment_ctx_t ctx, const int64_t* ids, int64_t max_n, const int64_t* qoff,
                                 const int64_t* qpos, uint64_t* const* peer_inbox, int64_t* const* peer_count,
                                 void* stream);

@@ -100,11 +100,14 @@ class PeerExchange:
     Setup is collective over `group`: this rank allocates its inbox (int64 [world][cap][2]), inbox counts
     (int64 [world]) and batch output (uint8 [cap][R]), exports them, and maps every peer's. Per batch
     (`gather`): bucket -> routed gather (own rows) -> relay_push (peer stores) -> barrier -> relay_serve_push
-    (peer stores into the requesters' outputs) -> barrier. The two barriers are the only host
-    synchronisation; with NCCL they are device collectives, with gloo host ones.
+    (peer stores into the requesters' outputs) -> barrier. device_barrier=False: each barrier is a stream
+    synchronize + process barrier (NCCL: device collective, gloo: host). device_barrier=True: each barrier is
+    `moment_signal_barrier` on the stream (release/acquire flag words in peer memory), so a
+    batch's exchange is enqueued without any host synchronisation; `check()` reports a watchdog timeout.
     """
 
-    def __init__(self, ctx, max_n: int, row_bytes: int, device, group=None):
+    def __init__(self, ctx, max_n: int, row_bytes: int, device, group=None, device_barrier: bool = False,
+                 timeout_s: float = 10.0):
         import paper_conf_sc_shi0s0x0w25_b200 as M
 
         self.M, self.ctx, self.group = M, ctx, group
@@ -117,13 +120,17 @@ class PeerExchange:
         self.route = torch.empty(self.cap, dtype=torch.int32, device=dev)
         self.qoff = torch.empty(64 * self.world + 1, dtype=torch.int64, device=dev)
         self.qpos = torch.empty(self.cap, dtype=torch.int64, device=dev)
-        mine = [M.ipc_export(t) for t in (self.inbox, self.count, self.out)]
+        self.device_barrier, self.timeout_ns, self.epoch = device_barrier, int(timeout_s * 1e9), 0
+        self.flags = torch.zeros(self.world, dtype=torch.int64, device=dev)  # uint64 flag words
+        self.status = torch.zeros(1, dtype=torch.int32, device=dev)
+        mine = [M.ipc_export(t) for t in (self.inbox, self.count, self.out, self.flags)]
         everyone = [None] * self.world
         dist.all_gather_object(everyone, mine, group=group)
         self._bases = []
         self.peer_inbox = [0] * self.world
         self.peer_count = [0] * self.world
         self.peer_out = [0] * self.world
+        self.peer_flag = [0] * self.world
         slot_bytes = self.cap * 2 * 8
         for h in range(self.world):
             if h == self.rank:
@@ -136,7 +143,19 @@ class PeerExchange:
             self.peer_inbox[h] = addr[0] + self.rank * slot_bytes  # rank h's inbox slot for this rank
             self.peer_count[h] = addr[1] + self.rank * 8
             self.peer_out[h] = addr[2]
+            self.peer_flag[h] = addr[3] + self.rank * 8  # rank h's flag word for this rank
         dist.barrier(group=group)
+
+    def _barrier(self, s):
+        self.epoch += 1
+        self.M.signal_barrier(self.world, self.rank, self.peer_flag, self.flags, self.epoch,
+                              timeout_ns=self.timeout_ns, status=self.status, stream=s)
+
+    def check(self):
+        """Raise if a device barrier timed out (synchronises)."""
+        st = int(self.status.item())
+        if st != 0:
+            raise self.M.MomentError(st, "PeerExchange: device barrier watchdog expired")
 
     def gather(self, ids: torch.Tensor, n: int, stream=None) -> torch.Tensor:
         """Collective: returns this rank's output view [n, R] = rows of ids[:n]."""
@@ -147,6 +166,12 @@ class PeerExchange:
             ctx.bucket(ids, self.route, self.qoff, self.qpos, max_n=n, stream=s)
             ctx.gather_routed(ids, self.route, self.out, max_n=n, stream=s)
             ctx.relay_push(ids, self.qoff, self.qpos, self.peer_inbox, self.peer_count, max_n=n, stream=s)
+            if self.device_barrier:
+                self._barrier(s)  # every rank's requests are in its relays' inboxes
+                ctx.relay_serve_push(self.inbox, self.count, self.cap, self.peer_out, stream=s)
+                self._barrier(s)  # every relayed row is in its requester's output
+        if self.device_barrier:
+            return self.out[:n]
         s.synchronize()
         dist.barrier(group=self.group)  # every rank's requests are in its relays' inboxes
         with torch.cuda.stream(s):
@@ -157,6 +182,7 @@ class PeerExchange:
 
     def close(self):
         """Collective: unmap the peers' buffers once every rank is done with them."""
+        torch.cuda.synchronize(self.out.device)
         dist.barrier(group=self.group)
         for b in self._bases:
             self.M.ipc_close(b)

@@ -33,7 +33,7 @@ EXPORTED = [
     "moment_sample", "moment_sample_check", "moment_hotness", "moment_bucket", "moment_gather", "moment_gather_group",
     "moment_step", "moment_step_host", "moment_gather_routed", "moment_relay_pack", "moment_relay_serve",
     "moment_relay_scatter", "moment_relay_push", "moment_relay_serve_push", "moment_ipc_export", "moment_ipc_import",
-    "moment_ipc_close", "moment_sage_mean", "moment_sage_mean_backward",
+    "moment_ipc_close", "moment_sage_mean", "moment_sage_mean_backward", "moment_signal_barrier",
 ]
 MAX_WORLD = 64
 
@@ -145,6 +145,7 @@ def lib():
             "moment_ipc_import": ([P, P], I32),
             "moment_ipc_close": ([P], I32),
             "moment_sage_mean": ([P, I64, I32, I64, P, P, I64, P, I64, P], I32),
+            "moment_signal_barrier": ([I32, I32, P, P, U64, I64, P, P], I32),
             "moment_sage_mean_backward": ([P, I64, I32, I64, P, P, I64, P, I64, P], I32),
         }
         for name, (args, res) in sig.items():
@@ -515,6 +516,14 @@ class Ctx:
         outs = (C.c_void_p * len(peer_out))(*[p or None for p in peer_out])
         _check(lib().moment_relay_serve_push(self.handle, inbox.data_ptr(), inbox_count.data_ptr(), cap,
                                              C.cast(outs, P), _stream(stream)))
+
+
+def signal_barrier(world: int, rank: int, peer_flags: list[int], flags, epoch: int, *, timeout_ns: int = 10**10,
+                   status=None, stream=None):
+    """Device-side barrier over peer-mapped flag words (moment_signal_barrier); enqueued, no host sync."""
+    arr = (C.c_void_p * world)(*[p or None for p in peer_flags])
+    _check(lib().moment_signal_barrier(world, rank, arr, _ptr(flags), epoch, timeout_ns, _ptr(status),
+                                       _stream(stream)))
 
 
 IPC_HANDLE_BYTES = 64

@@ -73,21 +73,31 @@ def _rank_main(rank, world, transport="alltoall"):
     nF = int(bufs.counts[2])
     ids = bufs.nodes[:nF].contiguous()
     want = oracle.gather(table.numpy(), ids.cpu().numpy())
-    if transport == "peer":
+    if transport in ("peer", "peer_dev"):
         # the exchange buffers are sized for the largest batch of any rank; two batches check reuse
         nmax = [None] * world
         dist.all_gather_object(nmax, int(bufs.nodes.numel()))
-        px = PeerExchange(ctx, max(nmax), R, dev)
+        px = PeerExchange(ctx, max(nmax), R, dev, device_barrier=transport == "peer_dev", timeout_s=30.0)
         ok = True
         for rep in range(2):
             out = px.gather(ids, nF)
             torch.cuda.synchronize()
             ok &= bool(np.array_equal(out.cpu().numpy(), want))
+        if transport == "peer_dev":
+            # several batches enqueued back to back with no host synchronisation between them
+            outs = []
+            for rep in range(3):
+                outs.append(px.gather(ids, nF).clone())
+            torch.cuda.synchronize()
+            ok &= all(bool(np.array_equal(o.cpu().numpy(), want)) for o in outs)
+            px.check()
         # an empty batch on this rank still serves the other's requests
         out = px.gather(ids, 0 if rank == 0 else nF)
         torch.cuda.synchronize()
         if rank == 1:
             ok &= bool(np.array_equal(out.cpu().numpy(), want))
+        if transport == "peer_dev":
+            px.check()
         px.close()
         info = {"sent": [0] * world, "served": [0] * world}
     else:
@@ -118,4 +128,13 @@ def test_peer_exchange_two_processes_one_gpu():
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
     res = run_world(_rank_main, 2, "peer")
+    assert all(r["ok"] for r in res), res
+
+
+def test_peer_exchange_device_barrier_two_processes_one_gpu():
+    """The peer-memory exchange with device-side signal barriers (moment_signal_barrier) instead of host
+    synchronisation: batches enqueued back to back, byte-exact with the oracle, no watchdog expiry."""
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    res = run_world(_rank_main, 2, "peer_dev")
     assert all(r["ok"] for r in res), res
