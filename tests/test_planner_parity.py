@@ -462,3 +462,17 @@ def test_standalone_traffic_vs_oracle(orc):
             assert T[-1] == T[-2]
     with pytest.raises(M.MomentError):
         M.place(topo, hot, [10] * 8 + [1000, 1000], bin_node=bins, traffic_mode=7)
+
+
+def test_signal_barrier_argument_errors():
+    # host-side validation happens before anything is enqueued (no GPU needed)
+    import ctypes as C
+    L = M.lib()
+    flags = np.zeros(2, np.uint64)
+    peers = (C.c_void_p * 2)(None, flags.ctypes.data)
+    for world, rank, epoch, timeout in [(0, 0, 1, 10), (2, 2, 1, 10), (65, 0, 1, 10), (2, 0, 0, 10), (2, 0, 1, 0)]:
+        st = L.moment_signal_barrier(world, rank, peers, flags.ctypes.data, epoch, timeout, None, None)
+        assert st == M.EINVAL, (world, rank, epoch, timeout)
+    # a null peer pointer for another rank
+    st = L.moment_signal_barrier(2, 0, (C.c_void_p * 2)(None, None), flags.ctypes.data, 1, 10, None, None)
+    assert st == M.EINVAL
