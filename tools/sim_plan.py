@@ -5,7 +5,8 @@ topology graph (`boxes.hgx_b200`), from hotness pre-sampled on the GPU at full g
 The paper evaluates candidate layouts with its model instead of running every one and reports
 its prediction error against measurement (8.61 %); the k = 1 rows here can be compared with the
 measured gathers of profiles/r01_results_matrix.jsonl. k > 1 is a PREDICTION (the pool's boxes have one
-GPU): NVLink at 900 GB/s per direction (spec), host DRAM / UPI capacities assumed (boxes.py).
+GPU): NVLink at the measured 770 GB/s peer-copy rate per direction (900 nominal), host DRAM / UPI capacities
+assumed (boxes.py).
 
     python tools/sim_plan.py [--configs C3,C4,C5] [--batches 512] [--switch 1] [--subsets] [--out FILE]
 
@@ -125,6 +126,8 @@ def main():
     ap.add_argument("--held", type=int, default=128, help="held-out batches (demand estimate)")
     ap.add_argument("--switch", default="1", help="GPUs per PCIe switch, a list (1 = direct to the socket)")
     ap.add_argument("--ks", default="1,2,4,8")
+    ap.add_argument("--nvlink-gbs", type=float, default=770.0,
+                    help="NVLink per direction per GPU: the measured B200 peer copy (B200_PROFILING; 900 nominal)")
     ap.add_argument("--subsets", action="store_true",
                     help="evaluate every class of active-GPU sets up to the box symmetry (P:L229-233)")
     ap.add_argument("--out", default="gpurun_out/plan_sim.jsonl")
@@ -132,7 +135,7 @@ def main():
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
         os.path.join(ROOT, "MEASURED_PEAKS.json")) else {"hbm_gbs": 6543.4}
     hbm_gbs = float(peaks["hbm_gbs"])
-    nv_gbs = 900.0
+    nv_gbs = a.nvlink_gbs
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     fout = open(a.out, "a")
     for name in a.configs.split(","):
