@@ -353,6 +353,20 @@ def main():
     e_b1.record(main_stream)
     torch.cuda.synchronize()
     gather_ms_b2b = e_b0.elapsed_time(e_b1) / (rounds * P)
+    # supplementary: the same gathers with the P lanes' launches concurrent (one stream per lane, as in the
+    # timed region but without the sampling kernels): whole-GPU throughput of the kernel once the ramp and
+    # tail of one launch overlap the others'
+    e_c0, e_c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e_c0.record(main_stream)
+    fork(e_c0)
+    for _ in range(rounds):
+        for L in st.lanes:
+            L.ctx.gather(L.bufs.nodes, L.rows, n_dev=L.bufs.counts[H:H + 1], max_n=L.bufs.nodes.numel(),
+                         stream=L.stream)
+    join()
+    e_c1.record(main_stream)
+    torch.cuda.synchronize()
+    gather_ms_conc = e_c0.elapsed_time(e_c1) / (rounds * P)
     nF_roof = []
     for i in range(n_roof):
         st.step(*batches[i], lane=0)
@@ -436,7 +450,13 @@ def main():
                              "achieved": nF_b2b * (2 * st.R + 8) / (gather_ms_b2b / 1000) / 1e9,
                              "frac": nF_b2b * (2 * st.R + 8) / (gather_ms_b2b / 1000) / 1e9 / peak,
                              "how": f"{rounds} rounds x {P} batches' gathers issued back to back on one stream, "
-                                    "one event pair (launch latency overlapped)"}},
+                                    "one event pair (launch latency overlapped)"},
+                         "concurrent": {
+                             "ms_per_launch": gather_ms_conc,
+                             "achieved": nF_b2b * (2 * st.R + 8) / (gather_ms_conc / 1000) / 1e9,
+                             "frac": nF_b2b * (2 * st.R + 8) / (gather_ms_conc / 1000) / 1e9 / peak,
+                             "how": f"the same {rounds} x {P} gathers, each lane's on its own stream (as in the "
+                                    "timed region, sampling absent): time per launch of the whole-GPU throughput"}},
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_val, "unit": "seeds/s", "h2d_bytes_per_step": st.B * 8,
                     "d2h_bytes_per_step": (2 * H + 1) * 8},
