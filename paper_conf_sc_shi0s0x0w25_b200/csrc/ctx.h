@@ -46,6 +46,9 @@ struct moment_ctx_s {
     uint32_t* newbits = nullptr;    // [n_words]: ids emitted at the current hop
     uint32_t* visited = nullptr;    // [n_words]: F_h membership
     uint32_t* summary = nullptr;    // [n_words / 32]: newbits words marked at the current hop (sparse scan)
+    uint2* rel = nullptr;           // dense scan: [max_hops][rel_stride] {new bits, rank} per word (rank relabel)
+    int64_t rel_stride = 0;         //   words per hop (n_words padded to whole scan tiles)
+    int32_t rank_relabel = 1;       // MOMENT_RANK_RELABEL (dense scan only)
     int64_t n_words = 0;
     // sparse scan (summary bitmap, scan cost proportional to the touched words) for large graphs: auto when
     // n_words > kSparseScanMinWords (MOMENT_SPARSE_SCAN=0/1 forces it off/on)

@@ -10,10 +10,13 @@
 //                 node's k-slot row of a padded buffer, its count to cnt_h, adds it to its compaction
 //                 tile's edge sum, and marks the ids in `newbits`.
 //   bitscan (h) : F_{h+1} = F_h ++ (newbits & ~visited) in ascending id order: chained scan of bitmap
-//                 popcounts (1024 words per tile) gives each new id its position; lidx[id] = position.
+//                 popcounts (1024 words per tile) gives each new id its position. Sparse scan (large graphs):
+//                 lidx[id] = position. Dense scan (rank relabelling): no lidx write; instead rel_h[w] = {new
+//                 bits of word w, rank of its first new id} for every word (a sequential, L2-resident table).
 //   compact     : every tile's global edge position from the per-tile edge sums (no chaining) -> per-hop
-//                 offsets, E_h, and src = lidx[padded id] copied into the packed output; then clears
-//                 `visited` for F_H.
+//                 offsets, E_h, and src = position of the padded id (lidx[id], or from rel: the latest hop
+//                 hh <= h whose word has the id's bit, counts[hh] + rank + popc of the lower bits; seeds via
+//                 lidx) copied into the packed output; then clears `visited` for F_H.
 #include <cooperative_groups.h>
 
 #include <algorithm>
@@ -427,6 +430,10 @@ struct ScanArgs {
     int32_t h;
     unsigned long long* zero;  // the next hop's compaction tile sums, zeroed here (before that hop runs)
     int64_t n_zero;
+    // dense scan with rank relabelling (else null): rel[w] = {new-id bits of word w at this hop, rank of the
+    // word's first new id among the hop's new ids}, written for EVERY word (no clearing needed); lidx is then
+    // not written for non-seed ids and the compaction finds an id's position from rel (L2-resident)
+    uint2* rel;
 };
 
 // F_{h+1} = F_h ++ ascending ids set in (newbits & ~visited).
@@ -469,21 +476,29 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
         const int64_t prefix = dev::lookback_block<kBitscanThreads>(a.tile_status, tile, agg, s_red, &s_nearest);
         int64_t pos = F + prefix + excl;
         if (tile == n_tiles - 1 && threadIdx.x == 0) a.counts[a.h + 1] = F + prefix + agg;
+        uint32_t rk[kScanWords];
 #pragma unroll
         for (int q = 0; q < kScanWords; q++) {
             const int64_t w = w0 + q;
             const uint32_t nw = nb[q] & ~vs[q];
+            rk[q] = (uint32_t)(pos - F);
             uint32_t bits = nw;
             while (bits) {
                 const int b = __ffs(bits) - 1;
                 bits &= bits - 1;
                 const int64_t id = w * 32 + b;
                 a.nodes[pos] = id;
-                a.lidx[id] = (int32_t)pos;
+                if (!a.rel) a.lidx[id] = (int32_t)pos;
                 pos++;
             }
             if (nb[q]) a.newbits[w] = 0u;
             if (nw) a.visited[w] = vs[q] | nw;  // no re-read: the tile owns its words
+        }
+        if (a.rel) {  // rel is padded to whole tiles: every thread's words exist
+            uint4* r4 = reinterpret_cast<uint4*>(a.rel + w0);
+#pragma unroll
+            for (int q = 0; q < kScanWords; q += 2)
+                r4[q / 2] = make_uint4(nb[q] & ~vs[q], rk[q], nb[q + 1] & ~vs[q + 1], rk[q + 1]);
         }
         __syncthreads();
     }
@@ -577,7 +592,21 @@ struct CompactArgs {
     uint32_t kmagic[kMaxHops];  // ceil(2^32 / k): slot / k = umulhi(slot, kmagic) for slot < 2^18, k <= 1024
     const int32_t* pad[kMaxHops];
     const int32_t* cnt[kMaxHops];
+    const uint2* rel;    // dense scan with rank relabelling: hop h's rel at rel + h * rel_stride, else null
+    int64_t rel_stride;
 };
+
+// Position in F_{h+1} of an id sampled at hop h, from the bitscans' rel tables (rank relabelling): the id
+// is new at the latest hop hh <= h whose rel word has its bit, at counts[hh] + the word's rank + the bits
+// below it in the word; an id in no table is a seed, whose position lidx holds.
+__device__ __forceinline__ int32_t rel_position(const CompactArgs& a, int32_t v, int hh) {
+    const uint32_t bit = 1u << (v & 31);
+    for (; hh >= 0; hh--) {
+        const uint2 r = __ldcg(a.rel + hh * a.rel_stride + (v >> 5));
+        if (r.x & bit) return (int32_t)(a.counts[hh] + r.y + __popc(r.x & (bit - 1)));
+    }
+    return dev::ld_rand(a.lidx + v);
+}
 
 // Block sum of two int64 per thread (every thread gets both sums).
 __device__ __forceinline__ void block_sum2(int64_t& x, int64_t& y, int64_t (*red)[2]) {
@@ -672,8 +701,25 @@ __global__ void __launch_bounds__(kSampleTile, MOMENT_SAMPLE_MIN_BLOCKS) compact
                         }
                     }
                 }
+                if (a.rel) {
+                    // first probe (hop h, where most targets are new) for all kCopyUnroll slots in flight
+                    const uint2* rel_h = a.rel + h * a.rel_stride;
+                    uint2 r[kCopyUnroll];
 #pragma unroll
-                for (int u = 0; u < kCopyUnroll; u++) id[u] = at[u] >= 0 ? dev::ld_rand(a.lidx + id[u]) : 0;
+                    for (int u = 0; u < kCopyUnroll; u++)
+                        r[u] = at[u] >= 0 ? __ldcg(rel_h + (id[u] >> 5)) : make_uint2(0u, 0u);
+                    const int64_t Fh = a.counts[h];
+#pragma unroll
+                    for (int u = 0; u < kCopyUnroll; u++) {
+                        if (at[u] < 0) continue;
+                        const uint32_t bit = 1u << (id[u] & 31);
+                        id[u] = (r[u].x & bit) ? (int32_t)(Fh + r[u].y + __popc(r[u].x & (bit - 1)))
+                                               : rel_position(a, id[u], h - 1);
+                    }
+                } else {
+#pragma unroll
+                    for (int u = 0; u < kCopyUnroll; u++) id[u] = at[u] >= 0 ? dev::ld_rand(a.lidx + id[u]) : 0;
+                }
 #pragma unroll
                 for (int u = 0; u < kCopyUnroll; u++)
                     if (at[u] >= 0) out[at[u]] = id[u];
@@ -840,9 +886,10 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         else if (k <= 16) launch_sample_hop<16>(a, F_bound, q, stream);
         else launch_sample_hop<32>(a, F_bound, q, stream);
         const int64_t n_zero = h + 1 < H ? ca.tb[h + 2] - ca.tb[h + 1] : 0;  // the next hop's tile sums
+        uint2* rel = (ctx->rel && !ctx->sparse_scan) ? ctx->rel + (int64_t)h * ctx->rel_stride : nullptr;
         ScanArgs s{out->nodes, out->counts, ctx->lidx, ctx->newbits, ctx->visited, ctx->summary,
                    ctx->tile_status + ctx->bitscan_tiles_off[h], ctx->tickets + 1 + h, ctx->n_words, h,
-                   ctx->tile_edges + ca.tb[h + 1], n_zero};
+                   ctx->tile_edges + ca.tb[h + 1], n_zero, rel};
         if (ctx->sparse_scan) {  // one summary word (32 newbits words) per thread
             const int nt = ctx->sparse_threads;
             const int64_t tiles = (ctx->n_words + 32 * nt - 1) / (32 * nt);
@@ -868,6 +915,8 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
     ca.nodes = out->nodes;
     ca.lidx = ctx->lidx;
     ca.visited = ctx->visited;
+    ca.rel = ctx->sparse_scan ? nullptr : ctx->rel;
+    ca.rel_stride = ctx->rel_stride;
     ca.tile_edges = ctx->tile_edges;
     ca.H = H;
     const int grid = (int)std::max<int64_t>(

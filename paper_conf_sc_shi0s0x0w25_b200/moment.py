@@ -13,7 +13,7 @@ from dataclasses import dataclass
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "lib", "libmoment.so")
+LIB_PATH = os.environ.get("MOMENT_LIB_PATH") or os.path.join(_PKG, "lib", "libmoment.so")
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, EINFEASIBLE, EOVERFLOW, EUNSUPPORTED, ETIMEDOUT = 0, -1, -2, -3, -4, -5, -6, -7, -8
 CAP_INF = np.iinfo(np.int64).max
