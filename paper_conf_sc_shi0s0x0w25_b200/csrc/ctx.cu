@@ -148,6 +148,16 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     // per hop) instead of random lidx traffic over n int32 (C2: 9.8 MB per ctx)
     const bool rel_on = !c->sparse_scan && c->rank_relabel && a->max_hops > 0;
     const int64_t o_rel = rel_on ? cv.take<uint2>(n_words_pad * a->max_hops) : -1;
+    // sparse scan: two-level tables (summary-word level + one entry per word holding new ids); entries of
+    // hop h <= min(its new ids, words) <= min(max_F[h] * max_fanout[h], n_words)
+    const bool srel_on = c->sparse_scan && c->rank_relabel && a->max_hops > 0;
+    const int64_t n_summary_pad = n_words_pad / 32;
+    const int64_t o_srel = srel_on ? cv.take<uint2>(n_summary_pad * a->max_hops) : -1;
+    c->trel_off.assign(a->max_hops + 1, 0);
+    for (int h = 0; h < a->max_hops; h++)
+        c->trel_off[h + 1] = c->trel_off[h] + std::max<int64_t>(1, std::min<int64_t>(c->max_F[h] * a->max_fanout[h],
+                                                                                        n_words_pad));
+    const int64_t o_trel = srel_on ? cv.take<uint2>(c->trel_off[a->max_hops]) : -1;
     const int64_t scan_tiles = n_words_pad / kBitscanTileWords;
     c->bitscan_tiles_off.resize(a->max_hops);
     int64_t nts = 0, cnt_total = 0;
@@ -196,6 +206,9 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     c->summary = reinterpret_cast<uint32_t*>(w + o_summary);
     c->rel = rel_on ? reinterpret_cast<uint2*>(w + o_rel) : nullptr;
     c->rel_stride = n_words_pad;
+    c->srel = srel_on ? reinterpret_cast<uint2*>(w + o_srel) : nullptr;
+    c->srel_stride = n_summary_pad;
+    c->trel = srel_on ? reinterpret_cast<uint2*>(w + o_trel) : nullptr;
     c->tile_status = reinterpret_cast<uint64_t*>(w + o_tiles);
     c->tile_edges = reinterpret_cast<unsigned long long*>(w + o_tile_edges);
     c->tickets = reinterpret_cast<uint32_t*>(w + o_tickets);

@@ -48,7 +48,11 @@ struct moment_ctx_s {
     uint32_t* summary = nullptr;    // [n_words / 32]: newbits words marked at the current hop (sparse scan)
     uint2* rel = nullptr;           // dense scan: [max_hops][rel_stride] {new bits, rank} per word (rank relabel)
     int64_t rel_stride = 0;         //   words per hop (n_words padded to whole scan tiles)
-    int32_t rank_relabel = 1;       // MOMENT_RANK_RELABEL (dense scan only)
+    int32_t rank_relabel = 1;       // MOMENT_RANK_RELABEL (dense and sparse scans)
+    uint2* srel = nullptr;          // sparse scan: [max_hops][srel_stride] {word mask, first entry} per summary word
+    int64_t srel_stride = 0;
+    uint2* trel = nullptr;          // sparse scan: per hop, {new bits, rank} of the words holding new ids
+    std::vector<int64_t> trel_off;  //   hop h's entries at trel + trel_off[h] (bound: max_F[h + 1] - max_F[0])
     int64_t n_words = 0;
     // sparse scan (summary bitmap, scan cost proportional to the touched words) for large graphs: auto when
     // n_words > kSparseScanMinWords (MOMENT_SPARSE_SCAN=0/1 forces it off/on)

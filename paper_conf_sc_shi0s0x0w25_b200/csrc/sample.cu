@@ -434,6 +434,11 @@ struct ScanArgs {
     // word's first new id among the hop's new ids}, written for EVERY word (no clearing needed); lidx is then
     // not written for non-seed ids and the compaction finds an id's position from rel (L2-resident)
     uint2* rel;
+    // sparse scan with rank relabelling (else null): per summary word sw, srel[sw] = {mask of its newbits
+    // words that hold new ids, index of its first entry in trel}; trel[e] = {new-id bits, rank of the word's
+    // first new id} for the words with new ids, in id order (a second count, packed into the scan's value)
+    uint2* srel;
+    uint2* trel;
 };
 
 // F_{h+1} = F_h ++ ascending ids set in (newbits & ~visited).
@@ -551,23 +556,34 @@ __global__ void __launch_bounds__(NT) bitscan_sparse_kernel(ScanArgs a) {
         const int64_t sw = tile * NT + threadIdx.x;  // this thread's summary word
         const uint32_t sm = sw < n_summary ? __ldcg(a.summary + sw) : 0u;
         const int64_t w_base = sw * 32;
-        int cnt = 0;
-        for_touched_words(sm, a.newbits, a.visited, w_base,
-                          [&](int64_t, uint32_t nb, uint32_t vs) { cnt += __popc(nb & ~vs); });
-        int64_t agg;
-        const int64_t excl = dev::block_exclusive_scan<NT>(cnt, &agg, s_red);
-        const int64_t prefix = dev::lookback_block<NT>(a.tile_status, tile, agg, s_red, &s_nearest);
-        int64_t pos = F + prefix + excl;
-        if (tile == n_tiles - 1 && threadIdx.x == 0) a.counts[a.h + 1] = F + prefix + agg;
+        // scanned value: new ids in the low 32 bits; with rank relabelling also the words holding new ids
+        // (trel entries) in the high bits — one scan and look-back serve both prefixes
+        int64_t val = 0;
+        uint32_t emask = 0;  // words of this summary word that hold new ids
         for_touched_words(sm, a.newbits, a.visited, w_base, [&](int64_t w, uint32_t nb, uint32_t vs) {
             const uint32_t nw = nb & ~vs;
+            val += __popc(nw);
+            if (nw) emask |= 1u << (uint32_t)(w - w_base);
+        });
+        if (a.srel) val += (int64_t)__popc(emask) << 32;
+        int64_t agg;
+        const int64_t excl = dev::block_exclusive_scan<NT>(val, &agg, s_red);
+        const int64_t prefix = dev::lookback_block<NT>(a.tile_status, tile, agg, s_red, &s_nearest);
+        const int64_t before = prefix + excl;
+        int64_t pos = F + (before & 0xFFFFFFFFll);
+        int64_t ent = before >> 32;
+        if (tile == n_tiles - 1 && threadIdx.x == 0) a.counts[a.h + 1] = F + ((prefix + agg) & 0xFFFFFFFFll);
+        if (a.srel && sw < n_summary) a.srel[sw] = make_uint2(emask, (uint32_t)ent);
+        for_touched_words(sm, a.newbits, a.visited, w_base, [&](int64_t w, uint32_t nb, uint32_t vs) {
+            const uint32_t nw = nb & ~vs;
+            if (a.srel && nw) a.trel[ent++] = make_uint2(nw, (uint32_t)(pos - F));
             uint32_t bits = nw;
             while (bits) {
                 const int b = __ffs(bits) - 1;
                 bits &= bits - 1;
                 const int64_t id = w * 32 + b;
                 a.nodes[pos] = id;
-                a.lidx[id] = (int32_t)pos;
+                if (!a.srel) a.lidx[id] = (int32_t)pos;
                 pos++;
             }
             a.newbits[w] = 0u;
@@ -594,13 +610,34 @@ struct CompactArgs {
     const int32_t* cnt[kMaxHops];
     const uint2* rel;    // dense scan with rank relabelling: hop h's rel at rel + h * rel_stride, else null
     int64_t rel_stride;
+    const uint2* srel;   // sparse scan with rank relabelling: hop h's tables at srel + h * srel_stride and
+    const uint2* trel[kMaxHops];  //   trel[h], else null
+    int64_t srel_stride;
 };
+
+// Sparse scan's two-level tables: is v new at hop hh, and at which position?
+__device__ __forceinline__ bool srel_probe(const CompactArgs& a, int32_t v, int hh, int32_t* out) {
+    const uint32_t w = (uint32_t)v >> 5, j = w & 31;
+    const uint2 m = __ldcg(a.srel + hh * a.srel_stride + (w >> 5));
+    if (!((m.x >> j) & 1u)) return false;
+    const uint2 r = __ldcg(a.trel[hh] + m.y + __popc(m.x & ((1u << j) - 1u)));
+    const uint32_t bit = 1u << (v & 31);
+    if (!(r.x & bit)) return false;
+    *out = (int32_t)(a.counts[hh] + r.y + __popc(r.x & (bit - 1)));
+    return true;
+}
 
 // Position in F_{h+1} of an id sampled at hop h, from the bitscans' rel tables (rank relabelling): the id
 // is new at the latest hop hh <= h whose rel word has its bit, at counts[hh] + the word's rank + the bits
 // below it in the word; an id in no table is a seed, whose position lidx holds.
 __device__ __forceinline__ int32_t rel_position(const CompactArgs& a, int32_t v, int hh) {
     const uint32_t bit = 1u << (v & 31);
+    if (a.srel) {
+        int32_t p;
+        for (; hh >= 0; hh--)
+            if (srel_probe(a, v, hh, &p)) return p;
+        return dev::ld_rand(a.lidx + v);
+    }
     for (; hh >= 0; hh--) {
         const uint2 r = __ldcg(a.rel + hh * a.rel_stride + (v >> 5));
         if (r.x & bit) return (int32_t)(a.counts[hh] + r.y + __popc(r.x & (bit - 1)));
@@ -708,6 +745,29 @@ __global__ void __launch_bounds__(kSampleTile, MOMENT_SAMPLE_MIN_BLOCKS) compact
 #pragma unroll
                     for (int u = 0; u < kCopyUnroll; u++)
                         r[u] = at[u] >= 0 ? __ldcg(rel_h + (id[u] >> 5)) : make_uint2(0u, 0u);
+                    const int64_t Fh = a.counts[h];
+#pragma unroll
+                    for (int u = 0; u < kCopyUnroll; u++) {
+                        if (at[u] < 0) continue;
+                        const uint32_t bit = 1u << (id[u] & 31);
+                        id[u] = (r[u].x & bit) ? (int32_t)(Fh + r[u].y + __popc(r[u].x & (bit - 1)))
+                                               : rel_position(a, id[u], h - 1);
+                    }
+                } else if (a.srel) {
+                    // two dependent L2 loads per probe (summary-level then entry); 8 slots in flight
+                    const uint2* s_h = a.srel + h * a.srel_stride;
+                    uint2 m[kCopyUnroll];
+#pragma unroll
+                    for (int u = 0; u < kCopyUnroll; u++)
+                        m[u] = at[u] >= 0 ? __ldcg(s_h + ((uint32_t)id[u] >> 10)) : make_uint2(0u, 0u);
+                    uint2 r[kCopyUnroll];
+#pragma unroll
+                    for (int u = 0; u < kCopyUnroll; u++) {
+                        const uint32_t j = ((uint32_t)id[u] >> 5) & 31;
+                        r[u] = (at[u] >= 0 && ((m[u].x >> j) & 1u))
+                                   ? __ldcg(a.trel[h] + m[u].y + __popc(m[u].x & ((1u << j) - 1u)))
+                                   : make_uint2(0u, 0u);
+                    }
                     const int64_t Fh = a.counts[h];
 #pragma unroll
                     for (int u = 0; u < kCopyUnroll; u++) {
@@ -887,9 +947,12 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         else launch_sample_hop<32>(a, F_bound, q, stream);
         const int64_t n_zero = h + 1 < H ? ca.tb[h + 2] - ca.tb[h + 1] : 0;  // the next hop's tile sums
         uint2* rel = (ctx->rel && !ctx->sparse_scan) ? ctx->rel + (int64_t)h * ctx->rel_stride : nullptr;
+        uint2* srel = ctx->srel ? ctx->srel + (int64_t)h * ctx->srel_stride : nullptr;
+        uint2* trel = ctx->srel ? ctx->trel + ctx->trel_off[h] : nullptr;
         ScanArgs s{out->nodes, out->counts, ctx->lidx, ctx->newbits, ctx->visited, ctx->summary,
                    ctx->tile_status + ctx->bitscan_tiles_off[h], ctx->tickets + 1 + h, ctx->n_words, h,
-                   ctx->tile_edges + ca.tb[h + 1], n_zero, rel};
+                   ctx->tile_edges + ca.tb[h + 1], n_zero, rel, srel, trel};
+        if (srel) ca.trel[h] = trel;
         if (ctx->sparse_scan) {  // one summary word (32 newbits words) per thread
             const int nt = ctx->sparse_threads;
             const int64_t tiles = (ctx->n_words + 32 * nt - 1) / (32 * nt);
@@ -917,6 +980,8 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
     ca.visited = ctx->visited;
     ca.rel = ctx->sparse_scan ? nullptr : ctx->rel;
     ca.rel_stride = ctx->rel_stride;
+    ca.srel = ctx->srel;
+    ca.srel_stride = ctx->srel_stride;
     ca.tile_edges = ctx->tile_edges;
     ca.H = H;
     const int grid = (int)std::max<int64_t>(
