@@ -70,13 +70,16 @@ def test_sample_fanouts_and_ragged(orc, c1, fanout, n_seeds):
 
 @pytest.mark.parametrize("knob", [(("MOMENT_HOP_WARP", "0"),), (("MOMENT_INIT_KERNEL", "1"),),
                                   (("MOMENT_SPARSE_SCAN", "1"),),
-                                  (("MOMENT_SPARSE_SCAN", "1"), ("MOMENT_SPARSE_NT", "1024"))])
+                                  (("MOMENT_SPARSE_SCAN", "1"), ("MOMENT_SPARSE_NT", "1024")),
+                                  (("MOMENT_RANK_RELABEL", "0"),),
+                                  (("MOMENT_RANK_RELABEL", "0"), ("MOMENT_SPARSE_SCAN", "1"))])
 @pytest.mark.parametrize("fanout", [[15, 10, 5], [7, 3], [20], [40, 2]])
 def test_sample_kernel_variants(orc, c1, fanout, knob, monkeypatch):
     """The other sampler kernels give the same result as the default: MOMENT_HOP_WARP=0 selects the
     power-of-two lane tiles (always used for k > 32), MOMENT_INIT_KERNEL=1 a separate init kernel instead of
     the first hop's sampler initialising the call, MOMENT_SPARSE_SCAN=1 the summary-bitmap bitscan that
-    graphs above 8.4 M vertices use (C3-C5)."""
+    graphs above 8.4 M vertices use (C3-C5), MOMENT_RANK_RELABEL=0 local indices through lidx for every
+    node instead of the rank tables (dense and sparse)."""
     _, g = c1
     for k, v in knob:
         monkeypatch.setenv(k, v)
@@ -139,12 +142,14 @@ def test_sample_check_flags_bad_seeds(c1):
     assert e.value.status == M.EINVAL
 
 
-@pytest.mark.parametrize("sparse", ["0", "1"])
-def test_sample_reused_ctx_many_batches(orc, c1, sparse, monkeypatch):
-    """The workspace (lidx, bitmaps, summary bitmap, tile descriptors) is reset correctly between calls,
-    for the dense and the sparse (summary-bitmap) bitscan."""
+@pytest.mark.parametrize("sparse,relabel", [("0", "1"), ("1", "1"), ("0", "0"), ("1", "0")])
+def test_sample_reused_ctx_many_batches(orc, c1, sparse, relabel, monkeypatch):
+    """The workspace (lidx, rank tables, bitmaps, summary bitmap, tile descriptors) is reset or rewritten
+    correctly between calls, for the dense and the sparse (summary-bitmap) bitscan, with and without rank
+    relabelling."""
     cfg, g = c1
     monkeypatch.setenv("MOMENT_SPARSE_SCAN", sparse)
+    monkeypatch.setenv("MOMENT_RANK_RELABEL", relabel)
     ctx = M.Ctx(n_vertices=g.n, max_seeds=1024, max_fanout=[10, 5], device=0)
     rng = np.random.default_rng(0)
     for b in range(4):
