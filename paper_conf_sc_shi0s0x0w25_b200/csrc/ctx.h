@@ -27,10 +27,14 @@ struct moment_ctx_s {
     // L2 promotion of the gathered rows: 64 B (measured: a 400-byte row then costs 448 B of DRAM reads instead
     // of the 512 B whole 128-byte lines the default fetches; MOMENT_TMA_PROMO: 0 none, 1 64B, 2 128B, 3 256B)
     int32_t tma_promo = 1;
-    int32_t tma4_blocks_per_sm = 3;  // 1-warp gather4 blocks per SM, 4 stages of 8 x 4 rows (MOMENT_TMA4_BLOCKS)
+    int32_t tma4_blocks_per_sm = 2;  // 1-warp gather4 blocks per SM, 4 stages of 8 x 4 rows (MOMENT_TMA4_BLOCKS)
     int32_t l2_load_policy = 0, l2_store_policy = 1;  // bulk gather L2 hints: 0 normal, 1 evict_first, 2 evict_last
-    int32_t hop_grid_per_sm = 4, compact_grid_per_sm = 1;  // launch caps (MOMENT_HOP_GRID / MOMENT_COMPACT_GRID)
-    int32_t hop_nodes_per_group = 4;  // nodes per lane group on large frontiers (MOMENT_HOP_Q: 1, 2, 4, 8)
+    // launch shapes, re-tuned after rank relabelling with 16 batches in flight (C2 bench 33.5 -> 36.5 M
+    // seeds/s, C3 10.5 -> 10.9 against the earlier 4 / 1 / 4 / 3): MOMENT_HOP_GRID, MOMENT_COMPACT_GRID,
+    // MOMENT_HOP_Q, MOMENT_TMA4_BLOCKS (1 block per SM: +4 % more on C2 but the single-launch gather drops to
+    // 0.55 of the copy peak)
+    int32_t hop_grid_per_sm = 1, compact_grid_per_sm = 2;  // launch caps (blocks per SM, grid-stride beyond)
+    int32_t hop_nodes_per_group = 2;  // nodes per lane group on large frontiers (1, 2, 4, 8)
     int32_t hop_warp_segmented = 1;   // k <= 32: k-lane groups packed in a warp (MOMENT_HOP_WARP=0: 2^n tiles)
     int32_t init_in_hop0 = 1;         // the first hop's sampler also initialises the call (MOMENT_INIT_KERNEL=1: separate)
     int32_t bulk_stages = 4, bulk_blocks_per_sm = 4, bulk_stage_kb = 14;  // bulk gather shape (MOMENT_BULK="S,B,KB")
