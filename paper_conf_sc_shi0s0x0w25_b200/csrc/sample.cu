@@ -57,8 +57,8 @@ struct HopArgs {
     // this hop's edges per compaction tile (kSampleTile consecutive nodes), summed here so that the
     // compaction needs no chained scan; zeroed before the hop (hop 0: set_call, hop h: bitscan h - 1)
     unsigned long long* tile_edges;
-    // 1: every sampled id's indptr line is prefetched into L2 for the next hop (MOMENT_HOP_PREFETCH; not on
-    // the last hop)
+    // 1: every sampled id's indptr line is prefetched into L2 (evict_last) for the next hop (MOMENT_HOP_PREFETCH;
+    // not on the last hop); 2: the same without the eviction hint
     int32_t prefetch_next;
 };
 
@@ -87,7 +87,8 @@ struct InitArgs {
 __device__ __forceinline__ void mark_new(const HopArgs& a, int32_t u) {
     atomicOr(a.newbits + (u >> 5), 1u << (u & 31));
     if (a.summary) atomicOr(a.summary + (u >> 10), 1u << ((u >> 5) & 31));
-    if (a.prefetch_next) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(a.indptr + u));
+    if (a.prefetch_next == 1) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(a.indptr + u));
+    else if (a.prefetch_next == 2) asm volatile("prefetch.global.L2 [%0];" ::"l"(a.indptr + u));
 }
 
 // Floyd's k choices for node v at hop h, lane i < k owning choice i (k <= G): t_i = uniform(draw(i),
@@ -941,7 +942,7 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         const int k = p->fanout[h];
         HopArgs a{csr->indptr, csr->indices, out->nodes, out->counts, ctx->pad + pad_off, ctx->cnt + cnt_off,
                   ctx->newbits, ctx->sparse_scan ? ctx->summary : nullptr, call, h, k, replace,
-                  ctx->hop_grid_per_sm, ctx->tile_edges + ca.tb[h], (ctx->hop_prefetch > 0 || (ctx->hop_prefetch < 0 && !ctx->sparse_scan)) && h + 1 < H};
+                  ctx->hop_grid_per_sm, ctx->tile_edges + ca.tb[h], h + 1 < H ? (ctx->hop_prefetch > 0 ? ctx->hop_prefetch : (ctx->hop_prefetch < 0 && !ctx->sparse_scan)) : 0};
         const int q = ctx->hop_nodes_per_group;
         if (h == 0 && init_in_hop0) launch_sample_warp_q<1, true>(a, F_bound, stream, init);
         else if (ctx->hop_warp_segmented && k <= 32) launch_sample_warp(a, F_bound, q, stream);
