@@ -104,6 +104,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
         std::sscanf(v, "%d,%d,%d", &c->bulk_stages, &c->bulk_blocks_per_sm, &c->bulk_stage_kb);
     if (const char* v = std::getenv("MOMENT_HOP_GRID")) c->hop_grid_per_sm = std::max(1, std::atoi(v));
     if (const char* v = std::getenv("MOMENT_HOP_PREFETCH")) c->hop_prefetch = std::atoi(v);
+    if (const char* v = std::getenv("MOMENT_SCAN_PREFETCH")) c->scan_prefetch = std::atoi(v);
     if (const char* v = std::getenv("MOMENT_HOP_Q")) c->hop_nodes_per_group = std::max(1, std::atoi(v));
     if (const char* v = std::getenv("MOMENT_HOP_WARP")) c->hop_warp_segmented = std::atoi(v) != 0;
     if (const char* v = std::getenv("MOMENT_STEP_FORK")) c->step_fork = std::atoi(v) != 0;

@@ -37,6 +37,9 @@ struct moment_ctx_s {
     // L2 prefetch of the next hop's indptr lines by the sampler (MOMENT_HOP_PREFETCH=0/1; -1 = on with the dense
     // scan only: C2 36.5 -> 36.9 M seeds/s, C3 (sparse, 0.9 GB indptr) 10.85 -> 10.81, profiles/r01_hop_prefetch.txt)
     int32_t hop_prefetch = -1;
+    // dense bitscan prefetches each new id's first neighbour line (MOMENT_SCAN_PREFETCH=0/1; -1 = only when the
+    // CSR has <= 8 M edges)
+    int32_t scan_prefetch = -1;
     int32_t hop_nodes_per_group = 2;  // nodes per lane group on large frontiers (1, 2, 4, 8)
     int32_t hop_warp_segmented = 1;   // k <= 32: k-lane groups packed in a warp (MOMENT_HOP_WARP=0: 2^n tiles)
     int32_t init_in_hop0 = 1;         // the first hop's sampler also initialises the call (MOMENT_INIT_KERNEL=1: separate)

@@ -422,6 +422,10 @@ __global__ void __launch_bounds__(256, MOMENT_SAMPLE_MIN_BLOCKS) hop_sample_warp
     }
 }
 
+// the bitscan's neighbour-list prefetch pays only while the CSR is L2-sized: C1 (1 M edges, 4 MB of indices)
+// 98.7 -> 109 M seeds/s, C2 (62 M edges) 36.7 -> 35.6 (profiles/r01_hop_prefetch.txt)
+constexpr int64_t kScanPrefetchMaxEdges = int64_t(8) << 20;
+
 struct ScanArgs {
     int64_t* nodes;
     int64_t* counts;
@@ -444,6 +448,12 @@ struct ScanArgs {
     // first new id} for the words with new ids, in id order (a second count, packed into the scan's value)
     uint2* srel;
     uint2* trel;
+    // dense scan, not the last hop (else 0): each new id's CSR row start is read (its indptr line is already
+    // L2-resident from the sampler's prefetch) and the first line of its neighbour list is prefetched into L2
+    // (evict_last) for the next hop's sampler (MOMENT_SCAN_PREFETCH)
+    const int64_t* indptr;
+    const int32_t* indices;
+    int32_t prefetch_idx;
 };
 
 // F_{h+1} = F_h ++ ascending ids set in (newbits & ~visited).
@@ -499,6 +509,8 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
                 const int64_t id = w * 32 + b;
                 a.nodes[pos] = id;
                 if (!a.rel) a.lidx[id] = (int32_t)pos;
+                if (a.prefetch_idx)
+                    asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(a.indices + __ldcg(a.indptr + id)));
                 pos++;
             }
             if (nb[q]) a.newbits[w] = 0u;
@@ -956,7 +968,9 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         uint2* trel = ctx->srel ? ctx->trel + ctx->trel_off[h] : nullptr;
         ScanArgs s{out->nodes, out->counts, ctx->lidx, ctx->newbits, ctx->visited, ctx->summary,
                    ctx->tile_status + ctx->bitscan_tiles_off[h], ctx->tickets + 1 + h, ctx->n_words, h,
-                   ctx->tile_edges + ca.tb[h + 1], n_zero, rel, srel, trel};
+                   ctx->tile_edges + ca.tb[h + 1], n_zero, rel, srel, trel, csr->indptr, csr->indices,
+                   !ctx->sparse_scan && h + 1 < H &&
+                       (ctx->scan_prefetch > 0 || (ctx->scan_prefetch < 0 && csr->n_edges <= kScanPrefetchMaxEdges))};
         if (srel) ca.trel[h] = trel;
         if (ctx->sparse_scan) {  // one summary word (32 newbits words) per thread
             const int nt = ctx->sparse_threads;
