@@ -457,6 +457,9 @@ struct ScanArgs {
 };
 
 // F_{h+1} = F_h ++ ascending ids set in (newbits & ~visited).
+// kPrefetch: a separate instantiation, so the default scan's code is not touched by the prefetch branch (the
+// runtime-flag version slowed the C2 scans by ~20 % with the flag off)
+template <bool kPrefetch>
 __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
     __shared__ int64_t s_red[kBitscanThreads / 32];
     __shared__ uint32_t s_tile;
@@ -509,7 +512,7 @@ __global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
                 const int64_t id = w * 32 + b;
                 a.nodes[pos] = id;
                 if (!a.rel) a.lidx[id] = (int32_t)pos;
-                if (a.prefetch_idx)
+                if (kPrefetch)
                     asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(a.indices + __ldcg(a.indptr + id)));
                 pos++;
             }
@@ -870,7 +873,8 @@ void launch_sample_warp(const HopArgs& a, int64_t max_F, int big_q, cudaStream_t
 // Same shared-memory carveout for every kernel of the library (see configure_gather_kernels).
 moment_status configure_sample_kernels(int carveout) {
     if (carveout < 0) return MOMENT_OK;
-    const void* fns[] = {(const void*)init_kernel, (const void*)bitscan_kernel, (const void*)bitscan_sparse_kernel<256>,
+    const void* fns[] = {(const void*)init_kernel, (const void*)bitscan_kernel<false>, (const void*)bitscan_kernel<true>,
+                         (const void*)bitscan_sparse_kernel<256>,
                          (const void*)bitscan_sparse_kernel<512>, (const void*)bitscan_sparse_kernel<1024>,
                          (const void*)compact_kernel,
                          (const void*)hop_sample_kernel<4, 1>, (const void*)hop_sample_kernel<8, 1>,
@@ -980,7 +984,9 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
             else if (nt == 512) bitscan_sparse_kernel<512><<<grid, 512, 0, stream>>>(s);
             else bitscan_sparse_kernel<256><<<grid, 256, 0, stream>>>(s);
         } else {
-            bitscan_kernel<<<(int)std::min<int64_t>(n_scan_tiles, 148 * 4), kBitscanThreads, 0, stream>>>(s);
+            const int nb = (int)std::min<int64_t>(n_scan_tiles, 148 * 4);
+            if (s.prefetch_idx) bitscan_kernel<true><<<nb, kBitscanThreads, 0, stream>>>(s);
+            else bitscan_kernel<false><<<nb, kBitscanThreads, 0, stream>>>(s);
         }
         ca.k[h] = k;
         ca.kmagic[h] = k == 1 ? 0u : (uint32_t)(((uint64_t(1) << 32) + (uint64_t)k - 1) / (uint64_t)k);
