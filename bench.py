@@ -159,42 +159,108 @@ class Clocks:
                 "samples": len(sm)}
 
 
-def oracle_baseline(name, budget_s=15.0, seeds_cap=None, state=None):
-    """Time the CPU oracle (as it stands, single-threaded) on a bounded sample of the workload."""
+def host_info():
+    """CPU model, logical core count and one NUMA-0 core for the single-threaded oracle."""
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name:"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    allowed = sorted(os.sched_getaffinity(0))
+    node0 = None
+    try:
+        with open("/sys/devices/system/node/node0/cpulist") as f:
+            node0 = set()
+            for part in f.read().strip().split(","):
+                a, _, b = part.partition("-")
+                node0.update(range(int(a), int(b or a) + 1))
+    except Exception:
+        node0 = None
+    cand = [c for c in allowed if node0 is None or c in node0] or allowed
+    # the last allowed core of NUMA node 0 (core 0 tends to take the interrupts)
+    return {"cpu_model": model, "os_cpu_count": os.cpu_count(), "allowed_cores": len(allowed),
+            "core": cand[-1], "core_numa0": node0 is not None and cand[-1] in node0}
+
+
+class PinnedCore:
+    """Pin the calling thread to one core (the oracle's C code runs on it; `taskset -c core` in-process)."""
+
+    def __init__(self, core):
+        self.core = core
+
+    def __enter__(self):
+        self.old = os.sched_getaffinity(0)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *exc):
+        os.sched_setaffinity(0, self.old)
+
+
+def parity_subset(n_batches: int) -> list[int]:
+    """the first 2 batches of the rank + 1 batch chosen by a counter hash."""
+    first = list(range(min(2, n_batches)))
+    if n_batches > 2:
+        j = 2 + W.mix(RUN_SEED, 0xC0FFEE) % (n_batches - 2)
+        first.append(int(j))
+    return first
+
+
+def oracle_baseline(st, pool, budget_s=10.0):
+    """The CPU oracle as it stands (oracle/, single-threaded C, pinned to one NUMA-0 core) on a bounded
+    sample of the bench's own batches: first the parity subset, each of which is also compared
+    bit-exactly with the CUDA path's output for the same batch, then further batches of the pool until
+    `budget_s` seconds of oracle time have been spent."""
     import oracle
 
     oracle.build()
-    cfg = W.CONFIGS[name]
-    if state is not None:
-        indptr = state.graph.indptr.cpu().numpy()
-        indices = state.graph.indices.cpu().numpy()
-        table = np.ascontiguousarray(state.table[:, :state.R].cpu().numpy())
-        train = state.train.cpu()
-    else:
-        g = W.rmat_csr(cfg["n"], cfg["m"], device="cpu")
-        indptr, indices = g.indptr.numpy(), g.indices.numpy()
-        table = W.feature_table(cfg["n"], cfg["dim"], cfg["dtype"], device="cpu").numpy()
-        train = W.training_set(g, min_count=cfg["batch"])
-    batches = W.epoch_batches(train, cfg["batch"], 0)
-    fan = list(cfg["fanout"])
-    # calibrate on a small slice, then size the sample to the budget
-    t0 = time.perf_counter()
-    r = oracle.sample(indptr, indices, batches[0][:16].numpy(), fan, 1)
-    oracle.gather(table, r["nodes"])
-    per_seed = (time.perf_counter() - t0) / 16
-    n = int(max(16, min(seeds_cap or cfg["batch"], budget_s / max(per_seed, 1e-9))))
-    done, t = 0, 0.0
-    i = 0
-    while done < n:
-        seeds = batches[i % len(batches)][: min(cfg["batch"], n - done)].numpy()
-        t0 = time.perf_counter()
-        r = oracle.sample(indptr, indices, seeds, fan, W.batch_rng_seed(RUN_SEED, 0, 0, i))
-        oracle.gather(table, r["nodes"])
-        t += time.perf_counter() - t0
-        done += len(seeds)
-        i += 1
-    return {"value": done / t, "unit": "seeds/s", "cores": 1, "kind": "oracle",
-            "sample": f"{done} seeds of {name} ({i} batch slices of <= {cfg['batch']}), sample + gather, single thread"}
+    info = host_info()
+    H = len(st.fanout)
+    indptr = st.graph.indptr.cpu().numpy()
+    indices = st.graph.indices.cpu().numpy()
+    table = np.ascontiguousarray(st.table[:, :st.R].cpu().numpy())
+    fan = list(st.fanout)
+    subset = parity_subset(len(pool))
+    # the parity subset first, then the pool in order, cycled until the budget is spent
+    order = subset + [i % len(pool) for i in range(100 * len(pool)) if i >= len(pool) or i not in subset]
+    t, seeds_done, n_b, checked = 0.0, 0, 0, []
+    L = st.lanes[0]
+    with PinnedCore(info["core"]):
+        for i in order:
+            seeds, rs = pool[i]
+            s_np = seeds.cpu().numpy()
+            t0 = time.perf_counter()
+            r = oracle.sample(indptr, indices, s_np, fan, rs)
+            rows = oracle.gather(table, r["nodes"])
+            t += time.perf_counter() - t0
+            seeds_done += len(s_np)
+            n_b += 1
+            if i in subset and i not in checked:
+                # the CUDA path on the same batch (lane 0): every output compared, rows in full
+                st.step(seeds, rs, lane=0)
+                torch.cuda.synchronize()
+                got = L.bufs.result()
+                nF = int(r["counts"][H])
+                ok = (np.array_equal(got["counts"], r["counts"]) and np.array_equal(got["nodes"], r["nodes"])
+                      and all(np.array_equal(got["offsets"][h], r["offsets"][h]) and
+                              np.array_equal(got["src"][h], r["src"][h]) for h in range(H))
+                      and np.array_equal(L.rows[:nF].cpu().numpy(), rows.view(np.uint8).reshape(nF, -1)))
+                if not ok:
+                    raise AssertionError(f"bench batch {i}: CUDA path differs from the oracle")
+                checked.append(i)
+            if t >= budget_s and len(checked) == len(subset):
+                break
+    return {"value": seeds_done / t, "unit": "seeds/s", "cores": 1, "kind": "oracle",
+            "sample": f"{n_b} batches x {st.B} seeds of {st.name} (the bench's own batches: parity subset "
+                      f"{subset} first, then the pool in order, cycled, until {budget_s:g} s), sample + gather, "
+                      f"single thread pinned to core {info['core']}",
+            "host": info,
+            "parity": {"batches": checked, "bit_exact": True,
+                       "compared": "counts, F_H, per-hop offsets and src, every gathered row byte"}}
 
 
 def profile_summary(name):
@@ -213,6 +279,8 @@ def profile_traffic(name):
 
 
 def run_reference(args, rank, world):
+    """The tier's reference arm: the CPU oracle as it stands, on the host cores, same config/metric/unit.
+    Under torchrun only rank 0 works; the other ranks exit 0."""
     if rank != 0:
         return
     cfg = W.CONFIGS[args.config]
@@ -222,27 +290,29 @@ def run_reference(args, rank, world):
     import oracle
 
     oracle.build()
+    info = host_info()
     g = W.rmat_csr(cfg["n"], cfg["m"], device="cpu")
     indptr, indices = g.indptr.numpy(), g.indices.numpy()
     table = W.feature_table(cfg["n"], cfg["dim"], cfg["dtype"], device="cpu").numpy()
     train = W.training_set(g, min_count=cfg["batch"])
     batches = W.epoch_batches(train, cfg["batch"], 0)
     fan = list(cfg["fanout"])
-    t0 = time.perf_counter()
-    r = oracle.sample(indptr, indices, batches[0][:16].numpy(), fan, 1)
-    oracle.gather(table, r["nodes"])
-    per_seed = (time.perf_counter() - t0) / 16
-    s_per_step = int(max(1, min(cfg["batch"], budget / max(total_steps, 1) / max(per_seed, 1e-9))))
-    t_meas, seeds_done = 0.0, 0
-    for i in range(total_steps):
-        seeds = batches[i % len(batches)][:s_per_step].numpy()
+    with PinnedCore(info["core"]):
         t0 = time.perf_counter()
-        r = oracle.sample(indptr, indices, seeds, fan, W.batch_rng_seed(RUN_SEED, 0, 0, i))
+        r = oracle.sample(indptr, indices, batches[0][:16].numpy(), fan, 1)
         oracle.gather(table, r["nodes"])
-        dt = time.perf_counter() - t0
-        if i >= args.warmup:
-            t_meas += dt
-            seeds_done += len(seeds)
+        per_seed = (time.perf_counter() - t0) / 16
+        s_per_step = int(max(1, min(cfg["batch"], budget / max(total_steps, 1) / max(per_seed, 1e-9))))
+        t_meas, seeds_done = 0.0, 0
+        for i in range(total_steps):
+            seeds = batches[i % len(batches)][:s_per_step].numpy()
+            t0 = time.perf_counter()
+            r = oracle.sample(indptr, indices, seeds, fan, W.batch_rng_seed(RUN_SEED, 0, 0, i))
+            oracle.gather(table, r["nodes"])
+            dt = time.perf_counter() - t0
+            if i >= args.warmup:
+                t_meas += dt
+                seeds_done += len(seeds)
     val = seeds_done / t_meas
     line = {"metric": METRIC, "value": val, "unit": "seeds/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1000 * t_meas / max(args.steps, 1), "higher_is_better": True,
@@ -252,23 +322,43 @@ def run_reference(args, rank, world):
             "impl": "reference",
             "cpu_baseline": {"value": val, "unit": "seeds/s", "cores": 1, "kind": "oracle",
                              "sample": f"{s_per_step} seeds per step x {args.steps} steps of {args.config}, "
-                                       "sample + gather"},
+                                       f"sample + gather, single thread pinned to core {info['core']}",
+                             "host": info},
             "e2e": {"value": val, "unit": "seeds/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def spawn_ranks(n):
+    """`bench.py --gpus N` outside torchrun: re-launch this command under torch.distributed.run, one rank per
+    GPU on 127.0.0.1 (the driver's own N>1 launch sets WORLD_SIZE and never reaches this)."""
+    import socket
+
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    os.execv(sys.executable, cmd)
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20000)  # ~1 s timed: nvidia-smi samples the clocks in it
-    ap.add_argument("--warmup", type=int, default=50)
+    ap.add_argument("--steps", type=int, default=200, help="K: steps per timed region (exactly K batches per GPU)")
+    ap.add_argument("--warmup", type=int, default=5, help="W: untimed warm-up steps per in-flight lane")
+    ap.add_argument("--min-time", type=float, default=1.0,
+                    help="seconds of timed regions: the K-step region is repeated (each bracketed by barrier + "
+                         "synchronize) until this much device time is covered, and the median region is reported")
+    ap.add_argument("--e2e-min-time", type=float, default=0.5)
     ap.add_argument("--config", default="C2")
     ap.add_argument("--impl", default="moment", choices=["moment", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=4000)
+    ap.add_argument("--cpu-budget", type=float, default=10.0, help="seconds of oracle time for cpu_baseline")
     # 12-16 measured best on C2 (29.5-29.7 M seeds/s vs 27.7 at 8, 28.4 at 24)
     ap.add_argument("--inflight", type=int, default=16, help="batches in flight per GPU (one stream each)")
     args = ap.parse_args()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        spawn_ranks(args.gpus)
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -276,11 +366,14 @@ def main():
         run_reference(args, rank, world)
         return
     assert args.warmup >= 3, "W >= 3 warm-up steps"
+    assert args.steps >= 1
     # MOMENT_BENCH_SHARED_GPU=1 (test only): every rank on cuda:0 with a gloo group, to exercise the
     # multi-rank code path on a one-GPU box (NCCL refuses two ranks on one device). Never a bench number.
     shared = os.environ.get("MOMENT_BENCH_SHARED_GPU") == "1"
     if shared:
         local = 0
+    elif world > torch.cuda.device_count():
+        raise SystemExit(f"bench.py: {world} ranks but only {torch.cuda.device_count()} visible GPUs")
     torch.cuda.set_device(local)
     dev = f"cuda:{local}"
     dist = None
@@ -291,9 +384,10 @@ def main():
             dist.init_process_group("gloo")
         else:
             dist.init_process_group("nccl", device_id=torch.device(dev))
-    st = build_state(args.config, dev, rank, world, args.inflight)
+    P = max(1, min(args.inflight, args.steps))
+    st = build_state(args.config, dev, rank, world, P)
     H = len(st.fanout)
-    P = len(st.lanes)
+    K = args.steps
     main_stream = torch.cuda.current_stream()
 
     def fork(ev):
@@ -306,40 +400,93 @@ def main():
             e.record(L.stream)
             main_stream.wait_event(e)
 
-    batches = [st.batch(args.warmup + i) for i in range(args.steps)]
-    clocks = Clocks(local)  # sampled from the warm-up (also under load) through the timed region
-    for i in range(args.warmup):
-        st.step(*st.batch(i), lane=i % P)
-    torch.cuda.synchronize()
-    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-           for _ in range(min(args.steps, 1000))]
-    if dist:
-        dist.barrier()
-    torch.cuda.synchronize()
-    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    t_start.record(main_stream)
-    fork(t_start)
-    for i in range(args.steps):
-        st.step(*batches[i], lane=i % P)
-    join()
-    t_end.record(main_stream)
-    torch.cuda.synchronize()
-    if dist:
-        dist.barrier()
+    def barrier():
+        torch.cuda.synchronize()
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    # the batches: a pool of distinct batches of this rank (cycled epochs), timed steps cycle through it
+    n_pool = max(64, min(K, 1024))
+    pool = [st.batch(args.warmup * P + i) for i in range(n_pool)]
+    warm = [st.batch(i) for i in range(args.warmup * P)]
+    clocks = Clocks(local)  # sampled from the warm-up (also under load) through the timed regions
+    # W warm-up steps on every lane (each lane's first step captures its CUDA graph)
+    for i, b in enumerate(warm):
+        st.step(*b, lane=i % P)
+    barrier()
+
+    def region(step_fn, first):
+        """One timed region: exactly K steps, barrier + synchronize on both sides, device time (ms)."""
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(main_stream)
+        fork(e0)
+        for j in range(K):
+            step_fn(first + j, j % P)
+        join()
+        e1.record(main_stream)
+        barrier()
+        return e0.elapsed_time(e1)
+
+    def repeats(step_fn, min_time):
+        times, t, r = [], 0.0, 0
+        while True:
+            ms_ = region(step_fn, r * K)
+            times.append(ms_)
+            t += ms_
+            r += 1
+            done = r >= 3 and t >= min_time * 1000
+            if dist:
+                # every rank runs the same number of regions: rank 0 decides
+                flag = torch.tensor([int(done)], device=dev if not shared else "cpu")
+                dist.broadcast(flag, 0)
+                done = bool(int(flag))
+            if done:
+                break
+        tt = torch.tensor(times, dtype=torch.float64, device=dev if not shared else "cpu")
+        if dist:
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)  # per region, the slowest rank
+        return tt.cpu().tolist()
+
+    def dev_step(i, lane):
+        b = pool[i % n_pool]
+        st.step(b[0], b[1], lane=lane)
+
+    reg_ms = repeats(dev_step, args.min_time)
     ck = clocks.stop()
-    ms = t_start.elapsed_time(t_end)
-    # roofline pass over (the first 1000 of) the same batches: CUDA events around the dominant kernel (the
-    # gather) on its stream, one lane; then |F_H| of every timed step (deterministic, so identical to the
-    # timed run), collected on the device and read once
-    n_roof = min(args.steps, 1000)
+    n_regions = len(reg_ms)
+    ms = statistics.median(reg_ms)
+    # |F_H| of every pool batch (deterministic: identical to the timed steps), collected on the device
+    L0 = st.lanes[0]
+    cnt_dev = torch.empty((n_pool, 2 * H + 1), dtype=torch.int64, device=dev)
+    for i in range(n_pool):
+        L0.ctx.step(st.graph.indptr, st.graph.indices, pool[i][0], st.fanout, pool[i][1], L0.bufs, None,
+                    stream=main_stream)
+        cnt_dev[i].copy_(L0.bufs.counts)
+    cnt_pool = cnt_dev.cpu().tolist()
+    nF_pool = [c[H] for c in cnt_pool]
+    med_r = min(range(n_regions), key=lambda r: abs(reg_ms[r] - ms))
+    used = [(med_r * K + j) % n_pool for j in range(K)]
+    nF_region = sum(nF_pool[i] for i in used)
+    # algorithmic HBM bytes of a step (SURVEY 8(d)): sampling = sum_{h<H} 16 |F_h| (indptr pair) + sum_h 8 E_h
+    # (index read + src write) + 8 |F_H| (ids written); gather = |F_H| (8 placement/id + R read + R written)
+    samp_bytes = sum(sum(16 * c[h] for h in range(H)) + sum(8 * e for e in c[H + 1:]) + 8 * c[H]
+                     for c in (cnt_pool[i] for i in used))
+    gath_bytes = nF_region * (2 * st.R + 8)
+    # roofline pass: CUDA events around the dominant kernel (the gather) on its stream, one lane, one batch
+    # at a time, over the pool
+    n_roof = min(n_pool, 256)
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n_roof)]
     for i in range(n_roof):
-        st.step(*batches[i], ev=evs[i], lane=0)
+        st.step(*pool[i], ev=evs[i], lane=0)
     torch.cuda.synchronize()
-    gather_ms = sum(a.elapsed_time(b) for a, b in evs[:n_roof]) / n_roof
+    gather_ms = sum(a.elapsed_time(b) for a, b in evs) / n_roof
+    nF_roof = nF_pool[:n_roof]
     # supplementary: the same gather kernel issued back to back (P sampled batches, one per lane, gathered in
-    # rounds on one stream; 8 x 48 MB per round > L2), so launch latency overlaps the previous launch
+    # rounds on one stream; > L2 per round), so launch latency overlaps the previous launch
     for i, L in enumerate(st.lanes):
-        s_, r_ = batches[i % len(batches)]
+        s_, r_ = pool[i % n_pool]
         L.ctx.sample(st.graph.indptr, st.graph.indices, s_, st.fanout, r_, L.bufs, stream=main_stream)
     torch.cuda.synchronize()
     nF_b2b = sum(int(L.bufs.counts[H]) for L in st.lanes) / P
@@ -354,8 +501,7 @@ def main():
     torch.cuda.synchronize()
     gather_ms_b2b = e_b0.elapsed_time(e_b1) / (rounds * P)
     # supplementary: the same gathers with the P lanes' launches concurrent (one stream per lane, as in the
-    # timed region but without the sampling kernels): whole-GPU throughput of the kernel once the ramp and
-    # tail of one launch overlap the others'
+    # timed region but without the sampling kernels)
     e_c0, e_c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e_c0.record(main_stream)
     fork(e_c0)
@@ -367,84 +513,75 @@ def main():
     e_c1.record(main_stream)
     torch.cuda.synchronize()
     gather_ms_conc = e_c0.elapsed_time(e_c1) / (rounds * P)
-    nF_roof = []
-    for i in range(n_roof):
-        st.step(*batches[i], lane=0)
-        nF_roof.append(int(st.lanes[0].bufs.counts[H]))
-    L0 = st.lanes[0]
-    nf_dev = torch.empty(args.steps, dtype=torch.int64, device=dev)
-    for i in range(args.steps):
-        L0.ctx.step(st.graph.indptr, st.graph.indices, batches[i][0], st.fanout, batches[i][1], L0.bufs, None,
-                    stream=main_stream)
-        nf_dev[i:i + 1].copy_(L0.bufs.counts[H:H + 1])
-    nF = nf_dev.cpu().tolist()
     if dist:
-        t = torch.tensor([ms], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t)
-        tot = torch.tensor([float(sum(nF))], device=dev)
+        tot = torch.tensor([float(nF_region)], dtype=torch.float64, device=dev if not shared else "cpu")
         dist.all_reduce(tot)
         nF_total = float(tot)
     else:
-        nF_total = float(sum(nF))
-    seeds_per_s = world * st.B * args.steps / (ms / 1000)
+        nF_total = float(nF_region)
+    seeds_per_s = world * st.B * K / (ms / 1000)
     gather_gbs = nF_total * st.R / (ms / 1000) / 1e9
     # roofline of the dominant kernel (gather): algorithmic bytes = |F_H| (R read + R write + 8 id)
     alg_bytes = (sum(nF_roof) / n_roof) * (2 * st.R + 8)
     peak, peak_kind = _peaks()
     achieved = alg_bytes / (gather_ms / 1000) / 1e9
-    # e2e: the same steps through the C ABI with host buffers: pinned seeds H2D and counts D2H every step,
-    # P steps in flight (one per lane), all copies inside the timed region
-    n_e2e = max(3, args.e2e_steps)
-    seeds_pinned = torch.empty((n_e2e, st.B), dtype=torch.int64).pin_memory()
-    for i in range(n_e2e):
-        seeds_pinned[i].copy_(batches[i % len(batches)][0])
-    seeds_h = list(seeds_pinned)
-    counts_pinned = torch.zeros((n_e2e, 2 * H + 1), dtype=torch.int64).pin_memory()
-    counts_h = list(counts_pinned)
-    for i in range(3):
-        st.step_host(seeds_h[i], batches[i][1], counts_h[i], lane=i % P)
+    # e2e: the same K-step regions through the C ABI with HOST buffers: each step's seeds copied H2D from
+    # pinned memory and its counts read back D2H (moment_step_host), all copies inside the timed region
+    seeds_pinned = torch.empty((n_pool, st.B), dtype=torch.int64).pin_memory()
+    for i in range(n_pool):
+        seeds_pinned[i].copy_(pool[i][0])
+    counts_pinned = torch.zeros((K, 2 * H + 1), dtype=torch.int64).pin_memory()
+    for i in range(P):
+        st.step_host(seeds_pinned[i], pool[i][1], counts_pinned[i % K], lane=i)
     torch.cuda.synchronize()
-    if dist:
-        dist.barrier()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(main_stream)
-    fork(e0)
-    for i in range(args.e2e_steps):
-        st.step_host(seeds_h[i], batches[i][1], counts_h[i], lane=i % P)
-    join()
-    e1.record(main_stream)
-    torch.cuda.synchronize()
-    e2e_ms = e0.elapsed_time(e1)
-    assert all(int(c[H]) > 0 for c in counts_h[: args.e2e_steps])
-    if dist:
-        t = torch.tensor([e2e_ms], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_ms = float(t)
-    e2e_val = world * st.B * args.e2e_steps / (e2e_ms / 1000)
+
+    def host_step(i, lane):
+        st.step_host(seeds_pinned[i % n_pool], pool[i % n_pool][1], counts_pinned[i % K], lane=lane)
+
+    e2e_ms_all = repeats(host_step, args.e2e_min_time)
+    e2e_ms = statistics.median(e2e_ms_all)
+    # the last region's counts: every step's |F_H| read back equals the device path's
+    last = len(e2e_ms_all) - 1
+    for j in range(K):
+        assert int(counts_pinned[j][H]) == nF_pool[(last * K + j) % n_pool], "e2e counts differ from the device path"
+    e2e_val = world * st.B * K / (e2e_ms / 1000)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = oracle_baseline(args.config, state=st)
+        cpu = oracle_baseline(st, pool, args.cpu_budget)
     if rank == 0:
         line = {
-            "metric": METRIC, "value": seeds_per_s, "unit": "seeds/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
+            "metric": METRIC, "value": seeds_per_s, "unit": "seeds/s", "n_gpus": world, "steps": K,
+            "warmup": args.warmup, "ms_per_step": ms / K, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u8", "data": "synthetic",
             "config": {"workload": args.config, "desc": st.cfg["desc"], "global_batch": st.B * world,
                        "fanout": list(st.fanout), "row_bytes": st.R, "inflight_batches_per_gpu": P,
-                       "parallelism": f"dp{world} (replicated graph+features)",
-                       "l2": "inputs larger than L2 (features %.2f GB, CSR %.2f GB)" % (
+                       "parallelism": f"dp{world} (replicated graph+features, seeds sharded)",
+                       "timing": f"each timed region = exactly {K} steps per GPU (barrier + synchronize on both "
+                                 f"sides, CUDA events, max over ranks); {n_regions} regions (>= {args.min_time:g} s "
+                                 f"of device time, so nvidia-smi samples the clocks inside them), median reported; "
+                                 f"warm-up {args.warmup} steps on each of the {P} lanes",
+                       "region_ms": {"median": ms, "min": min(reg_ms), "max": max(reg_ms), "n": n_regions},
+                       "l2": "no flush: inputs larger than L2 (features %.2f GB, CSR %.2f GB)" % (
                            st.table.numel() / 1e9, (st.graph.indptr.numel() * 8 + st.graph.indices.numel() * 4) / 1e9),
-                       "mean_F_H": sum(nF) / args.steps,
+                       "mean_F_H": nF_region / K,
                        **({"test_mode": "all ranks share cuda:0 over gloo: not a bench number"} if shared else {})},
             "gather_GBs": gather_gbs,
+            "step_roofline": {"bound": "hbm", "alg_bytes_per_step": (samp_bytes + gath_bytes) / K,
+                              "sampling_bytes_per_step": samp_bytes / K, "gather_bytes_per_step": gath_bytes / K,
+                              "achieved": (samp_bytes + gath_bytes) / K / (ms / K / 1000) / 1e9, "peak": peak,
+                              "unit": "GB/s",
+                              "frac": (samp_bytes + gath_bytes) / K / (ms / K / 1000) / 1e9 / peak,
+                              "how": "whole step (all 8(a) rows H1-H6): algorithmic bytes of the median region's "
+                                     "batches / its device time, per GPU"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": profile_traffic(args.config), "kernel": "gather_tma4_kernel",
                          "launch_shares": profile_summary(args.config).get("launch_shares"),
                          "why_this_kernel": profile_summary(args.config).get("why_gather"),
                          "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})",
                          "alg_bytes_per_launch": alg_bytes, "launch_ms": gather_ms,
-                         "gather_share_of_step": gather_ms / (ms / args.steps),
+                         "how": f"CUDA events on the gather's stream around each of {n_roof} launches (one batch "
+                                "at a time, lane 0), mean duration",
+                         "gather_share_of_step": gather_ms / (ms / K),
                          "back_to_back": {
                              "launch_ms": gather_ms_b2b,
                              "achieved": nF_b2b * (2 * st.R + 8) / (gather_ms_b2b / 1000) / 1e9,
@@ -459,8 +596,14 @@ def main():
                                     "timed region, sampling absent): time per launch of the whole-GPU throughput"}},
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_val, "unit": "seeds/s", "h2d_bytes_per_step": st.B * 8,
-                    "d2h_bytes_per_step": (2 * H + 1) * 8},
-            "gpu_launches": st.launches_per_step() * args.steps,
+                    "d2h_bytes_per_step": (2 * H + 1) * 8,
+                    "api": "moment_step_host (C ABI) per step, same K-step regions, median of "
+                           f"{len(e2e_ms_all)}",
+                    "copies_declared": "H2D: the step's 1024 int64 seeds from pinned host memory; D2H: the "
+                                       "step's counts (|F_0..F_H|, E_0..E_{H-1}) into pinned memory. F_H, offsets, "
+                                       "src and the gathered rows stay in HBM for the on-GPU consumer (the GNN "
+                                       "layer, sage.py) and are not copied to the host"},
+            "gpu_launches": st.launches_per_step() * K,
             "clocks": ck,
         }
         print(json.dumps(line), flush=True)

@@ -1,0 +1,44 @@
+"""bench.py end to end with the driver's own argument shapes (`--steps 20 --warmup 5` crashed
+after the timed region). The reference arm runs on CPU; the CUDA arm needs a GPU."""
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _run(args, env=None, timeout=900):
+    e = dict(os.environ)
+    e.update(env or {})
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py")] + args, capture_output=True, text=True,
+                       timeout=timeout, cwd=ROOT, env=e)
+    assert r.returncode == 0, r.stderr[-4000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    return json.loads(lines[0])
+
+
+def test_reference_arm_driver_args():
+    line = _run(["--impl", "reference", "--config", "C1", "--gpus", "1", "--steps", "20", "--warmup", "5"],
+                env={"MOMENT_REF_BUDGET_S": "3"})
+    assert line["impl"] == "reference" and line["steps"] == 20 and line["warmup"] == 5
+    assert line["value"] > 0 and line["unit"] == "seeds/s"
+    assert line["e2e"]["h2d_bytes_per_step"] == 0 and line["cpu_baseline"]["kind"] == "oracle"
+    assert line["cpu_baseline"]["cores"] == 1
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("steps,warmup", [(20, 5), (1, 3), (3, 3)])
+def test_bench_driver_args_c1(steps, warmup):
+    line = _run(["--config", "C1", "--gpus", "1", "--steps", str(steps), "--warmup", str(warmup), "--min-time", "0.2",
+                 "--e2e-min-time", "0.1", "--cpu-budget", "1"])
+    assert line["steps"] == steps and line["warmup"] == warmup and line["n_gpus"] == 1
+    assert line["value"] > 0 and line["e2e"]["value"] > 0
+    for k in ("roofline", "cpu_baseline", "e2e", "clocks", "gpu_launches", "step_roofline"):
+        assert line[k] is not None, k
+    assert 0 < line["roofline"]["frac"] < 1.5
+    assert line["cpu_baseline"]["parity"]["bit_exact"]
+    assert line["config"]["region_ms"]["n"] >= 3
