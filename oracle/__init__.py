@@ -73,6 +73,10 @@ def _setup(L):
     L.orc_time_bisect.restype = C.c_int
     L.orc_plan_closed_forms.argtypes = [I32, I32, P, P, P, I64, I64, I64, P, P]
     L.orc_plan_closed_forms.restype = C.c_int
+    L.orc_quota.argtypes = [I32, I32, P, P, P, I32, I32, I32, P, P]
+    L.orc_quota.restype = C.c_int
+    L.orc_hash_place.argtypes = [I64, I32, P, P, P, P]
+    L.orc_hash_place.restype = C.c_int
     L.orc_bucket.argtypes = [I32, I32, I32, P, P, P, I64, P, P, P]
     L.orc_bucket.restype = C.c_int
     L.orc_ddak.argtypes = [I64, P, I32, P, P, P, I64, P, P, P, P]
@@ -212,6 +216,34 @@ def plan_closed_forms(k: int, hbm_owner, d, x, nvlink_cap: int, hbm_cap: int, re
     if st != OK:
         raise OracleError(st, "plan_closed_forms")
     return int(tn[0]), int(th[0])
+
+
+def quota(n_nodes: int, links, flow, s: int, t: int, gpu_nodes):
+    """Path decomposition of a given ingest flow (R11): x[n_nodes][k], k = len(gpu_nodes) (rank order)."""
+    fr = _c([l[0] for l in links], np.int32)
+    to = _c([l[1] for l in links], np.int32)
+    fl = _c(flow, np.int64)
+    k = len(gpu_nodes)
+    rank = np.full(n_nodes, -1, np.int32)
+    for r, v in enumerate(gpu_nodes):
+        rank[v] = r
+    x = np.zeros((n_nodes, k), np.int64)
+    st = lib().orc_quota(n_nodes, len(links), _p(fr), _p(to), _p(fl), s, t, k, _p(rank), _p(x))
+    if st != OK:
+        raise OracleError(st, "quota")
+    return x
+
+
+def hash_place(n: int, cap_rows):
+    """Hash-partitioning baseline (R24): (bin_of int32[n], slot_of int64[n], used int64[n_bins])."""
+    cap = _c(cap_rows, np.int64)
+    bin_of = np.full(max(n, 1), -1, np.int32)
+    slot_of = np.full(max(n, 1), -1, np.int64)
+    used = np.zeros(len(cap), np.int64)
+    st = lib().orc_hash_place(n, len(cap), _p(cap), _p(bin_of), _p(slot_of), _p(used))
+    if st != OK:
+        raise OracleError(st, "hash_place")
+    return bin_of[:n], slot_of[:n], used
 
 
 def bucket(g: int, k: int, hbm_owner, x, bin_of_id):

@@ -18,7 +18,9 @@
  *   orc_maxflow .............. Edmonds-Karp on the capacity graph (§3.2 LP) (R7-R9)
  *   orc_time_bisect .......... minimum integer time T* meeting the sinks' demand (R10)
  *   orc_plan_closed_forms .... NVLink / HBM closed-form times of the ingest plan (R11)
+ *   orc_quota ................ ingest quotas x[j][h]: path decomposition of a given ingest flow (R11)
  *   orc_bucket ............... per-request routing by placement + quota (R12)
+ *   orc_hash_place ........... the hash-partitioning baseline placement (R24)
  *   orc_ddak ................. data-distribution-aware knapsack, Eq. 2 (R13-R17)
  *   orc_ddak_replicate ....... the same with the r hottest rows replicated in every GPU bin (R25)
  *   orc_sage_mean(_backward) . GraphSAGE mean aggregation over a sampled block and its adjoint (Eq. 1)
@@ -424,6 +426,113 @@ int orc_plan_closed_forms(int32_t k, int32_t n_bins, const int32_t* hbm_owner, c
     *t_nvlink = max_link == 0 ? 0 : ceil_div_u128((unsigned __int128)max_link, (unsigned __int128)nvlink_cap);
     if (hbm_cap <= 0) return ORC_EINVAL;
     *t_hbm = ceil_div_u128((unsigned __int128)max_hbm, (unsigned __int128)hbm_cap);
+    return ORC_OK;
+}
+
+/* ------------------------------------------------------------------------------------------------
+ * Ingest quotas ("time-bisection Ford-Fulkerson"; the paper does not say how the single-
+ * commodity flow becomes per-GPU routing, R11). x[j][h] = bytes of host bin j that enter through GPU
+ * h's port = a path decomposition of the GIVEN ingest flow f (flows are not unique, so the quotas are a
+ * function of the flow the planner produced). The decomposition is the textbook one (follow positive
+ * flow from the source, cancel any cycle met on the way), in this fixed order:
+ *   for every supply link s -> j in link order, while its remaining flow is > 0:
+ *     walk from j; at node u:
+ *       if u is an active GPU (rank_of_node[u] >= 0) and one of its links into t has remaining flow
+ *         (the first such in link order), the walk ends there;
+ *       else follow the first out-link of u in link order (not into t) with remaining flow;
+ *       if that link leads back to a node w already on the walk, the closed cycle (the walk's links
+ *         from w on, plus this link) loses its minimum remaining flow on every link, the walk is cut
+ *         back to w, and it resumes from w;
+ *     m = minimum remaining flow over the supply link and the walk's links; subtract m from each;
+ *     x[j][rank of the walk's last GPU] += m.
+ * x is [n_nodes][k] (rows of non-host nodes stay 0). Returns ORC_EINVAL if the flow is not
+ * conserved (a walk gets stuck).
+ * ------------------------------------------------------------------------------------------------ */
+int orc_quota(int32_t n_nodes, int32_t n_links, const int32_t* from, const int32_t* to, const int64_t* flow,
+              int32_t s, int32_t t, int32_t k, const int32_t* rank_of_node, int64_t* x) {
+    if (n_nodes <= 0 || n_links < 0 || k <= 0) return ORC_EINVAL;
+    int64_t* rem = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n_links > 0 ? n_links : 1));
+    int32_t* walk = (int32_t*)malloc(sizeof(int32_t) * (size_t)(n_links + 1)); /* link indices */
+    int32_t* at = (int32_t*)malloc(sizeof(int32_t) * (size_t)n_nodes);         /* position on walk or -1 */
+    if (!rem || !walk || !at) { free(rem); free(walk); free(at); return ORC_ENOMEM; }
+    for (int32_t e = 0; e < n_links; e++) rem[e] = flow[e];
+    for (int64_t i = 0; i < (int64_t)n_nodes * k; i++) x[i] = 0;
+    int rc = ORC_OK;
+    for (int32_t e0 = 0; e0 < n_links && rc == ORC_OK; e0++) {
+        if (from[e0] != s) continue;
+        int32_t j = to[e0];
+        while (rem[e0] > 0) {
+            int32_t len = 0;
+            for (int32_t v = 0; v < n_nodes; v++) at[v] = -1;
+            int32_t u = j;
+            at[u] = 0;
+            int32_t last_gpu = -1;
+            for (;;) {
+                int32_t sink = -1;
+                if (rank_of_node[u] >= 0)
+                    for (int32_t e = 0; e < n_links; e++)
+                        if (from[e] == u && to[e] == t && rem[e] > 0) { sink = e; break; }
+                if (sink >= 0) { walk[len++] = sink; last_gpu = u; break; }
+                int32_t nxt = -1;
+                for (int32_t e = 0; e < n_links; e++)
+                    if (from[e] == u && to[e] != t && rem[e] > 0) { nxt = e; break; }
+                if (nxt < 0) { rc = ORC_EINVAL; break; }
+                int32_t w = to[nxt];
+                if (at[w] >= 0) {
+                    /* cycle: walk[at[w] .. len-1] + nxt */
+                    int64_t m = rem[nxt];
+                    for (int32_t q = at[w]; q < len; q++) if (rem[walk[q]] < m) m = rem[walk[q]];
+                    rem[nxt] -= m;
+                    for (int32_t q = at[w]; q < len; q++) rem[walk[q]] -= m;
+                    for (int32_t q = at[w]; q < len; q++) at[to[walk[q]]] = -1;
+                    len = at[w];
+                    at[w] = len;
+                    u = w;
+                    continue;
+                }
+                walk[len++] = nxt;
+                at[w] = len;
+                u = w;
+            }
+            if (rc != ORC_OK) break;
+            int64_t m = rem[e0];
+            for (int32_t q = 0; q < len; q++) if (rem[walk[q]] < m) m = rem[walk[q]];
+            rem[e0] -= m;
+            for (int32_t q = 0; q < len; q++) rem[walk[q]] -= m;
+            x[(int64_t)j * k + rank_of_node[last_gpu]] += m;
+        }
+    }
+    free(rem); free(walk); free(at);
+    return rc;
+}
+
+/* ------------------------------------------------------------------------------------------------
+ * Hash-partitioning baseline placement (the systems Moment compares against partition
+ * embeddings by hash; R24): vertices in id order; bin = splitmix64(v) mod n_bins (the splitmix64
+ * output function of Steele et al. with state v); a full bin passes the vertex to the next bin index
+ * (cyclically); slot = the bin's fill count at that moment. ORC_EINFEASIBLE if the capacities hold
+ * fewer than n rows.
+ * ------------------------------------------------------------------------------------------------ */
+static uint64_t orc_splitmix64(uint64_t state) {
+    uint64_t z = state + 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+int orc_hash_place(int64_t n, int32_t n_bins, const int64_t* cap_rows, int32_t* bin_of, int64_t* slot_of,
+                   int64_t* used) {
+    if (n < 0 || n_bins <= 0) return ORC_EINVAL;
+    int64_t total = 0;
+    for (int32_t b = 0; b < n_bins; b++) { used[b] = 0; total += cap_rows[b]; }
+    if (total < n) return ORC_EINFEASIBLE;
+    for (int64_t v = 0; v < n; v++) {
+        int32_t b = (int32_t)(orc_splitmix64((uint64_t)v) % (uint64_t)n_bins);
+        while (used[b] >= cap_rows[b]) b = (b + 1) % n_bins;
+        bin_of[v] = b;
+        slot_of[v] = used[b];
+        used[b]++;
+    }
     return ORC_OK;
 }
 

@@ -626,7 +626,7 @@ moment_status flow_at_time(const Ingest& G, int64_t T, int64_t* value, std::vect
     std::vector<int64_t> c(G.cap.size());
     for (size_t i = 0; i < c.size(); i++) {
         if (G.supply[i] || G.cap[i] == kInf) c[i] = G.cap[i];
-        else if (T < 0) c[i] = kInf;
+        else if (T < 0) c[i] = G.cap[i] == 0 ? 0 : kInf;  // reachability: a closed link stays closed
         else if (G.cap[i] != 0 && T > kScaledLimit / G.cap[i]) c[i] = kScaledLimit;
         else c[i] = G.cap[i] * T;
     }

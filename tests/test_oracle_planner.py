@@ -419,3 +419,177 @@ def test_ddak_zero_hotness_spreads_by_fill(orc):
     hot[:10] = 100
     bin_of, _, A, U = orc.ddak(hot, [1, 1], [600, 600], [5, 5], 1)
     assert abs(int(U[0]) - int(U[1])) <= 1 and A[0] > 0 and A[1] > 0
+
+
+# ---------------------------------------------------------------------------------------------- quotas (R11)
+def test_quota_hand_worked_cycle(orc):
+    # s=0 -> host bin j=1 -> a=2 <-> b=3 (a cycle a->b->a carrying 3), b -> GPU 5, a -> GPU 6, GPUs -> t=7.
+    # Worked by hand in the documented order (DESIGN R11): the walk j->a->b meets a again, cancels the
+    # cycle (3 units off a->b and b->a), resumes at a: a->b->g5 (4 units), then a->g6 (6 units).
+    links = [(0, 1, 0), (1, 2, 0), (2, 3, 0), (3, 2, 0), (3, 5, 0), (2, 6, 0), (5, 7, 0), (6, 7, 0)]
+    flow = [10, 10, 7, 3, 4, 6, 4, 6]
+    x = orc.quota(8, links, flow, 0, 7, [5, 6])
+    assert x[1].tolist() == [4, 6]
+    assert x.sum() == 10 and x[[0, 2, 3, 4, 5, 6, 7]].sum() == 0
+
+
+def test_quota_hand_worked_shared_switch(orc):
+    # two host bins j1=1, j2=2 into one switch x=3, switch -> GPU 4 (6 units) and GPU 5 (4 units).
+    # Supply links in order: j1 takes the switch's first out-link (to GPU 4) for all 5 units; j2 then
+    # finds 1 unit left on it and the other 4 on the link to GPU 5.
+    links = [(0, 1, 0), (0, 2, 0), (1, 3, 0), (2, 3, 0), (3, 4, 0), (3, 5, 0), (4, 6, 0), (5, 6, 0)]
+    flow = [5, 5, 5, 5, 6, 4, 6, 4]
+    x = orc.quota(7, links, flow, 0, 6, [4, 5])
+    assert x[1].tolist() == [5, 0] and x[2].tolist() == [1, 4]
+    # GPU ranks follow the order of the gpu list, not node ids
+    x = orc.quota(7, links, flow, 0, 6, [5, 4])
+    assert x[1].tolist() == [0, 5] and x[2].tolist() == [4, 1]
+
+
+def test_quota_rejects_unconserved_flow(orc):
+    links = [(0, 1, 0), (1, 2, 0), (2, 3, 0)]
+    with pytest.raises(orc.OracleError):
+        orc.quota(4, links, [5, 5, 4], 0, 3, [2])  # GPU 2 can pass on only 4 of the 5 units
+
+
+@pytest.mark.parametrize("S0,S1,p", [(800, 200, 10), (1000, 1000, 3), (5000, 0, 7), (300, 250, 2)])
+def test_quota_two_socket_without_upi_closed_form(orc, S0, S1, p):
+    # no UPI: every GPU is reachable from one socket's bin only, so x[j][h] is unique = the flow on h's sink
+    # link for h on j's socket, 0 elsewhere; and T* = max(ceil(S0/4p), ceil(S1/4p)) (the two-socket closed form
+    # with u = 0).
+    s, h0, h1, c0, c1, t = 0, 1, 2, 3, 4, 5
+    gpus = list(range(6, 14))
+    links = [(s, h0, S0), (s, h1, S1), (h0, c0, INF), (h1, c1, INF)]
+    sink_link = {}
+    for i, g in enumerate(gpus):
+        links.append((c0 if i < 4 else c1, g, p))
+        sink_link[g] = len(links)
+        links.append((g, t, INF))
+    T, flow = _tb(orc, 14, links, {0, 1}, s, t)
+    assert T == max(-(-S0 // (4 * p)), -(-S1 // (4 * p)))
+    x = orc.quota(14, links, flow, s, t, gpus)
+    for r, g in enumerate(gpus):
+        j = h0 if r < 4 else h1
+        assert x[j][r] == flow[sink_link[g]]
+        assert x[h1 if j == h0 else h0][r] == 0
+        assert x[j][r] <= p * T  # the port's capacity at T*
+    assert x[h0].sum() == S0 and x[h1].sum() == S1
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_quota_invariants_random_flows(orc, seed):
+    # flows built as sums of random s-j-...-g-t paths plus random cycles (so a decomposition exists), on
+    # random graphs; the decomposition must return every supply unit to exactly one GPU reachable from j in
+    # the flow's support, with row sums = supply flows and column sums = sink-link flows
+    rng = np.random.default_rng(seed)
+    n_host, n_mid, k = int(rng.integers(1, 4)), int(rng.integers(2, 6)), int(rng.integers(1, 5))
+    s = 0
+    host = list(range(1, 1 + n_host))
+    mid = list(range(1 + n_host, 1 + n_host + n_mid))
+    gpus = list(range(1 + n_host + n_mid, 1 + n_host + n_mid + k))
+    t = 1 + n_host + n_mid + k
+    N = t + 1
+    links, idx = [], {}
+
+    def link(u, v):
+        if (u, v) not in idx or rng.random() < 0.2:  # sometimes a parallel link
+            idx[(u, v)] = len(links)
+            links.append((u, v, INF))
+        return idx[(u, v)]
+
+    for j in host:
+        link(s, j)
+    for g in gpus:
+        link(g, t)
+    flow = np.zeros(200, np.int64)
+    for _ in range(int(rng.integers(1, 12))):  # paths
+        j = host[int(rng.integers(0, n_host))]
+        g = gpus[int(rng.integers(0, k))]
+        hops = [j] + [mid[int(i)] for i in rng.choice(n_mid, int(rng.integers(0, n_mid + 1)), replace=False)] + [g]
+        a = int(rng.integers(1, 20))
+        flow[link(s, j)] += a
+        for u, v in zip(hops, hops[1:]):
+            flow[link(u, v)] += a
+        flow[link(g, t)] += a
+    for _ in range(int(rng.integers(0, 4))):  # cycles among interconnect nodes and GPUs
+        cyc = [int(v) for v in rng.choice(mid + gpus, min(3, n_mid + k), replace=False)]
+        a = int(rng.integers(1, 10))
+        for u, v in zip(cyc, cyc[1:] + cyc[:1]):
+            flow[link(u, v)] += a
+    flow = flow[: len(links)]
+    x = orc.quota(N, links, flow, s, t, gpus)
+    assert (x >= 0).all()
+    for v in range(N):
+        sup = sum(int(f) for (u, w, _), f in zip(links, flow) if u == s and w == v)
+        assert x[v].sum() == sup
+    for r, g in enumerate(gpus):
+        assert x[:, r].sum() == sum(int(f) for (u, w, _), f in zip(links, flow) if u == g and w == t)
+    for j in host:
+        reach, st = {j}, [j]
+        while st:
+            u = st.pop()
+            for (a_, b_, _), f in zip(links, flow):
+                if a_ == u and f > 0 and b_ != t and b_ not in reach:
+                    reach.add(b_)
+                    st.append(b_)
+        for r, g in enumerate(gpus):
+            if x[j][r] > 0:
+                assert g in reach
+
+
+# ---------------------------------------------------------------------------------------------- hash baseline (R24)
+def _splitmix64_out(state):
+    z = (state + 0x9E3779B97F4A7C15) & ((1 << 64) - 1)
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & ((1 << 64) - 1)
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & ((1 << 64) - 1)
+    return z ^ (z >> 31)
+
+
+def test_hash_place_known_answer(orc):
+    # SplitMix64 (Steele, Lea, Flood 2014) seeded with 0 first outputs 0xE220A8397B1DCDAF, and with state
+    # 0x9E3779B97F4A7C15 (its second step) 0x6E789E6AA1B965F4: the oracle's vertex-0 bin must be the first
+    # value mod n_bins when no bin fills
+    for nb in (3, 7, 64):
+        b, sl, used = orc.hash_place(1, [10] * nb)
+        assert b[0] == 0xE220A8397B1DCDAF % nb and sl[0] == 0
+    assert _splitmix64_out(0) == 0xE220A8397B1DCDAF and _splitmix64_out(0x9E3779B97F4A7C15) == 0x6E789E6AA1B965F4
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_hash_place_properties(orc, seed):
+    rng = np.random.default_rng(seed)
+    nb = int(rng.integers(1, 6))
+    n = int(rng.integers(0, 40))
+    caps = [int(c) for c in rng.integers(0, 15, nb)]
+    if sum(caps) < n:
+        with pytest.raises(orc.OracleError) as e:
+            orc.hash_place(n, caps)
+        assert e.value.status == orc.EINFEASIBLE
+        caps[0] += n - sum(caps)
+    b, sl, used = orc.hash_place(n, caps)
+    for q in range(nb):
+        mine = [v for v in range(n) if b[v] == q]
+        assert len(mine) == used[q] <= caps[q]
+        assert [int(sl[v]) for v in mine] == list(range(len(mine)))  # slots in id order, contiguous
+    # a vertex leaves its hash bin only if that bin was already full when its turn came, and then lands in
+    # the first bin after it (cyclically) that still had room
+    fill = [0] * nb
+    for v in range(n):
+        h = _splitmix64_out(v) % nb
+        if fill[h] < caps[h]:
+            assert b[v] == h
+        else:
+            q = h
+            while fill[q] >= caps[q]:
+                q = (q + 1) % nb
+            assert b[v] == q
+        fill[b[v]] += 1
+
+
+def test_hash_place_uniform_when_roomy(orc):
+    # ample capacity: the bin counts of 2^16 ids follow the hash's uniformity (chi-square, 7 dof, p ~ 1e-4)
+    n, nb = 1 << 16, 8
+    b, _, used = orc.hash_place(n, [n] * nb)
+    exp = n / nb
+    chi2 = sum((u - exp) ** 2 / exp for u in used)
+    assert chi2 < 30

@@ -476,3 +476,115 @@ def test_signal_barrier_argument_errors():
     # a null peer pointer for another rank
     st = L.moment_signal_barrier(2, 0, (C.c_void_p * 2)(None, None), flags.ctypes.data, 1, 10, None, None)
     assert st == M.EINVAL
+
+
+# ---------------------------------------------------------------------------------------------- P5 quotas
+def _quota_vs_oracle(orc, topo, active, demand, nvlink=770, hbm=6000):
+    """moment_plan's x[j][h] == the oracle's decomposition (R11) of the product's own ingest flow, bit-exact;
+    column sums == the active GPUs' sink-link flows; row sums == the host bins' supplies."""
+    N, _, s, t = topo.info()
+    allnodes, alllinks, _, _ = topo.export()
+    p = M.plan(topo, active, demand, nvlink, hbm).info()
+    x = orc.quota(N, alllinks, p["link_flow"], s, t, active)
+    assert np.array_equal(p["quota"], x)
+    for r, g in enumerate(active):
+        sink = sum(int(f) for (u, v, _), f in zip(alllinks, p["link_flow"]) if u == g and v == t)
+        assert p["quota"][:, r].sum() == sink
+    k = len(active)
+    for v in range(N):
+        want = k * demand[v] if allnodes[v][0] == M.NODE_STORAGE and allnodes[v][1] != M.TIER_GPU_HBM else 0
+        assert p["quota"][v].sum() == want
+    return p
+
+
+@pytest.mark.parametrize("k,d_host0,d_host1,d_hbm", [(8, 4000, 1000, 500), (4, 100, 9000, 0), (2, 0, 0, 300),
+                                                     (8, 12345, 777, 4096), (1, 500, 500, 500), (3, 7, 11, 0)])
+def test_plan_quota_bit_exact_two_socket(orc, k, d_host0, d_host1, d_hbm):
+    nodes, links, host, hbm_nodes, gpu_nodes = two_socket_box(k=8)
+    topo = M.topology(nodes, links)
+    N = topo.info()[0]
+    demand = np.zeros(N, np.int64)
+    demand[host[0]], demand[host[1]] = d_host0, d_host1
+    for g in range(k):
+        demand[hbm_nodes[g]] = d_hbm
+    _quota_vs_oracle(orc, topo, gpu_nodes[:k], demand)
+
+
+@pytest.mark.parametrize("k,gps,uplink", [(8, 1, None), (8, 2, None), (4, 2, 30.0), (6, 1, None), (8, 4, 80.0)])
+def test_plan_quota_bit_exact_hgx(orc, k, gps, uplink):
+    from paper_conf_sc_shi0s0x0w25_b200 import boxes
+
+    act = boxes.spread_gpus(k, gpus_per_switch=gps)
+    box = boxes.hgx_b200(8, gpus_per_switch=gps, uplink_gbs=uplink, active=act)
+    topo = M.topology(box.nodes, box.links)
+    N = topo.info()[0]
+    rng = np.random.default_rng(k * 10 + gps)
+    demand = np.zeros(N, np.int64)
+    for j in box.host_bin:
+        demand[j] = int(rng.integers(10**5, 10**8))
+    for g in act:
+        demand[box.hbm_bin[g]] = int(rng.integers(0, 10**7))
+    _quota_vs_oracle(orc, topo, [box.gpu[g] for g in act], demand)
+
+
+@pytest.mark.parametrize("seed", range(15))
+def test_plan_quota_bit_exact_random_topologies(orc, seed):
+    # random interconnect between 1-3 host bins and 1-4 GPUs (antiparallel interconnect links make cycles
+    # in the flow possible), random capacities and demands
+    rng = np.random.default_rng(100 + seed)
+    n_host, n_mid, k = int(rng.integers(1, 4)), int(rng.integers(1, 5)), int(rng.integers(1, 5))
+    nodes = [(M.NODE_STORAGE, M.TIER_HOST_DRAM, j) for j in range(n_host)]
+    mid = list(range(len(nodes), len(nodes) + n_mid))
+    nodes += [(M.NODE_INTERCONNECT, M.TIER_NONE, -1)] * n_mid
+    gpus = list(range(len(nodes), len(nodes) + k))
+    nodes += [(M.NODE_COMPUTE, M.TIER_NONE, g) for g in range(k)]
+    links = []
+    for j in range(n_host):
+        for v in rng.choice(mid, int(rng.integers(1, n_mid + 1)), replace=False):
+            links.append((j, int(v), int(rng.integers(1, 100))))
+    for a in mid:  # interconnect <-> interconnect (antiparallel pairs) and interconnect -> GPU (P:L215)
+        for b in mid + gpus:
+            if a != b and rng.random() < 0.5:
+                links.append((a, b, int(rng.integers(1, 60))))
+    for m_ in mid:  # every interconnect node reaches some GPU
+        links.append((m_, gpus[int(rng.integers(0, k))], int(rng.integers(1, 60))))
+    topo = M.topology(nodes, links)
+    N = topo.info()[0]
+    demand = np.zeros(N, np.int64)
+    for j in range(n_host):
+        demand[j] = int(rng.integers(0, 5000))
+    act = sorted(int(g) for g in rng.choice(gpus, int(rng.integers(1, k + 1)), replace=False))
+    try:
+        _quota_vs_oracle(orc, topo, act, demand, nvlink=100, hbm=1000)
+    except M.MomentError as e:
+        # a demanded host bin that reaches no active GPU: the oracle's bisection must agree it is infeasible
+        assert e.status == M.EINFEASIBLE and "unreachable" in str(e)
+        _, alllinks, s, t = topo.export()
+        il = [(u, v, k * 0 + (len(act) * demand[v] if u == s else (INF if u in act else 0) if v == t else c))
+              for (u, v, c) in alllinks]
+        with pytest.raises(orc.OracleError) as oe:
+            orc.time_bisect(N, il, [1 if u == s else 0 for (u, _, _) in alllinks], s, t)
+        assert oe.value.status == orc.EINFEASIBLE
+
+
+# ---------------------------------------------------------------------------------------------- hash baseline
+@pytest.mark.parametrize("seed", range(12))
+def test_hash_place_bit_exact_vs_oracle(orc, seed):
+    rng = np.random.default_rng(500 + seed)
+    nb = int(rng.integers(1, 9))
+    n = int(rng.integers(0, 3000))
+    caps = rng.integers(0, max(2, 2 * n // nb + 2), nb)
+    if caps.sum() < n:
+        caps[int(rng.integers(0, nb))] += n - caps.sum()
+    hot = rng.integers(0, 50, n).astype(np.uint64)
+    b, sl, acc, used, _ = M.place(None, hot, caps, bin_tier=[1] * nb, bin_traffic=[1] * nb, mode=M.PLACE_HASH)
+    ob, osl, oused = orc.hash_place(n, caps)
+    assert np.array_equal(b, ob) and np.array_equal(sl, osl) and np.array_equal(used, oused)
+    for q in range(nb):
+        assert acc[q] == hot[b == q].sum()
+
+
+def test_hash_place_infeasible():
+    with pytest.raises(M.MomentError) as e:
+        M.place(None, np.zeros(10, np.uint64), [3, 3], bin_tier=[1, 1], bin_traffic=[1, 1], mode=M.PLACE_HASH)
+    assert e.value.status == M.EINFEASIBLE
