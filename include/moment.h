@@ -317,7 +317,8 @@ moment_status moment_bucket(moment_ctx_t ctx, const int64_t* ids, const int64_t*
  * out[i * R .. (i+1) * R) = row of ids[i], read from wherever the placement put it: local HBM, a peer's
  * HBM (NVLink load through bin_ptr) or pinned host DRAM (zero-copy PCIe read), 128-bit vectors.
  * Rows routed through a relay GPU h != rank are read by h from host DRAM and stored into this rank's out
- * over NVLink; moment_gather is then collective over the ranks of moment_gather_group.
+ * over NVLink; moment_gather is then collective: one process per GPU after moment_ctx_set_exchange (one
+ * enqueue per batch, below), or all ranks from one thread with moment_gather_group.
  * ids: device [max_n]; n_dev: device count or NULL (= max_n); out: device [max_n * R].
  * ================================================================================================ */
 moment_status moment_gather(moment_ctx_t ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n,
@@ -393,6 +394,48 @@ moment_status moment_relay_push(moment_ctx_t ctx, const int64_t* ids, int64_t ma
 moment_status moment_relay_serve_push(moment_ctx_t ctx, const uint64_t* inbox, const int64_t* inbox_count,
                                       int64_t cap, void* const* peer_out, void* stream);
 
+/* ================================================================================================
+ * One-call collective exchange (the ctx holds the inbox / signal pointers; P:L391-393 relay
+ * through a peer). After moment_ctx_set_exchange, moment_gather and moment_step on a ctx whose quota
+ * routes host rows through other ranks run the whole per-batch exchange as ONE enqueue on the stream,
+ * with no host synchronisation:
+ *   moment_bucket -> moment_gather_routed (this rank's own reads) -> moment_relay_push (requests stored
+ *   into the relay ranks' inboxes) -> signal barrier -> moment_relay_serve_push (rows stored into the
+ *   requesters' outputs) -> signal barrier.
+ * The barrier epoch lives in device memory (a counter in the ctx, advanced by each barrier kernel), so the
+ * sequence replays from moment_step's cached CUDA graph. Collective: every rank of the ctxs' world calls
+ * moment_gather / moment_step the same number of times in the same order (a rank with nothing to gather
+ * still calls, with max_n or *n_dev = 0). Peers store relayed rows into this rank's REGISTERED output,
+ * so moment_gather's `out` / moment_step's `d_rows` must be args->out, and max_n <= args->cap.
+ * args (device pointers, retained by the ctx until moment_ctx_free; peer pointers mapped in THIS
+ * process, e.g. by moment_ipc_import; entries [rank] are ignored):
+ *   cap            requests per source rank one inbox slot holds = rows of out (>= every rank's largest batch)
+ *   inbox          this rank's inbox, uint64 [world][cap][2];  inbox_count: int64 [world]
+ *   flags          this rank's barrier flag words, uint64 [world], zero before the first collective call
+ *   out            this rank's batch output, [cap][row_bytes] bytes, 16-byte aligned
+ *   peer_inbox[h]  = &inbox_h[rank][0][0];  peer_count[h] = &count_h[rank];  peer_out[h] = out_h;
+ *   peer_flag[h]   = &flags_h[rank]
+ *   timeout_ns     barrier watchdog (> 0): on expiry the wait ends and moment_exchange_status reports it.
+ * Errors: EINVAL (null / misaligned pointer, cap < 0, timeout <= 0), EUNSUPPORTED (world > MOMENT_MAX_WORLD).
+ * moment_exchange_status synchronises `stream`, then returns MOMENT_ETIMEDOUT (and clears it) if a barrier
+ * of this ctx expired since the last call, else MOMENT_OK.
+ * ================================================================================================ */
+typedef struct {
+    int64_t cap;
+    uint64_t* inbox;
+    int64_t* inbox_count;
+    uint64_t* flags;
+    void* out;
+    uint64_t* peer_inbox[MOMENT_MAX_WORLD];
+    int64_t* peer_count[MOMENT_MAX_WORLD];
+    void* peer_out[MOMENT_MAX_WORLD];
+    uint64_t* peer_flag[MOMENT_MAX_WORLD];
+    int64_t timeout_ns;
+} moment_exchange_args;
+
+moment_status moment_ctx_set_exchange(moment_ctx_t ctx, const moment_exchange_args* args);
+moment_status moment_exchange_status(moment_ctx_t ctx, void* stream);
+
 /* Cross-process device memory (another rank's HBM bin mapped into this process: the NVLink peer
  * pointer of bin_ptr). export: 64-byte handle of the allocation containing dptr and dptr's byte offset in
  * it; import: map the allocation (peer access enabled lazily) and return its base (add the offset);
@@ -405,7 +448,8 @@ moment_status moment_ipc_close(void* dptr);
 
 /* ================================================================================================
  * One whole hot-path step on device buffers: moment_sample of `seeds` followed by moment_gather of F_H
- * into d_rows (NULL: sample only; rows relayed through other ranks are not supported here). The 2H + 3
+ * into d_rows (NULL: sample only; rows relayed through other ranks need moment_ctx_set_exchange, and
+ * d_rows must then be its registered output: the step is then collective, see above). The 2H + 3
  * kernels are replayed from a CUDA graph cached in the ctx (captured on the first call of a given shape:
  * csr, n_seeds, fanout, flags, out and d_rows pointers; re-captured when any of them changes), so the host
  * cost per step is two launches. The per-batch rng_seed and seeds pointer reach the kernels through a

@@ -34,6 +34,46 @@ moment_status check_ctx(moment_ctx_t ctx, const char* what) {
     return MOMENT_OK;
 }
 
+bool has_remote_relay(const moment_ctx_s* c);
+
+// The per-batch exchange of one process per GPU as one enqueue (moment_ctx_set_exchange): bucket, this
+// rank's own reads, requests pushed into the relays' inboxes, barrier, relayed rows pushed into the
+// requesters' outputs, barrier. Every buffer is the ctx's (bucketing workspace) or registered with it.
+moment_status launch_gather_collective(moment_ctx_s* c, const int64_t* ids, const int64_t* n_dev, int64_t max_n,
+                                       void* out, cudaStream_t s) {
+    MOMENT_TRY(launch_bucket(c, ids, n_dev, max_n, c->bk_route, c->bk_qoff, c->bk_qpos, s));
+    MOMENT_TRY(launch_gather(c, ids, n_dev, max_n, out, c->bk_route, c->rank, s));
+    MOMENT_TRY(launch_relay_push(c, ids, c->bk_qoff, c->bk_qpos, max_n, c->ex.peer_inbox, c->ex.peer_count, s));
+    MOMENT_TRY(launch_signal_barrier_dev(c, s));  // every rank's requests are in its relays' inboxes
+    MOMENT_TRY(launch_relay_serve_push(c, c->ex.inbox, c->ex.inbox_count, c->ex.cap, c->ex.peer_out, s));
+    return launch_signal_barrier_dev(c, s);       // every relayed row is in its requester's output
+}
+
+// Gather for moment_gather / moment_step: the collective exchange when the quota relays rows through other
+// ranks (checked by check_gather_out), else the direct gather.
+moment_status launch_gather_any(moment_ctx_s* c, const int64_t* ids, const int64_t* n_dev, int64_t max_n, void* out,
+                                cudaStream_t s) {
+    if (c->world > 1 && c->has_exchange && has_remote_relay(c))
+        return launch_gather_collective(c, ids, n_dev, max_n, out, s);
+    return launch_gather(c, ids, n_dev, max_n, out, nullptr, c->rank, s);
+}
+
+// A gather whose quota relays through other ranks needs the registered exchange and its output buffer.
+moment_status check_gather_out(const moment_ctx_s* c, const void* out, int64_t max_n, const char* what) {
+    if (c->world > 1 && has_remote_relay(c)) {
+        if (!c->has_exchange)
+            return fail(MOMENT_EUNSUPPORTED, "%s: the quota relays host rows through other ranks: call "
+                        "moment_ctx_set_exchange first (or use moment_gather_group)", what);
+        if (out != c->ex.out)
+            return fail(MOMENT_EINVAL, "%s: with relays through other ranks the output must be the registered "
+                        "exchange output", what);
+        if (max_n > c->ex.cap || max_n > c->max_requests)
+            return fail(MOMENT_EOVERFLOW, "%s: max_n %lld > exchange cap %lld / workspace %lld", what, (long long)max_n,
+                        (long long)c->ex.cap, (long long)c->max_requests);
+    }
+    return MOMENT_OK;
+}
+
 bool has_remote_relay(const moment_ctx_s* c) {
     for (int b = 0; b < c->n_bins; b++) {
         if (c->bin_owner[b] >= 0 || c->quota.empty()) continue;
@@ -44,6 +84,17 @@ bool has_remote_relay(const moment_ctx_s* c) {
 }
 
 }  // namespace
+
+int moment::device_sms() {
+    static int cache[64] = {0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0) return 148;
+    if (dev < 64 && cache[dev] > 0) return cache[dev];
+    int n = 0;
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+    if (dev < 64) cache[dev] = n;
+    return n;
+}
 
 extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_t* out) {
     if (!a || !out) return fail(MOMENT_EINVAL, "moment_ctx_create: null argument");
@@ -94,6 +145,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     c->bin_owner.assign(a->bin_owner, a->bin_owner + a->n_bins);
     c->bin_ptr.assign(a->bin_ptr, a->bin_ptr + a->n_bins);
     c->placement = a->placement;
+    c->n_sms = device_sms();
     if (const char* gp = std::getenv("MOMENT_GATHER_PATH")) {
         const std::string v(gp);
         c->gather_path = v == "ldg" ? 1 : (v == "bulk" ? 2 : (v == "tma4" ? 3 : 0));
@@ -278,9 +330,53 @@ extern "C" moment_status moment_ctx_free(moment_ctx_t ctx) {
     if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
     if (ctx->ev_join) cudaEventDestroy(ctx->ev_join);
     cudaError_t e = ctx->ws ? cudaFree(ctx->ws) : cudaSuccess;
+    if (ctx->ex_ws) cudaFree(ctx->ex_ws);
     cudaSetDevice(cur);
     delete ctx;
     return cuda_check(e, "moment_ctx_free");
+}
+
+extern "C" moment_status moment_ctx_set_exchange(moment_ctx_t ctx, const moment_exchange_args* a) {
+    MOMENT_TRY(check_ctx(ctx, "moment_ctx_set_exchange"));
+    if (!a) return fail(MOMENT_EINVAL, "moment_ctx_set_exchange: null argument");
+    if (ctx->world > MOMENT_MAX_WORLD) return fail(MOMENT_EUNSUPPORTED, "moment_ctx_set_exchange: world > %d", MOMENT_MAX_WORLD);
+    if (a->cap < 0 || a->timeout_ns <= 0) return fail(MOMENT_EINVAL, "moment_ctx_set_exchange: cap < 0 or timeout <= 0");
+    if (!a->inbox || !a->inbox_count || !a->flags || !a->out || (reinterpret_cast<uintptr_t>(a->out) & 15))
+        return fail(MOMENT_EINVAL, "moment_ctx_set_exchange: inbox / counts / flags / out null or out not 16-byte aligned");
+    if (ctx->n_bins <= 0 || !ctx->placement) return fail(MOMENT_EINVAL, "moment_ctx_set_exchange: ctx has no placement map");
+    for (int h = 0; h < ctx->world; h++) {
+        if (h == ctx->rank) continue;
+        if (!a->peer_inbox[h] || !a->peer_count[h] || !a->peer_flag[h] || !a->peer_out[h] ||
+            (reinterpret_cast<uintptr_t>(a->peer_out[h]) & 15))
+            return fail(MOMENT_EINVAL, "moment_ctx_set_exchange: peer %d pointer null or misaligned", h);
+    }
+    if (!ctx->ex_ws) {
+        MOMENT_TRY(cuda_check(cudaMalloc(&ctx->ex_ws, 16), "moment_ctx_set_exchange: cudaMalloc"));
+        MOMENT_TRY(cuda_check(cudaMemset(ctx->ex_ws, 0, 16), "moment_ctx_set_exchange: memset"));
+        MOMENT_TRY(cuda_check(cudaDeviceSynchronize(), "moment_ctx_set_exchange: sync"));
+        ctx->d_epoch = static_cast<uint64_t*>(ctx->ex_ws);
+        ctx->d_xstatus = reinterpret_cast<int32_t*>(static_cast<char*>(ctx->ex_ws) + 8);
+    }
+    ctx->ex = *a;
+    ctx->has_exchange = true;
+    if (ctx->step_exec) {  // a cached step graph captured without the exchange is stale
+        cudaGraphExecDestroy(ctx->step_exec);
+        ctx->step_exec = nullptr;
+    }
+    return MOMENT_OK;
+}
+
+extern "C" moment_status moment_exchange_status(moment_ctx_t ctx, void* stream) {
+    MOMENT_TRY(check_ctx(ctx, "moment_exchange_status"));
+    if (!ctx->has_exchange) return MOMENT_OK;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    int32_t st = 0;
+    MOMENT_TRY(cuda_check(cudaMemcpyAsync(&st, ctx->d_xstatus, sizeof(st), cudaMemcpyDeviceToHost, s), "moment_exchange_status"));
+    MOMENT_TRY(cuda_check(cudaStreamSynchronize(s), "moment_exchange_status"));
+    if (st == 0) return MOMENT_OK;
+    MOMENT_TRY(cuda_check(cudaMemsetAsync(ctx->d_xstatus, 0, sizeof(int32_t), s), "moment_exchange_status"));
+    MOMENT_TRY(cuda_check(cudaStreamSynchronize(s), "moment_exchange_status"));
+    return fail(MOMENT_ETIMEDOUT, "moment_exchange_status: a device barrier of rank %d timed out", ctx->rank);
 }
 
 extern "C" moment_status moment_ctx_workspace_bytes(moment_ctx_t ctx, int64_t* bytes) {
@@ -329,7 +425,7 @@ moment_status run_step(moment_ctx_s* c, const moment_csr* csr, int64_t n_seeds, 
     MOMENT_TRY(cuda_check(cudaStreamIsCapturing(s, &cs), "moment_step"));
     if (cs != cudaStreamCaptureStatusNone || std::getenv("MOMENT_NO_GRAPH")) {
         MOMENT_TRY(launch_sample(c, csr, c->d_call, n_seeds, p, out, s));
-        if (rows) MOMENT_TRY(launch_gather(c, out->nodes, out->counts + H, out->cap_nodes, rows, nullptr, c->rank, s));
+        if (rows) MOMENT_TRY(launch_gather_any(c, out->nodes, out->counts + H, out->cap_nodes, rows, s));
         return MOMENT_OK;
     }
     if (!c->step_exec || !same_key(c->step_key, csr, n_seeds, p, out, rows)) {
@@ -342,11 +438,11 @@ moment_status run_step(moment_ctx_s* c, const moment_csr* csr, int64_t n_seeds, 
         const bool fork = rows && c->step_fork;
         moment_status st = launch_sample(c, csr, c->d_call, n_seeds, p, out, c->cap_stream, fork ? c->ev_fork : nullptr);
         if (st == MOMENT_OK && rows && !fork)
-            st = launch_gather(c, out->nodes, out->counts + H, out->cap_nodes, rows, nullptr, c->rank, c->cap_stream);
+            st = launch_gather_any(c, out->nodes, out->counts + H, out->cap_nodes, rows, c->cap_stream);
         if (st == MOMENT_OK && fork) {  // gather on a branch that joins after the compaction
             st = cuda_check(cudaStreamWaitEvent(c->cap_side, c->ev_fork, 0), "moment_step: fork");
             if (st == MOMENT_OK)
-                st = launch_gather(c, out->nodes, out->counts + H, out->cap_nodes, rows, nullptr, c->rank, c->cap_side);
+                st = launch_gather_any(c, out->nodes, out->counts + H, out->cap_nodes, rows, c->cap_side);
             if (st == MOMENT_OK) st = cuda_check(cudaEventRecord(c->ev_join, c->cap_side), "moment_step: join");
             if (st == MOMENT_OK) st = cuda_check(cudaStreamWaitEvent(c->cap_stream, c->ev_join, 0), "moment_step: join");
         }
@@ -374,8 +470,7 @@ moment_status run_step(moment_ctx_s* c, const moment_csr* csr, int64_t n_seeds, 
 moment_status check_rows(const moment_ctx_s* c, void* rows, const moment_sample_out* out) {
     if (!rows) return MOMENT_OK;
     if (c->n_bins <= 0) return fail(MOMENT_EINVAL, "moment_step: ctx has no feature bins");
-    if (c->world > 1 && has_remote_relay(c))
-        return fail(MOMENT_EUNSUPPORTED, "moment_step: the quota relays host rows through other ranks; use moment_gather_group");
+    MOMENT_TRY(check_gather_out(c, rows, out->cap_nodes, "moment_step"));
     if ((reinterpret_cast<uintptr_t>(rows) & 15) != 0) return fail(MOMENT_EINVAL, "moment_step: rows must be 16-byte aligned");
     if (out->cap_nodes * (c->row_bytes / 16) >= (int64_t(1) << 32))
         return fail(MOMENT_EUNSUPPORTED, "moment_step: %lld rows exceed 2^32 vectors per call", (long long)out->cap_nodes);
@@ -434,9 +529,8 @@ extern "C" moment_status moment_bucket(moment_ctx_t ctx, const int64_t* ids, con
 extern "C" moment_status moment_gather(moment_ctx_t ctx, const int64_t* ids, const int64_t* n_dev, int64_t max_n, void* out,
                                        void* stream) {
     MOMENT_TRY(check_ctx(ctx, "moment_gather"));
-    if (ctx->world > 1 && has_remote_relay(ctx))
-        return fail(MOMENT_EUNSUPPORTED, "moment_gather: the quota relays host rows through other ranks; use moment_gather_group");
-    return launch_gather(ctx, ids, n_dev, max_n, out, nullptr, ctx->rank, static_cast<cudaStream_t>(stream));
+    MOMENT_TRY(check_gather_out(ctx, out, max_n, "moment_gather"));
+    return launch_gather_any(ctx, ids, n_dev, max_n, out, static_cast<cudaStream_t>(stream));
 }
 
 extern "C" moment_status moment_gather_group(moment_ctx_t const* ctxs, int32_t world, const int64_t* const* ids,

@@ -44,6 +44,7 @@ struct moment_ctx_s {
     int32_t hop_warp_segmented = 1;   // k <= 32: k-lane groups packed in a warp (MOMENT_HOP_WARP=0: 2^n tiles)
     int32_t init_in_hop0 = 1;         // the first hop's sampler also initialises the call (MOMENT_INIT_KERNEL=1: separate)
     int32_t bulk_stages = 4, bulk_blocks_per_sm = 4, bulk_stage_kb = 14;  // bulk gather shape (MOMENT_BULK="S,B,KB")
+    int32_t n_sms = 148;  // multiprocessors of the ctx's device (cudaDevAttrMultiProcessorCount)
     std::vector<int32_t> bin_owner;
     std::vector<void*> bin_ptr;
     const uint64_t* placement = nullptr;
@@ -88,6 +89,13 @@ struct moment_ctx_s {
     int64_t* d_quota = nullptr;         // [n_bins * world]
     int32_t* d_bin_owner = nullptr;     // [n_bins]
     int64_t* d_seed_stage = nullptr;    // [max_seeds] for moment_step_host
+    // one-call collective exchange (moment_ctx_set_exchange): peer inboxes / outputs / flags, and the
+    // device-side barrier epoch counter and watchdog status (so the exchange replays from a CUDA graph)
+    bool has_exchange = false;
+    moment_exchange_args ex{};
+    void* ex_ws = nullptr;          // [0] uint64 epoch counter, [8] int32 watchdog status
+    uint64_t* d_epoch = nullptr;
+    int32_t* d_xstatus = nullptr;
     // per-call arguments the kernels read from device memory (so one captured graph serves every batch)
     uint64_t* d_call = nullptr;         // [2]: rng_seed, seeds pointer (written by set_call_kernel per call)
     // cached CUDA graph of one moment_step (sample + gather), re-captured when its shape changes
@@ -124,6 +132,14 @@ constexpr int kBitscanTileWords = kBitscanWordsPerThread * kBitscanThreads;  // 
 constexpr int64_t kSparseScanMinWords = 1 << 18;  // > 8.4 M vertices: C3-C5 scan sparsely, C1/C2 densely
 constexpr int kBucketTile = 1024;    // requests per bucketing tile
 constexpr int kMaxFanout = 1024;
+
+// Multiprocessors of the current device (queried once per device, cached): every launcher sizes its grid
+// as a multiple of it instead of assuming 148.
+int device_sms();
+
+// Device-side barrier with the epoch read from / advanced in device memory (signal.cu): the ctx's
+// collective gather enqueues it between its phases, replayable from a CUDA graph.
+moment_status launch_signal_barrier_dev(const moment_ctx_s* ctx, cudaStream_t stream);
 
 // Launchers (defined in sample.cu / gather.cu).
 moment_status check_sample(const moment_ctx_s* ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,

@@ -562,7 +562,7 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
         const int stages = 4, bps = ctx->tma4_blocks_per_sm;
         const size_t smem = (size_t)stages * 8 * G;
         const int64_t tiles = (max_n + kTma4Rows - 1) / kTma4Rows;
-        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)148 * bps));
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)device_sms() * bps));
         gather_tma4_kernel<4><<<grid, 32, smem, stream>>>(ctx->tma_map, ids, n_dev, max_n, (uint32_t)ctx->row_bytes,
                                                           ctx->l2_load_policy, ctx->l2_store_policy,
                                                           reinterpret_cast<char*>(out));
@@ -577,7 +577,7 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
         const size_t smem = (size_t)stages * rows * ctx->row_bytes;
         if (smem > (size_t)kBulkSmemMax) return fail(MOMENT_EINVAL, "moment_gather: bulk stage config needs %zu B smem", smem);
         const int64_t tiles = (max_n + rows - 1) / rows;
-        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)148 * bps));
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)device_sms() * bps));
         auto launch = [&](auto kern) {
             kern<<<grid, 32, smem, stream>>>(make_bins(ctx), ctx->placement, ids, n_dev, max_n, (uint32_t)ctx->row_bytes,
                                              ctx->row_stride, rows, ctx->l2_load_policy, ctx->l2_store_policy,
@@ -588,7 +588,7 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
         else if (stages <= 6) launch(gather_bulk_kernel<6>);
         else launch(gather_bulk_kernel<8>);
     } else {
-        const int grid = grid_for(max_n * rv, kGatherThreads * kGatherUnroll, 148 * 8);
+        const int grid = grid_for(max_n * rv, kGatherThreads * kGatherUnroll, device_sms() * 8);
         gather_kernel<<<grid, kGatherThreads, 0, stream>>>(make_bins(ctx), ctx->placement, ids, n_dev, max_n,
                                                             make_fastdiv((uint32_t)rv), ctx->row_stride / 16, route,
                                                             ctx->world, serve_rank, reinterpret_cast<int4*>(out));
@@ -607,7 +607,7 @@ moment_status launch_bucket(moment_ctx_s* ctx, const int64_t* ids, const int64_t
     if (max_n == 0)  // no requests: empty queues (the tile kernels below would read stale tile counts)
         return cuda_check(cudaMemsetAsync(qoff, 0, (size_t)(Q + 1) * sizeof(int64_t), stream), "moment_bucket: empty");
     const int64_t n_tiles = std::max<int64_t>(1, (max_n + kBucketTile - 1) / kBucketTile);
-    const int grid = (int)std::min<int64_t>(n_tiles, 148 * 2);
+    const int grid = (int)std::min<int64_t>(n_tiles, device_sms() * 2);
     bucket_count_kernel<<<grid, 256, 0, stream>>>(ctx->placement, ids, n_dev, max_n, ctx->n_bins, ctx->bk_tile_counts);
     bucket_scan_kernel<<<1, 64, 0, stream>>>(ctx->bk_tile_counts, n_tiles, ctx->n_bins, ctx->bk_bin_total);
     const int32_t* owner_dev = ctx->d_bin_owner;
@@ -624,7 +624,7 @@ moment_status launch_relay(moment_ctx_s* server, moment_ctx_s* requester, const 
                            const int64_t* qoff, const int64_t* qpos, void* requester_out, cudaStream_t stream) {
     (void)route;
     const int64_t rv = server->row_bytes / 16;
-    const int grid = 148 * 4;
+    const int grid = device_sms() * 4;
     relay_kernel<<<grid, kGatherThreads, 0, stream>>>(make_bins(server), requester->placement, ids, qoff, qpos,
                                                        server->n_bins, server->world, server->rank,
                                                        make_fastdiv((uint32_t)rv), server->row_stride / 16,
@@ -797,7 +797,7 @@ moment_status launch_relay_pack(moment_ctx_s* ctx, const int64_t* ids, const int
                                 int64_t max_n, uint64_t* words, int64_t* counts, cudaStream_t stream) {
     if (!ctx->placement) return fail(MOMENT_EINVAL, "moment_relay_pack: ctx has no placement map");
     if (ctx->n_bins * (ctx->world - 1) > kMaxSegs) return fail(MOMENT_EUNSUPPORTED, "moment_relay_pack: too many segments");
-    const int grid = grid_for(std::max<int64_t>(max_n, 1), 256, 148 * 4);
+    const int grid = grid_for(std::max<int64_t>(max_n, 1), 256, device_sms() * 4);
     relay_pack_kernel<<<grid, 256, 0, stream>>>(make_bins(ctx), ctx->placement, ids, qoff, qpos, ctx->n_bins, ctx->world,
                                                 ctx->rank, words, counts);
     return cuda_check(cudaGetLastError(), "moment_relay_pack: launch");
@@ -808,7 +808,7 @@ moment_status launch_relay_serve(moment_ctx_s* ctx, const uint64_t* words, const
     const int64_t rv = ctx->row_bytes / 16;
     if (max_n * rv >= (int64_t(1) << 32)) return fail(MOMENT_EUNSUPPORTED, "moment_relay_serve: too many rows");
     if (max_n == 0) return MOMENT_OK;
-    relay_serve_kernel<<<grid_for(max_n * rv, kGatherThreads, 148 * 8), kGatherThreads, 0, stream>>>(
+    relay_serve_kernel<<<grid_for(max_n * rv, kGatherThreads, device_sms() * 8), kGatherThreads, 0, stream>>>(
         make_bins(ctx), words, n_dev, max_n, make_fastdiv((uint32_t)rv), ctx->row_stride / 16,
         reinterpret_cast<int4*>(rows));
     return cuda_check(cudaGetLastError(), "moment_relay_serve: launch");
@@ -819,7 +819,7 @@ moment_status launch_relay_scatter(moment_ctx_s* ctx, const uint64_t* words, con
     const int64_t rv = ctx->row_bytes / 16;
     if (max_n * rv >= (int64_t(1) << 32)) return fail(MOMENT_EUNSUPPORTED, "moment_relay_scatter: too many rows");
     if (max_n == 0) return MOMENT_OK;
-    relay_scatter_kernel<<<grid_for(max_n * rv, kGatherThreads, 148 * 8), kGatherThreads, 0, stream>>>(
+    relay_scatter_kernel<<<grid_for(max_n * rv, kGatherThreads, device_sms() * 8), kGatherThreads, 0, stream>>>(
         words, n_dev, max_n, make_fastdiv((uint32_t)rv), reinterpret_cast<const int4*>(rows),
         reinterpret_cast<int4*>(out));
     return cuda_check(cudaGetLastError(), "moment_relay_scatter: launch");
@@ -839,7 +839,7 @@ moment_status launch_relay_push(moment_ctx_s* ctx, const int64_t* ids, const int
         p.inbox[h] = peer_inbox[h];
         p.count[h] = peer_count[h];
     }
-    const int grid = grid_for(std::max<int64_t>(max_n, 1), 256, 148 * 4);
+    const int grid = grid_for(std::max<int64_t>(max_n, 1), 256, device_sms() * 4);
     relay_push_kernel<<<grid, 256, 0, stream>>>(make_bins(ctx), ctx->placement, ids, qoff, qpos, ctx->n_bins, ctx->world,
                                                 ctx->rank, p);
     return cuda_check(cudaGetLastError(), "moment_relay_push: launch");
@@ -857,7 +857,7 @@ moment_status launch_relay_serve_push(moment_ctx_s* ctx, const uint64_t* inbox, 
     }
     const int64_t rv = ctx->row_bytes / 16;
     // grid sized for the worst case (every source's full inbox); blocks without work exit at once
-    const int grid = grid_for(std::max<int64_t>(cap * (ctx->world - 1) * rv, 1), kGatherThreads, 148 * 8);
+    const int grid = grid_for(std::max<int64_t>(cap * (ctx->world - 1) * rv, 1), kGatherThreads, device_sms() * 8);
     relay_serve_push_kernel<<<grid, kGatherThreads, 0, stream>>>(make_bins(ctx), inbox, inbox_count, cap, ctx->world,
                                                                  ctx->rank, make_fastdiv((uint32_t)rv),
                                                                  ctx->row_stride / 16, o);
@@ -887,7 +887,7 @@ moment_status configure_gather_kernels(int carveout) {
 
 moment_status launch_hotness(const int64_t* ids, const int64_t* n_dev, int64_t max_n, uint64_t* hot, cudaStream_t stream) {
     if (max_n <= 0) return MOMENT_OK;
-    hotness_kernel<<<grid_for(max_n, 256, 148 * 8), 256, 0, stream>>>(ids, n_dev, max_n, hot);
+    hotness_kernel<<<grid_for(max_n, 256, device_sms() * 8), 256, 0, stream>>>(ids, n_dev, max_n, hot);
     return cuda_check(cudaGetLastError(), "moment_hotness: launch");
 }
 

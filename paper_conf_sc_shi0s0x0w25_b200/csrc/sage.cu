@@ -178,7 +178,7 @@ moment_status check_args(const void* x, int64_t ld_x, int32_t dtype, int64_t dim
 }
 
 int grid_for(int64_t n_dst) {
-    return (int)std::max<int64_t>(1, std::min<int64_t>((n_dst + kWarps - 1) / kWarps, 148 * 8));
+    return (int)std::max<int64_t>(1, std::min<int64_t>((n_dst + kWarps - 1) / kWarps, device_sms() * 8));
 }
 
 }  // namespace

@@ -840,7 +840,7 @@ template <int G, int Q>
 void launch_sample_hop_q(const HopArgs& a, int64_t max_F, cudaStream_t stream) {
     const int64_t groups = (max_F + Q - 1) / Q;
     const int64_t blocks = std::max<int64_t>(1, (groups * G + 255) / 256);
-    hop_sample_kernel<G, Q><<<(int)std::min<int64_t>(blocks, (int64_t)148 * a.grid_per_sm), 256, 0, stream>>>(a);
+    hop_sample_kernel<G, Q><<<(int)std::min<int64_t>(blocks, (int64_t)device_sms() * a.grid_per_sm), 256, 0, stream>>>(a);
 }
 
 // Small frontiers keep one node per group (latency: every node in flight at once); large frontiers batch
@@ -859,7 +859,7 @@ void launch_sample_warp_q(const HopArgs& a, int64_t max_F, cudaStream_t stream, 
     const int64_t warps = (max_F + per_warp - 1) / per_warp;
     const int64_t blocks = std::max<int64_t>(1, (warps + 7) / 8);
     hop_sample_warp_kernel<Q, kInit>
-        <<<(int)std::min<int64_t>(blocks, (int64_t)148 * a.grid_per_sm), 256, 0, stream>>>(a, in);
+        <<<(int)std::min<int64_t>(blocks, (int64_t)device_sms() * a.grid_per_sm), 256, 0, stream>>>(a, in);
 }
 
 void launch_sample_warp(const HopArgs& a, int64_t max_F, int big_q, cudaStream_t stream) {
@@ -935,7 +935,7 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
                         check, ctx->tile_status, ctx->n_tile_status, ctx->tickets, 1 + std::max(1, ctx->max_hops),
                         ctx->ebase, std::max(1, ctx->max_hops)};
     if (!init_in_hop0) {
-        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n_seeds + 255) / 256, 148 * 4));
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n_seeds + 255) / 256, device_sms() * 4));
         init_kernel<<<grid, 256, 0, stream>>>(call, n_seeds, ctx->n_vertices, out->nodes, ctx->lidx, ctx->visited,
                                               out->counts, ctx->error_flag, check, ctx->tile_status, ctx->n_tile_status,
                                               ctx->tickets, 1 + std::max(1, ctx->max_hops), ctx->ebase,
@@ -979,12 +979,12 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
         if (ctx->sparse_scan) {  // one summary word (32 newbits words) per thread
             const int nt = ctx->sparse_threads;
             const int64_t tiles = (ctx->n_words + 32 * nt - 1) / (32 * nt);
-            const int grid = (int)std::min<int64_t>(tiles, 148 * (1024 / nt) * 2);
+            const int grid = (int)std::min<int64_t>(tiles, device_sms() * (1024 / nt) * 2);
             if (nt == 1024) bitscan_sparse_kernel<1024><<<grid, 1024, 0, stream>>>(s);
             else if (nt == 512) bitscan_sparse_kernel<512><<<grid, 512, 0, stream>>>(s);
             else bitscan_sparse_kernel<256><<<grid, 256, 0, stream>>>(s);
         } else {
-            const int nb = (int)std::min<int64_t>(n_scan_tiles, 148 * 4);
+            const int nb = (int)std::min<int64_t>(n_scan_tiles, device_sms() * 4);
             if (s.prefetch_idx) bitscan_kernel<true><<<nb, kBitscanThreads, 0, stream>>>(s);
             else bitscan_kernel<false><<<nb, kBitscanThreads, 0, stream>>>(s);
         }
@@ -1010,7 +1010,7 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
     ca.tile_edges = ctx->tile_edges;
     ca.H = H;
     const int grid = (int)std::max<int64_t>(
-        1, std::min<int64_t>(std::max(ca.tb[H], (F_bound + 1023) / 1024), (int64_t)148 * ctx->compact_grid_per_sm));
+        1, std::min<int64_t>(std::max(ca.tb[H], (F_bound + 1023) / 1024), (int64_t)device_sms() * ctx->compact_grid_per_sm));
     compact_kernel<<<grid, kSampleTile, 0, stream>>>(ca);
     return cuda_check(cudaGetLastError(), "moment_sample: launch");
 }

@@ -57,7 +57,45 @@ __global__ void signal_barrier_kernel(PeerFlags peer, int world, int rank, const
     __syncthreads();
 }
 
+// The same barrier with its epoch in device memory: every thread reads the counter, waits on epoch + 1, and
+// thread 0 stores epoch + 1 back once all have left. Barriers on one stream run one after another, so each
+// sees the previous one's value; a captured graph replays with fresh epochs.
+__global__ void signal_barrier_dev_kernel(PeerFlags peer, int world, int rank, const uint64_t* flags,
+                                          uint64_t* epoch_ctr, int64_t timeout_ns, int32_t* status) {
+    const uint64_t epoch = *reinterpret_cast<volatile uint64_t*>(epoch_ctr) + 1;
+    const int h = threadIdx.x;
+    if (h < world && h != rank) {
+        asm volatile("fence.sc.sys;" ::: "memory");
+        st_release_sys(peer.p[h], epoch);
+        const uint64_t t0 = globaltimer();
+        unsigned ns = 32;
+        while (ld_acquire_sys(flags + h) < epoch) {
+            if ((int64_t)(globaltimer() - t0) > timeout_ns) {
+                atomicExch(status, (int32_t)MOMENT_ETIMEDOUT);
+                break;
+            }
+            __nanosleep(ns);
+            ns = ns < 4096 ? ns * 2 : ns;
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) *epoch_ctr = epoch;
+}
+
 }  // namespace
+
+namespace moment {
+
+moment_status launch_signal_barrier_dev(const moment_ctx_s* c, cudaStream_t stream) {
+    if (c->world == 1) return MOMENT_OK;
+    PeerFlags pf{};
+    for (int h = 0; h < c->world; h++) pf.p[h] = h == c->rank ? nullptr : c->ex.peer_flag[h];
+    signal_barrier_dev_kernel<<<1, 64, 0, stream>>>(pf, c->world, c->rank, c->ex.flags, c->d_epoch, c->ex.timeout_ns,
+                                                     c->d_xstatus);
+    return cuda_check(cudaGetLastError(), "exchange barrier: launch");
+}
+
+}  // namespace moment
 
 extern "C" moment_status moment_signal_barrier(int32_t world, int32_t rank, uint64_t* const* peer_flags,
                                                const uint64_t* flags, uint64_t epoch, int64_t timeout_ns,

@@ -98,16 +98,20 @@ class PeerExchange:
     through CUDA-IPC-mapped peer pointers (NVLink loads/stores between the GPUs of one node).
 
     Setup is collective over `group`: this rank allocates its inbox (int64 [world][cap][2]), inbox counts
-    (int64 [world]) and batch output (uint8 [cap][R]), exports them, and maps every peer's. Per batch
-    (`gather`): bucket -> routed gather (own rows) -> relay_push (peer stores) -> barrier -> relay_serve_push
-    (peer stores into the requesters' outputs) -> barrier. device_barrier=False: each barrier is a stream
-    synchronize + process barrier (NCCL: device collective, gloo: host). device_barrier=True: each barrier is
-    `moment_signal_barrier` on the stream (release/acquire flag words in peer memory), so a
-    batch's exchange is enqueued without any host synchronisation; `check()` reports a watchdog timeout.
+    (int64 [world]), barrier flags and batch output (uint8 [cap][R]), exports them, and maps every peer's.
+
+    one_call=True (default): the pointers are registered with the ctx (moment_ctx_set_exchange), and a batch
+    is ONE library call: `gather` = moment_gather, `step` = moment_step (sample + the whole exchange,
+    replayed from the ctx's CUDA graph), with device-side signal barriers between the phases and no host
+    synchronisation. This class is then setup only.
+    one_call=False: the phases are sequenced from here (bucket -> routed gather -> relay_push -> barrier ->
+    relay_serve_push -> barrier); device_barrier=False: each barrier is a stream synchronize + process barrier
+    (NCCL: device collective, gloo: host); device_barrier=True: `moment_signal_barrier` on the stream.
+    `check()` reports a watchdog timeout of a device barrier.
     """
 
     def __init__(self, ctx, max_n: int, row_bytes: int, device, group=None, device_barrier: bool = False,
-                 timeout_s: float = 10.0):
+                 timeout_s: float = 10.0, one_call: bool = True):
         import paper_conf_sc_shi0s0x0w25_b200 as M
 
         self.M, self.ctx, self.group = M, ctx, group
@@ -144,6 +148,11 @@ class PeerExchange:
             self.peer_count[h] = addr[1] + self.rank * 8
             self.peer_out[h] = addr[2]
             self.peer_flag[h] = addr[3] + self.rank * 8  # rank h's flag word for this rank
+        self.one_call = one_call
+        if one_call:
+            ctx.set_exchange(cap=self.cap, inbox=self.inbox, inbox_count=self.count, flags=self.flags, out=self.out,
+                             peer_inbox=self.peer_inbox, peer_count=self.peer_count, peer_out=self.peer_out,
+                             peer_flag=self.peer_flag, timeout_ns=self.timeout_ns)
         dist.barrier(group=group)
 
     def _barrier(self, s):
@@ -153,6 +162,9 @@ class PeerExchange:
 
     def check(self):
         """Raise if a device barrier timed out (synchronises)."""
+        if self.one_call:
+            self.ctx.exchange_status()
+            return
         st = int(self.status.item())
         if st != 0:
             raise self.M.MomentError(st, "PeerExchange: device barrier watchdog expired")
@@ -162,6 +174,9 @@ class PeerExchange:
         assert n <= self.cap
         s = stream if stream is not None else torch.cuda.current_stream(ids.device)
         ctx = self.ctx
+        if self.one_call:
+            ctx.gather(ids, self.out, max_n=n, stream=s)
+            return self.out[:n]
         with torch.cuda.stream(s):
             ctx.bucket(ids, self.route, self.qoff, self.qpos, max_n=n, stream=s)
             ctx.gather_routed(ids, self.route, self.out, max_n=n, stream=s)
@@ -179,6 +194,13 @@ class PeerExchange:
         s.synchronize()
         dist.barrier(group=self.group)  # every relayed row is in its requester's output
         return self.out[:n]
+
+    def step(self, indptr, indices, seeds, fanout, rng_seed: int, bufs, stream=None):
+        """Collective (one_call only): sample `seeds` and gather F_H with the relay exchange, all in ONE
+        moment_step call replayed from the ctx's CUDA graph; the rows land in self.out[:|F_H|]."""
+        assert self.one_call
+        self.ctx.step(indptr, indices, seeds, fanout, rng_seed, bufs, self.out, stream=stream)
+        return self.out
 
     def close(self):
         """Collective: unmap the peers' buffers once every rank is done with them."""

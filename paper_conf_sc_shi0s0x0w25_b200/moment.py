@@ -34,6 +34,7 @@ EXPORTED = [
     "moment_step", "moment_step_host", "moment_gather_routed", "moment_relay_pack", "moment_relay_serve",
     "moment_relay_scatter", "moment_relay_push", "moment_relay_serve_push", "moment_ipc_export", "moment_ipc_import",
     "moment_ipc_close", "moment_sage_mean", "moment_sage_mean_backward", "moment_signal_barrier",
+    "moment_ctx_set_exchange", "moment_exchange_status",
 ]
 MAX_WORLD = 64
 
@@ -81,6 +82,12 @@ class CtxArgs(C.Structure):
                 ("max_seeds", C.c_int64), ("max_hops", C.c_int32), ("max_fanout", C.c_void_p),
                 ("row_bytes", C.c_int64), ("row_stride", C.c_int64), ("n_bins", C.c_int32),
                 ("bin_owner", C.c_void_p), ("bin_ptr", C.c_void_p), ("placement", C.c_void_p), ("quota", C.c_void_p)]
+
+
+class ExchangeArgs(C.Structure):
+    _fields_ = [("cap", C.c_int64), ("inbox", C.c_void_p), ("inbox_count", C.c_void_p), ("flags", C.c_void_p),
+                ("out", C.c_void_p), ("peer_inbox", C.c_void_p * 64), ("peer_count", C.c_void_p * 64),
+                ("peer_out", C.c_void_p * 64), ("peer_flag", C.c_void_p * 64), ("timeout_ns", C.c_int64)]
 
 
 class Csr(C.Structure):
@@ -147,6 +154,8 @@ def lib():
             "moment_sage_mean": ([P, I64, I32, I64, P, P, I64, P, I64, P], I32),
             "moment_signal_barrier": ([I32, I32, P, P, U64, I64, P, P], I32),
             "moment_sage_mean_backward": ([P, I64, I32, I64, P, P, I64, P, I64, P], I32),
+            "moment_ctx_set_exchange": ([P, P], I32),
+            "moment_exchange_status": ([P, P], I32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -501,7 +510,28 @@ class Ctx:
         _check(lib().moment_relay_scatter(self.handle, words.data_ptr(), None, n, rows.data_ptr(), out.data_ptr(),
                                           _stream(stream)))
 
-    # ---- the same exchange over peer memory (see exchange.PeerExchange) ----
+    # ---- one-call collective exchange (moment_ctx_set_exchange; exchange.PeerExchange sets it up) ----
+    def set_exchange(self, *, cap: int, inbox, inbox_count, flags, out, peer_inbox: list[int], peer_count: list[int],
+                     peer_out: list[int], peer_flag: list[int], timeout_ns: int = 10**10):
+        """Register this rank's inbox / counts / flags / output and the peers' mapped addresses: moment_gather
+        and moment_step then run the relay exchange as one enqueue (collective over the ctx's world)."""
+        a = ExchangeArgs()
+        a.cap, a.inbox, a.inbox_count, a.flags, a.out = cap, inbox.data_ptr(), inbox_count.data_ptr(), \
+            flags.data_ptr(), out.data_ptr()
+        for h in range(self.world):
+            a.peer_inbox[h] = peer_inbox[h] or None
+            a.peer_count[h] = peer_count[h] or None
+            a.peer_out[h] = peer_out[h] or None
+            a.peer_flag[h] = peer_flag[h] or None
+        a.timeout_ns = timeout_ns
+        _check(lib().moment_ctx_set_exchange(self.handle, C.byref(a)))
+        self._keep_ex = (inbox, inbox_count, flags, out)
+
+    def exchange_status(self, stream=None):
+        """Raise MomentError(ETIMEDOUT) if a device barrier of this ctx expired (synchronises the stream)."""
+        _check(lib().moment_exchange_status(self.handle, _stream(stream)))
+
+    # ---- the same exchange over peer memory, phase by phase (see exchange.PeerExchange) ----
     def relay_push(self, ids, qoff, qpos, peer_inbox: list[int], peer_count: list[int], *, max_n: int | None = None,
                    stream=None):
         """peer_inbox[h] / peer_count[h]: device addresses of rank h's inbox / count slot for this rank."""

@@ -73,11 +73,42 @@ def _rank_main(rank, world, transport="alltoall"):
     nF = int(bufs.counts[2])
     ids = bufs.nodes[:nF].contiguous()
     want = oracle.gather(table.numpy(), ids.cpu().numpy())
-    if transport in ("peer", "peer_dev"):
+    if transport == "one_call":
+        # moment_ctx_set_exchange: each batch is ONE library call (moment_gather, then moment_step = sample +
+        # exchange from the ctx's CUDA graph), device barriers inside, nothing host-synchronised between calls
+        nmax = [None] * world
+        dist.all_gather_object(nmax, int(bufs.nodes.numel()))
+        px = PeerExchange(ctx, max(nmax), R, dev, timeout_s=30.0)
+        outs = [px.gather(ids, nF).clone() for _ in range(3)]
+        torch.cuda.synchronize()
+        ok = all(bool(np.array_equal(o.cpu().numpy(), want)) for o in outs)
+        steps = []
+        for rep in range(4):  # rep 0 captures the graph, the others replay it
+            px.step(g.indptr, g.indices, seeds, [10, 5], 900 + rank, bufs)
+            steps.append(px.out[:nF].clone())
+        torch.cuda.synchronize()
+        ok &= int(bufs.counts[2]) == nF
+        ok &= all(bool(np.array_equal(o.cpu().numpy(), want)) for o in steps)
+        # an empty batch on this rank still serves the other's requests
+        out = px.gather(ids, 0 if rank == 0 else nF)
+        torch.cuda.synchronize()
+        if rank == 1:
+            ok &= bool(np.array_equal(out.cpu().numpy(), want))
+        px.check()
+        # the registered output is required: another buffer is refused
+        try:
+            ctx.gather(ids, torch.empty_like(px.out), max_n=nF)
+            ok = False
+        except M.MomentError as e:
+            ok &= e.status == M.EINVAL
+        px.close()
+        info = {"sent": [0] * world, "served": [0] * world}
+    elif transport in ("peer", "peer_dev"):
         # the exchange buffers are sized for the largest batch of any rank; two batches check reuse
         nmax = [None] * world
         dist.all_gather_object(nmax, int(bufs.nodes.numel()))
-        px = PeerExchange(ctx, max(nmax), R, dev, device_barrier=transport == "peer_dev", timeout_s=30.0)
+        px = PeerExchange(ctx, max(nmax), R, dev, device_barrier=transport == "peer_dev", timeout_s=30.0,
+                          one_call=False)
         ok = True
         for rep in range(2):
             out = px.gather(ids, nF)
@@ -137,4 +168,14 @@ def test_peer_exchange_device_barrier_two_processes_one_gpu():
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
     res = run_world(_rank_main, 2, "peer_dev")
+    assert all(r["ok"] for r in res), res
+
+
+def test_one_call_exchange_two_processes_one_gpu():
+    """moment_ctx_set_exchange: the whole relay exchange inside ONE moment_gather / moment_step call per batch
+    (bucket, own reads, peer-store requests, device barrier, peer-store rows, device barrier), replayed from
+    the ctx's CUDA graph with no host barrier between batches; byte-exact with the oracle."""
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    res = run_world(_rank_main, 2, "one_call")
     assert all(r["ok"] for r in res), res
