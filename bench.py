@@ -116,7 +116,138 @@ class State:
         return 1 + 2 * len(self.fanout) + 1 + 1
 
 
-def build_state(name, device="cuda:0", rank=0, world=1, inflight=1):
+NVLINK_GBS = 770.0  # measured B200 peer copy per direction (B200_PROFILING.md; 900 GB/s nominal)
+PRESAMPLE_EPOCH = 2**32 - 1  # R18: the pre-sample batches use their own rng stream
+
+
+class PartState(State):
+    """Resident inputs of one rank with the feature table PARTITIONED over the ranks' HBM (C3: "knapsack
+    placement across 8 GPU caches, max-flow routed"): pre-sampled hotness (P2) summed over the
+    ranks, DDAK placement (P4) over the k HBM bins of an HGX B200 topology graph with the rate max-flow's
+    per-bin traffic (P3), optionally the hottest rows replicated in every bin (R25), and the plan's predicted
+    per-batch time (P5). Each rank holds its own bin; the other ranks' bins are CUDA-IPC mapped, so a batch's
+    peer rows are NVLink loads inside the gather kernel (no exchange: there is no host tier to relay)."""
+
+    def __init__(self, name, device, rank, world, inflight, *, dist, shared, placement="ddak", presample=64,
+                 replicate_frac=1 / 16):
+        import paper_conf_sc_shi0s0x0w25_b200 as M
+
+        self.M = M
+        cfg = W.CONFIGS[name]
+        self.name, self.cfg = name, cfg
+        self.device, self.rank, self.world = device, rank, world
+        self.fanout = tuple(cfg["fanout"])
+        self.B = cfg["batch"]
+        H = len(self.fanout)
+        self.dim, self.dtype = cfg["dim"], cfg["dtype"]
+        self.graph = W.rmat_csr(cfg["n"], cfg["m"], device=device)
+        n = self.graph.n
+        self.R = self.dim * torch.empty(0, dtype=self.dtype).element_size()
+        self.stride = (self.R + 63) // 64 * 64
+        self.train = W.training_set(self.graph, min_count=self.B * world)
+        dev_idx = torch.device(device).index or 0
+        t0 = time.perf_counter()
+        # P2: pre-sampling hotness, every rank its own seeds, counts summed over the ranks
+        ctx0 = M.Ctx(n_vertices=n, max_seeds=self.B, max_fanout=self.fanout, rank=rank, world=world, device=dev_idx)
+        bufs0 = M.SampleBuffers.allocate(self.B, self.fanout, n, device)
+        hot = torch.zeros(n, dtype=torch.int64, device=device)
+        pre = W.epoch_batches(self.train, self.B, PRESAMPLE_EPOCH, rank, world)
+        for b in range(presample):
+            ctx0.step(self.graph.indptr, self.graph.indices, pre[b % len(pre)], self.fanout,
+                      W.batch_rng_seed(RUN_SEED, PRESAMPLE_EPOCH, rank, b), bufs0, None)
+            ctx0.hotness(bufs0.nodes, hot, n_dev=bufs0.counts[H:H + 1], max_n=bufs0.nodes.numel())
+        if dist is not None:
+            if shared:
+                h_cpu = hot.cpu()
+                dist.all_reduce(h_cpu)
+                hot.copy_(h_cpu)
+            else:
+                dist.all_reduce(hot)
+        hot_np = hot.cpu().numpy().astype(np.uint64)
+        del hot, ctx0, bufs0
+        self.t_hotness = time.perf_counter() - t0
+        # P1/P3/P4: topology graph of the box, DDAK over the k HBM bins (rate max-flow traffic, R17a)
+        if world > 8:
+            raise SystemExit("partitioned placement: at most 8 GPUs (one HGX node)")
+        active = M.boxes.spread_gpus(world) if world in (1, 2, 4, 8) else list(range(world))
+        hbm_gbs = _peaks()[0]
+        box = M.boxes.hgx_b200(8, hbm_gbs=hbm_gbs, active=active)
+        topo = box.topology()
+        bin_node = [box.hbm_bin[g] for g in active]
+        r = int(n * replicate_frac) if placement == "ddak-rep" and world > 1 else 0
+        cap = r + -(-(n - r) // world)
+        t1 = time.perf_counter()
+        bin_of, slot_of, A, U, T, rep_acc = M.place(topo, hot_np, [cap] * world, bin_node=bin_node,
+                                                   replicate_rows=r, traffic_mode=M.TRAFFIC_STANDALONE,
+                                                   return_replica_access=True)
+        self.t_place = time.perf_counter() - t1
+        # P5: the plan's predicted per-batch time for this layout (in-sample demand per GPU per batch)
+        N = topo.info()[0]
+        d = np.zeros(N, np.int64)
+        for i, v in enumerate(bin_node):
+            d[v] = int(A[i]) * self.R // (presample * world)
+        self.plan = M.plan(topo, [box.gpu[g] for g in active], d, int(NVLINK_GBS * 1000), int(hbm_gbs * 1000),
+                           replica_demand=int(rep_acc) * self.R // (presample * world)).info()
+        self.placement_mode, self.replicated_rows = placement, r
+        self.bin_rows = [int(x) for x in U]
+        # this rank's HBM bin: replicas at slots 0..r-1, then its partition
+        mine = np.nonzero((bin_of == rank) | (bin_of == M.BIN_REPLICA))[0]
+        rows_mine = r + int(U[rank])
+        self.table = torch.zeros((max(1, rows_mine), self.stride), dtype=torch.uint8, device=device)
+        ch = 1 << 20
+        for c0 in range(0, len(mine), ch):
+            ids = torch.as_tensor(mine[c0:c0 + ch], device=device)
+            sl = torch.as_tensor(slot_of[mine[c0:c0 + ch]], device=device)
+            self.table[sl, :self.R] = W.feature_rows(ids, self.dim, self.dtype)
+        del mine
+        packed = M.place_pack_rank(bin_of, slot_of, rank) if r else M.place_pack(bin_of, slot_of)
+        self.placement = torch.as_tensor(packed.view(np.int64), device=device)
+        del packed, bin_of, slot_of
+        # peer bins: CUDA IPC (NVLink peer pointers between the GPUs of one node)
+        self._imported = []
+        ptrs = [0] * world
+        ptrs[rank] = self.table.data_ptr()
+        if world > 1:
+            mine_h = M.ipc_export(self.table)
+            allh = [None] * world
+            dist.all_gather_object(allh, mine_h)
+            for h in range(world):
+                if h != rank:
+                    base = M.ipc_import(allh[h][0])
+                    self._imported.append(base)
+                    ptrs[h] = base + allh[h][1]
+        streams = [torch.cuda.current_stream(device)] + [torch.cuda.Stream(device) for _ in range(inflight - 1)]
+        self.lanes = []
+        for s_ in streams:
+            L = Lane.__new__(Lane)
+            L.ctx = M.Ctx(n_vertices=n, max_seeds=self.B, max_fanout=self.fanout, rank=rank, world=world,
+                          device=dev_idx, row_bytes=self.R, row_stride=self.stride, bin_owner=list(range(world)),
+                          bin_ptr=ptrs, placement=self.placement)
+            L.bufs = M.SampleBuffers.allocate(self.B, self.fanout, n, device)
+            L.rows = torch.empty((L.bufs.nodes.numel(), self.R), dtype=torch.uint8, device=device)
+            L.stream = s_
+            self.lanes.append(L)
+        self.ctx, self.bufs, self.rows = self.lanes[0].ctx, self.lanes[0].bufs, self.lanes[0].rows
+        self._batches = []
+        self._epoch = 0
+
+    def bins_of(self, nodes, nF):
+        """Rows of a batch per owning bin (measurement bookkeeping, after the timed region)."""
+        b = torch.bitwise_right_shift(self.placement[nodes[:nF]], 40)
+        return torch.bincount(b, minlength=self.world)
+
+    def close(self, dist):
+        torch.cuda.synchronize()
+        if dist is not None:
+            dist.barrier()
+        for base in self._imported:
+            self.M.ipc_close(base)
+        self._imported = []
+
+
+def build_state(name, device="cuda:0", rank=0, world=1, inflight=1, **kw):
+    if kw.get("placement", "replicated") != "replicated":
+        return PartState(name, device, rank, world, inflight, **kw)
     return State(name, device, rank, world, inflight)
 
 
@@ -263,6 +394,48 @@ def oracle_baseline(st, pool, budget_s=10.0):
                        "compared": "counts, F_H, per-hop offsets and src, every gathered row byte"}}
 
 
+def partition_parity(st, pool):
+    """Partitioned placement (no host copy of the table): the parity subset's samples are compared with the
+    oracle's and every gathered row with its generated bytes (the oracle's gather is out[i] = table[ids[i]] with
+    table[v] = featgen(v)); the oracle is timed on sampling only."""
+    import oracle
+
+    oracle.build()
+    info = host_info()
+    H = len(st.fanout)
+    indptr = st.graph.indptr.cpu().numpy()
+    indices = st.graph.indices.cpu().numpy()
+    subset = parity_subset(len(pool))
+    L = st.lanes[0]
+    t, done = 0.0, 0
+    with PinnedCore(info["core"]):
+        for i in subset:
+            seeds, rs = pool[i]
+            t0 = time.perf_counter()
+            r = oracle.sample(indptr, indices, seeds.cpu().numpy(), list(st.fanout), rs)
+            t += time.perf_counter() - t0
+            done += len(seeds)
+            st.step(seeds, rs, lane=0)
+            torch.cuda.synchronize()
+            got = L.bufs.result()
+            nF = int(r["counts"][H])
+            ok = (np.array_equal(got["counts"], r["counts"]) and np.array_equal(got["nodes"], r["nodes"])
+                  and all(np.array_equal(got["offsets"][h], r["offsets"][h]) and
+                          np.array_equal(got["src"][h], r["src"][h]) for h in range(H)))
+            ids = torch.as_tensor(r["nodes"], device=L.rows.device)
+            for c0 in range(0, nF, 1 << 18):
+                ok &= bool(torch.equal(L.rows[c0:min(nF, c0 + (1 << 18))],
+                                       W.feature_rows(ids[c0:c0 + (1 << 18)], st.dim, st.dtype)))
+            if not ok:
+                raise AssertionError(f"bench batch {i}: CUDA path differs from the oracle")
+    return {"value": done / t, "unit": "seeds/s (sampling only)", "cores": 1, "kind": "oracle",
+            "sample": f"parity subset {subset} of {st.name}: oracle sampling timed (the partitioned table has no "
+                      f"host copy to gather from), single thread pinned to core {info['core']}",
+            "host": info,
+            "parity": {"batches": subset, "bit_exact": True,
+                       "compared": "counts, F_H, per-hop offsets and src; every gathered row vs its generated bytes"}}
+
+
 def profile_summary(name):
     """The committed ncu summary of the gather kernel for `name` (per-launch DRAM bytes, launch shares)."""
     path = os.path.join(ROOT, "profiles", "ncu_gather_summary.json")
@@ -356,6 +529,12 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=10.0, help="seconds of oracle time for cpu_baseline")
     # 12-16 measured best on C2 (29.5-29.7 M seeds/s vs 27.7 at 8, 28.4 at 24)
     ap.add_argument("--inflight", type=int, default=16, help="batches in flight per GPU (one stream each)")
+    ap.add_argument("--placement", default="replicated", choices=["replicated", "ddak", "ddak-rep"],
+                    help="replicated: every GPU holds the whole table (C2 'all features in HBM'); ddak: the table "
+                         "partitioned over the GPUs' HBM by DDAK (C3), peer rows read over NVLink; ddak-rep: the "
+                         "same with the hottest --replicate-frac of the rows in every GPU (R25)")
+    ap.add_argument("--presample", type=int, default=64, help="pre-sample batches per rank for DDAK hotness (P2)")
+    ap.add_argument("--replicate-frac", type=float, default=1 / 16)
     args = ap.parse_args()
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         spawn_ranks(args.gpus)
@@ -385,7 +564,10 @@ def main():
         else:
             dist.init_process_group("nccl", device_id=torch.device(dev))
     P = max(1, min(args.inflight, args.steps))
-    st = build_state(args.config, dev, rank, world, P)
+    part = args.placement != "replicated"
+    kw = dict(placement=args.placement, dist=dist, shared=shared, presample=args.presample,
+              replicate_frac=args.replicate_frac) if part else {}
+    st = build_state(args.config, dev, rank, world, P, **kw)
     H = len(st.fanout)
     K = args.steps
     main_stream = torch.cuda.current_stream()
@@ -474,6 +656,45 @@ def main():
     samp_bytes = sum(sum(16 * c[h] for h in range(H)) + sum(8 * e for e in c[H + 1:]) + 8 * c[H]
                      for c in (cnt_pool[i] for i in used))
     gath_bytes = nF_region * (2 * st.R + 8)
+    tiers = None
+    if part:
+        # rows per owning bin of the median region's batches (deterministic: rerun on lane 0), then every
+        # rank's counts, so each rank also knows how many of its bin's rows its peers read over NVLink
+        per_bin = torch.zeros(world, dtype=torch.int64, device=dev)
+        for i in sorted(set(used)):
+            L0.ctx.step(st.graph.indptr, st.graph.indices, pool[i][0], st.fanout, pool[i][1], L0.bufs, None,
+                        stream=main_stream)
+            per_bin += st.bins_of(L0.bufs.nodes, nF_pool[i]) * used.count(i)
+        allb = [torch.zeros_like(per_bin) for _ in range(world)]
+        if dist:
+            if shared:
+                allc = [torch.zeros(world, dtype=torch.int64) for _ in range(world)]
+                dist.all_gather(allc, per_bin.cpu())
+                allb = [c.to(dev) for c in allc]
+            else:
+                dist.all_gather(allb, per_bin)
+        else:
+            allb = [per_bin]
+        mat = torch.stack(allb).cpu().numpy() / K  # [requester][owner] rows per batch
+        local = mat[rank, rank]
+        peer_in = mat[rank].sum() - local
+        peer_out = mat[:, rank].sum() - local
+        nf_b = nF_region / K
+        hbm_b = (local + peer_out) * st.R + nf_b * (st.R + 8) + samp_bytes / K
+        t_hbm = hbm_b / (_peaks()[0] * 1e9)
+        t_nvl = max(peer_in, peer_out) * st.R / (NVLINK_GBS * 1e9)
+        t_meas = ms / K / 1000
+        tiers = {"placement": st.placement_mode, "replicated_rows": st.replicated_rows, "bin_rows": st.bin_rows,
+                 "rows_per_batch": {"local_hbm": local, "peer_in_nvlink": peer_in, "served_to_peers_nvlink": peer_out},
+                 "bytes_per_batch": {"hbm": hbm_b, "nvlink_in": peer_in * st.R, "nvlink_out": peer_out * st.R},
+                 "t_us": {"hbm": t_hbm * 1e6, "nvlink": t_nvl * 1e6, "measured": t_meas * 1e6},
+                 "binding": "nvlink" if t_nvl > t_hbm else "hbm", "frac": max(t_hbm, t_nvl) / t_meas,
+                 "peaks": {"hbm_gbs": _peaks()[0], "nvlink_gbs": NVLINK_GBS,
+                           "nvlink_source": "measured B200 peer copy per direction (B200_PROFILING.md; 900 nominal)"},
+                 "plan": {"t_star_us": st.plan["t_star"], "t_nvlink_us": st.plan["t_nvlink"],
+                          "t_hbm_us": st.plan["t_hbm"],
+                          "note": "the plan predicts the gather per batch (P:L229-235, P:L339)"},
+                 "offline_s": {"hotness": st.t_hotness, "ddak": st.t_place}}
     # roofline pass: CUDA events around the dominant kernel (the gather) on its stream, one lane, one batch
     # at a time, over the pool
     n_roof = min(n_pool, 256)
@@ -547,7 +768,7 @@ def main():
     e2e_val = world * st.B * K / (e2e_ms / 1000)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = oracle_baseline(st, pool, args.cpu_budget)
+        cpu = oracle_baseline(st, pool, args.cpu_budget) if not part else partition_parity(st, pool)
     if rank == 0:
         line = {
             "metric": METRIC, "value": seeds_per_s, "unit": "seeds/s", "n_gpus": world, "steps": K,
@@ -606,7 +827,20 @@ def main():
             "gpu_launches": st.launches_per_step() * K,
             "clocks": ck,
         }
+        if part:
+            tiers["plan"]["gather_us_measured"] = gather_ms * 1000
+            line["tiers"] = tiers
+            line["config"]["parallelism"] = f"dp{world}, features DDAK-partitioned over {world} HBM bins" + (
+                f" + {st.replicated_rows} replicated rows" if st.replicated_rows else "")
+            line["config"]["l2"] = "no flush: inputs larger than L2 (features %.2f GB over all GPUs, CSR %.2f GB)" % (
+                st.graph.n * st.stride / 1e9, (st.graph.indptr.numel() * 8 + st.graph.indices.numel() * 4) / 1e9)
+            line["roofline"]["kernel"] = "gather_kernel (placement map; peer rows over NVLink)"
+            line["roofline"]["traffic"] = None
+            line["roofline"]["launch_shares"] = None
+            line["roofline"]["why_this_kernel"] = None
         print(json.dumps(line), flush=True)
+    if part:
+        st.close(dist)
     if dist:
         dist.barrier()
         dist.destroy_process_group()

@@ -42,3 +42,49 @@ def test_bench_driver_args_c1(steps, warmup):
     assert 0 < line["roofline"]["frac"] < 1.5
     assert line["cpu_baseline"]["parity"]["bit_exact"]
     assert line["config"]["region_ms"]["n"] >= 3
+
+
+def _run_torchrun(nproc, args, env=None, timeout=900):
+    import socket
+
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    e = dict(os.environ)
+    e.update(env or {})
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.join(ROOT, "bench.py")] + args
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=timeout, cwd=ROOT, env=e)
+    assert r.returncode == 0, r.stderr[-4000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    return json.loads(lines[0])
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("placement", ["ddak", "ddak-rep"])
+def test_bench_partitioned_one_rank(placement):
+    """N = 1: the partitioned path (placement map, DDAK over one HBM bin) with the parity subset checked."""
+    line = _run(["--config", "C1", "--placement", placement, "--steps", "20", "--warmup", "3", "--min-time", "0.2",
+                 "--e2e-min-time", "0.1", "--presample", "8"])
+    assert line["cpu_baseline"]["parity"]["bit_exact"]
+    t = line["tiers"]
+    assert t["rows_per_batch"]["peer_in_nvlink"] == 0 and t["rows_per_batch"]["local_hbm"] > 0
+    assert t["plan"]["t_star_us"] >= 0
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("placement", ["ddak", "ddak-rep"])
+def test_bench_partitioned_two_ranks_shared_gpu(placement):
+    """N = 2 ranks sharing cuda:0 over gloo (MOMENT_BENCH_SHARED_GPU: the multi-rank code path on a one-GPU box,
+    never a bench number): the table is split over the two ranks' bins, each maps the other's by CUDA IPC,
+    and every batch reads peer rows; DDAK's bins partition the non-replicated rows."""
+    line = _run_torchrun(2, ["--gpus", "2", "--config", "C1", "--placement", placement, "--steps", "10",
+                             "--warmup", "3", "--min-time", "0.1", "--e2e-min-time", "0.05", "--presample", "8"],
+                         env={"MOMENT_BENCH_SHARED_GPU": "1"})
+    assert line["n_gpus"] == 2 and "test_mode" in line["config"]
+    t = line["tiers"]
+    assert t["rows_per_batch"]["peer_in_nvlink"] > 0 and t["rows_per_batch"]["served_to_peers_nvlink"] > 0
+    assert sum(t["bin_rows"]) == (1 << 16) - t["replicated_rows"]  # a partition of the non-replicated rows
+    if placement == "ddak-rep":
+        assert t["replicated_rows"] > 0
