@@ -26,6 +26,13 @@ class Box:
     hbm_bin: list = field(default_factory=list)    # node of GPU g's HBM bin
     gpu: list = field(default_factory=list)        # computation node of GPU g
     socket_of_gpu: list = field(default_factory=list)
+    rc: list = field(default_factory=list)         # interconnect node of socket j's root complex
+    upi_links: list = field(default_factory=list)  # indices (in `links`) of the socket-to-socket links
+
+    def upi_bytes(self, link_flow) -> int:
+        """Bytes a plan's flow moves across sockets (the paper's QPI traffic): the flow on the
+        UPI links (link indices are those of `links`, which the topology export keeps)."""
+        return int(sum(int(link_flow[i]) for i in self.upi_links))
 
     def topology(self) -> M.Topology:
         return M.topology(self.nodes, self.links)
@@ -63,9 +70,11 @@ def hgx_b200(k_total: int = 8, *, port_gbs: float = 55.6, hbm_gbs: float = 6543.
             nodes.append((M.NODE_COMPUTE, M.TIER_NONE, g))
     for j in range(sockets):
         links.append((b.host_bin[j], rc[j], cap(dram_gbs)))
+    b.rc = rc
     for j in range(sockets):
         for i in range(sockets):
             if i != j:
+                b.upi_links.append(len(links))
                 links.append((rc[j], rc[i], cap(upi_gbs)))
     per_socket = k_total // sockets
     for g in range(k_total):
@@ -116,3 +125,34 @@ def gpu_subset_classes(k: int, k_total: int = 8, sockets: int = 2, gpus_per_swit
         if sig not in reps:
             reps[sig] = list(sub)
     return sorted(reps.values())
+
+
+# Capacities of hgx_b200 that this pool's boxes cannot measure (one GPU, one socket): assumptions for a
+# two-socket HGX B200 host.
+ASSUMED = {"dram_gbs": 250.0, "upi_gbs": 62.0}
+
+
+def from_probe(probe: dict) -> tuple[dict, dict]:
+    """hgx_b200 keyword arguments from a tools/probe_box.py JSON (capacities are profiled limits),
+    and the provenance of each: {"port_gbs": "measured", "upi_gbs": "assumed", ...}.
+    port = the slowest GPU's local-NUMA pinned H2D copy (or, when every GPU copied at once, the slowest
+    concurrent rate); hbm = the device copy (read + write); nvlink = the peer copy when the box has 2+ GPUs
+    (else the B200_PROFILING.md figure, 770 GB/s); UPI = the remote-NUMA H2D rate when the box has 2+ NUMA
+    nodes (a lower bound on what one GPU can pull across sockets), else assumed; socket DRAM assumed."""
+    kw, src = {}, {}
+    conc = probe.get("port_concurrent_gbs")
+    kw["port_gbs"] = float(min(conc)) if conc else float(probe["port_gbs"])
+    src["port_gbs"] = "measured (concurrent)" if conc else "measured (one GPU at a time)"
+    kw["hbm_gbs"] = float(probe["hbm_gbs"])
+    src["hbm_gbs"] = "measured"
+    if probe.get("port_remote_gbs"):
+        kw["upi_gbs"] = float(probe["port_remote_gbs"])
+        src["upi_gbs"] = "measured (remote-NUMA H2D, lower bound)"
+    else:
+        kw["upi_gbs"] = ASSUMED["upi_gbs"]
+        src["upi_gbs"] = "assumed"
+    kw["dram_gbs"] = ASSUMED["dram_gbs"]
+    src["dram_gbs"] = "assumed"
+    nv = probe.get("nvlink_gbs")
+    src["nvlink_gbs"] = "measured (peer copy)" if nv else "B200_PROFILING.md peer copy (770 GB/s)"
+    return kw, dict(src, nvlink_value=float(nv) if nv else 770.0)

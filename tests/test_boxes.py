@@ -99,3 +99,39 @@ def test_subset_choice_matters_with_shared_switches():
             d[v] += int(A[i]) * R
         out[tuple(act)] = M.plan(topo, [box.gpu[g] for g in act], d, 900000, 6543400).info()["t_ingest"]
     assert out[(0, 1)] >= 2 * out[(0, 2)] - 1
+
+
+def test_upi_bytes_closed_form():
+    # all host demand on socket 0's bin, 8 GPUs: the 4 socket-1 ports can only be fed across UPI, so at T*
+    # = ceil(8 d / (4 p + u)) (ports p, UPI u, ample DRAM) the plan moves u T* (rounded to the flow) over UPI
+    p, u, d = 50_000, 20_000, 3_000_000
+    box = M.boxes.hgx_b200(8, port_gbs=p / 1000, upi_gbs=u / 1000, dram_gbs=10_000)
+    topo = box.topology()
+    N, _, s, t = topo.info()
+    _, links, _, _ = topo.export()
+    assert all(links[i][0] in box.rc and links[i][1] in box.rc for i in box.upi_links) and len(box.upi_links) == 2
+    dem = np.zeros(N, np.int64)
+    dem[box.host_bin[0]] = d
+    plan = M.plan(topo, box.gpu, dem, 770_000, 6_500_000).info()
+    T = plan["t_ingest"]
+    assert T == -(-8 * d // (4 * p + u))
+    upi = box.upi_bytes(plan["link_flow"])
+    assert 8 * d - 4 * p * T <= upi <= u * T  # what the socket-0 ports cannot take crosses, within capacity
+    # symmetric demand: no reason to cross sockets at all at T* = ceil(8 d / 8 p)
+    dem[box.host_bin[1]] = d
+    plan = M.plan(topo, box.gpu, dem, 770_000, 6_500_000).info()
+    assert plan["t_ingest"] == -(-8 * d // (4 * p))
+    assert box.upi_bytes(plan["link_flow"]) <= u * plan["t_ingest"]
+
+
+def test_from_probe_provenance():
+    one_gpu = {"gpus": 1, "port_gbs": 55.6, "port_remote_gbs": None, "port_concurrent_gbs": None,
+               "hbm_gbs": 6500.0, "nvlink_gbs": None}
+    kw, src = M.boxes.from_probe(one_gpu)
+    assert kw["port_gbs"] == 55.6 and kw["hbm_gbs"] == 6500.0
+    assert src["upi_gbs"] == "assumed" and src["dram_gbs"] == "assumed" and src["nvlink_value"] == 770.0
+    eight = dict(one_gpu, gpus=8, port_remote_gbs=40.0, port_concurrent_gbs=[50.0] * 7 + [45.0], nvlink_gbs=760.0)
+    kw, src = M.boxes.from_probe(eight)
+    assert kw["port_gbs"] == 45.0 and kw["upi_gbs"] == 40.0 and src["nvlink_value"] == 760.0
+    assert src["port_gbs"].startswith("measured")
+    M.boxes.hgx_b200(8, **kw)  # builds

@@ -1,50 +1,193 @@
-"""Box probe: host/GPU topology facts and link bandwidths.
+"""Box probe (the paper builds its capacity graph from profiled link limits):
+measures the capacities the planner's topology graph needs on THIS box and writes them as JSON that
+`boxes.from_probe` turns into `boxes.hgx_b200` arguments (each capacity tagged measured / assumed).
 
-Writes gpurun_out/probe.json. Not part of the product; plain torch only.
+    python tools/probe_box.py [--out gpurun_out/probe.json]
+
+Measured here (CUDA events, best of several):
+  * hbm_gbs          device copy, read + write bytes (the HBM bin -> GPU link)
+  * port_gbs         pinned host -> device copy per GPU with the host buffer on the GPU's own NUMA node
+                     (the GPU's PCIe port), alone; port_concurrent_gbs: every GPU at once (a shared uplink or
+                     socket DRAM limit shows as a lower per-GPU rate)
+  * port_remote_gbs  the same with the buffer on another NUMA node (crosses UPI), if the box has > 1 node
+  * zero_copy_gbs    SM-issued zero-copy reads of pinned host rows by the library's own gather (the tier the
+                     product reads host rows through)
+  * nvlink_gbs       peer copy GPU 0 -> GPU 1 per direction, if the box has > 1 GPU
+Not measurable from a process (assumed unless the box shows them): socket DRAM bandwidth and UPI capacity
+beyond what port_remote_gbs bounds.
 """
-import json, os, subprocess, time
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+
 import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
 
 def sh(cmd):
     try:
         return subprocess.run(cmd, shell=True, capture_output=True, text=True, timeout=60).stdout
-    except Exception as e:  # noqa
+    except Exception as e:  # noqa: BLE001
         return f"ERR {e}"
 
-out = {}
-out["lscpu"] = sh("lscpu")
-out["meminfo"] = sh("head -5 /proc/meminfo")
-out["numa"] = sh("numactl -H 2>/dev/null || ls /sys/devices/system/node/")
-out["nproc"] = os.cpu_count()
-out["smi_topo"] = sh("nvidia-smi topo -m")
-out["smi_q"] = sh("nvidia-smi -q | grep -iE 'Product Name|Bus Id|Link Width|PCIe Generation|Max|Current' | head -60")
-out["hugepages"] = sh("grep -i huge /proc/meminfo")
-dev = torch.device("cuda:0")
-props = torch.cuda.get_device_properties(0)
-out["sm_count"] = props.multi_processor_count
-out["total_mem"] = props.total_memory
 
-def bw(fn, nbytes, reps=10):
-    fn(); torch.cuda.synchronize()
-    s = torch.cuda.Event(enable_timing=True); e = torch.cuda.Event(enable_timing=True)
-    best = 1e9
-    for _ in range(reps):
-        s.record(); fn(); e.record(); torch.cuda.synchronize()
-        best = min(best, s.elapsed_time(e))
+def numa_nodes():
+    base = "/sys/devices/system/node"
+    nodes = {}
+    try:
+        for d in sorted(os.listdir(base)):
+            if d.startswith("node") and d[4:].isdigit():
+                cpus = set()
+                with open(os.path.join(base, d, "cpulist")) as f:
+                    for part in f.read().strip().split(","):
+                        if part:
+                            a, _, b = part.partition("-")
+                            cpus.update(range(int(a), int(b or a) + 1))
+                if cpus:
+                    nodes[int(d[4:])] = sorted(cpus)
+    except OSError:
+        pass
+    return nodes or {0: sorted(os.sched_getaffinity(0))}
+
+
+def gpu_numa(i):
+    """NUMA node of GPU i's PCIe function (sysfs), 0 if unknown."""
+    try:
+        bus = torch.cuda.get_device_properties(i).pci_bus_id if hasattr(torch.cuda.get_device_properties(i), "pci_bus_id") else None
+    except Exception:  # noqa: BLE001
+        bus = None
+    if bus is None:
+        out = sh(f"nvidia-smi -i {i} --query-gpu=pci.bus_id --format=csv,noheader").strip()
+        bus = out or None
+    if bus:
+        bus = bus.lower()
+        if bus.count(":") == 2 and len(bus.split(":")[0]) == 8:
+            bus = bus[4:]
+        try:
+            with open(f"/sys/bus/pci/devices/{bus}/numa_node") as f:
+                v = int(f.read().strip())
+                return max(v, 0)
+        except OSError:
+            pass
+    return 0
+
+
+def timed(fn, nbytes, dev, reps=8):
+    with torch.cuda.device(dev):
+        fn()
+        torch.cuda.synchronize(dev)
+        best = 1e30
+        for _ in range(reps):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            fn()
+            b.record()
+            torch.cuda.synchronize(dev)
+            best = min(best, a.elapsed_time(b))
     return nbytes / (best * 1e-3) / 1e9
 
-N = 1 << 30
-h = torch.empty(N, dtype=torch.uint8, pin_memory=True)
-d = torch.empty(N, dtype=torch.uint8, device=dev)
-out["h2d_pinned_GBs"] = bw(lambda: d.copy_(h, non_blocking=True), N)
-out["d2h_pinned_GBs"] = bw(lambda: h.copy_(d, non_blocking=True), N)
-d2 = torch.empty_like(d)
-out["d2d_copy_GBs_rw"] = bw(lambda: d2.copy_(d), 2 * N)
-# random row gather in HBM (torch index_select), 400 B rows
-tab = torch.empty((2_449_029, 100), dtype=torch.float32, device=dev)
-idx = torch.randint(0, tab.shape[0], (700_000,), device=dev)
-o = torch.empty((idx.numel(), 100), dtype=torch.float32, device=dev)
-out["torch_index_select_400B_GBs_rw"] = bw(lambda: torch.index_select(tab, 0, idx, out=o), 2 * idx.numel() * 400)
-# zero-copy: gather from pinned host via index_select on a mapped view is not expressible in torch; use UVA via cuda-python later
-json.dump(out, open("gpurun_out/probe.json", "w"), indent=1)
-print(json.dumps({k: v for k, v in out.items() if not isinstance(v, str)}, indent=1))
+
+def pinned_on(node_cpus, nbytes):
+    """A pinned host buffer whose pages were first touched from a core of the given NUMA node."""
+    old = os.sched_getaffinity(0)
+    try:
+        os.sched_setaffinity(0, set(node_cpus))
+        h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+        h.fill_(1)
+    finally:
+        os.sched_setaffinity(0, old)
+    return h
+
+
+def zero_copy_gbs(dev, host_rows, R=512):
+    """The library's gather reading every row zero-copy from a pinned host table (bin 0 on the host)."""
+    import paper_conf_sc_shi0s0x0w25_b200 as M
+
+    n = host_rows.shape[0]
+    ctx = M.Ctx(n_vertices=n, max_seeds=1, max_fanout=[1], device=dev.index or 0, row_bytes=R, bin_owner=[-1],
+                bin_ptr=[host_rows.data_ptr()])
+    m = 1 << 18
+    ids = torch.randint(0, n, (m,), device=dev, dtype=torch.int64)
+    out = torch.empty((m, R), dtype=torch.uint8, device=dev)
+    return timed(lambda: ctx.gather(ids, out), m * R, dev)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--out", default="gpurun_out/probe.json")
+    ap.add_argument("--mib", type=int, default=1024)
+    a = ap.parse_args()
+    nb = a.mib << 20
+    nodes = numa_nodes()
+    k = torch.cuda.device_count()
+    res = {"gpus": k, "numa_nodes": len(nodes), "cpu_count": os.cpu_count(),
+           "cpu_model": next((l.split(":", 1)[1].strip() for l in sh("lscpu").splitlines()
+                              if l.startswith("Model name:")), None),
+           "gpu_name": torch.cuda.get_device_name(0), "gpu_numa": [gpu_numa(i) for i in range(k)],
+           "sm_count": torch.cuda.get_device_properties(0).multi_processor_count,
+           "smi_topo": sh("nvidia-smi topo -m")}
+    d0 = torch.device("cuda:0")
+    x = torch.empty(nb, dtype=torch.uint8, device=d0)
+    y = torch.empty_like(x)
+    res["hbm_gbs"] = timed(lambda: y.copy_(x), 2 * nb, d0)
+    del y
+    port, remote = [], []
+    for i in range(k):
+        di = torch.device(f"cuda:{i}")
+        xi = torch.empty(nb, dtype=torch.uint8, device=di)
+        loc = res["gpu_numa"][i] if res["gpu_numa"][i] in nodes else next(iter(nodes))
+        h = pinned_on(nodes[loc], nb)
+        port.append(timed(lambda: xi.copy_(h, non_blocking=True), nb, di))
+        others = [j for j in nodes if j != loc]
+        if others:
+            hr = pinned_on(nodes[others[0]], nb)
+            remote.append(timed(lambda: xi.copy_(hr, non_blocking=True), nb, di))
+            del hr
+        del h, xi
+    res["port_gbs_per_gpu"] = port
+    res["port_gbs"] = min(port)
+    res["port_remote_gbs"] = min(remote) if remote else None
+    if k > 1:  # every GPU's port at once: per-GPU rate under contention
+        bufs = []
+        for i in range(k):
+            di = torch.device(f"cuda:{i}")
+            loc = res["gpu_numa"][i] if res["gpu_numa"][i] in nodes else next(iter(nodes))
+            bufs.append((di, torch.empty(nb, dtype=torch.uint8, device=di), pinned_on(nodes[loc], nb)))
+        rates = [0.0] * k
+
+        def run(i):
+            di, xi, hi = bufs[i]
+            rates[i] = timed(lambda: xi.copy_(hi, non_blocking=True), nb, di, reps=4)
+
+        th = [threading.Thread(target=run, args=(i,)) for i in range(k)]
+        for t in th:
+            t.start()
+        for t in th:
+            t.join()
+        res["port_concurrent_gbs"] = rates
+        del bufs
+        d1 = torch.device("cuda:1")
+        z = torch.empty(nb, dtype=torch.uint8, device=d1)
+        res["nvlink_gbs"] = timed(lambda: z.copy_(x), nb, d0)
+        del z
+    else:
+        res["port_concurrent_gbs"] = None
+        res["nvlink_gbs"] = None
+    rows = (256 << 20) // 512
+    host_rows = torch.empty((rows, 512), dtype=torch.uint8, pin_memory=True)
+    res["zero_copy_gbs"] = zero_copy_gbs(d0, host_rows)
+    res["measured"] = [key for key in ("hbm_gbs", "port_gbs", "port_remote_gbs", "nvlink_gbs", "zero_copy_gbs")
+                       if res.get(key) is not None]
+    os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
+    with open(a.out, "w") as f:
+        json.dump(res, f, indent=1)
+    print(json.dumps({kk: v for kk, v in res.items() if kk != "smi_topo"}))
+
+
+if __name__ == "__main__":
+    main()

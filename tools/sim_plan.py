@@ -69,8 +69,9 @@ def counts(cfg, batches, held):
     return out[0], out[1], nF / 8
 
 
-def breakdown(topo, box, active, hot, dem, caps, bin_node, R, held, r, nv, hbm):
-    b, s, A, U, T = M.place(topo, hot, caps, bin_node=bin_node, replicate_rows=r, traffic_mode=M.TRAFFIC_STANDALONE)
+def breakdown(topo, box, active, hot, dem, caps, bin_node, R, held, r, nv, hbm, mode=M.PLACE_DDAK):
+    b, s, A, U, T = M.place(topo, hot, caps, bin_node=bin_node, replicate_rows=r, traffic_mode=M.TRAFFIC_STANDALONE,
+                            mode=mode)
     N = topo.info()[0]
     per_bin = np.bincount(b.astype(np.int64) + 2, weights=dem.astype(np.float64), minlength=len(bin_node) + 2)
     d = np.zeros(N, np.int64)
@@ -83,12 +84,20 @@ def breakdown(topo, box, active, hot, dem, caps, bin_node, R, held, r, nv, hbm):
             "partition_rows_hbm": hbm_rows, "host_rows": int(U[len(active):].sum()),
             "host_bytes_per_gpu_batch": int(sum(d[v] for v in box.host_bin)),
             "peer_bytes_per_gpu_batch": int(sum(d[box.hbm_bin[g]] for g in active) * (len(active) - 1) // len(active)),
-            "replica_bytes_per_gpu_batch": rep * R // held}
+            "replica_bytes_per_gpu_batch": rep * R // held,
+            # the paper's QPI traffic: host bytes of all k GPUs' batches that cross sockets in
+            # the plan's ingest flow (UPI links), per batch
+            "upi_bytes_per_batch": box.upi_bytes(p["link_flow"]),
+            "host_bytes_per_batch_all_gpus": int(sum(d[v] for v in box.host_bin)) * len(active)}
 
 
-def evaluate(name, cfg, hot, dem, R, k, active, cap_gpu, a, hbm_gbs, nv_gbs, mean_fh, t_hot, gps):
+def evaluate(name, cfg, hot, dem, R, k, active, cap_gpu, a, hbm_gbs, nv_gbs, mean_fh, t_hot, gps, box_kw=None,
+             provenance=None):
     n = len(hot)
-    box = M.boxes.hgx_b200(8, hbm_gbs=hbm_gbs, gpus_per_switch=gps, active=active)
+    kw = dict(box_kw or {})
+    kw.setdefault("hbm_gbs", hbm_gbs)
+    hbm_gbs = kw["hbm_gbs"]
+    box = M.boxes.hgx_b200(8, gpus_per_switch=gps, active=active, **kw)
     topo = box.topology()
     bin_node = [box.hbm_bin[g] for g in active] + box.host_bin
     caps = [cap_gpu] * k + [n, n]
@@ -102,19 +111,26 @@ def evaluate(name, cfg, hot, dem, R, k, active, cap_gpu, a, hbm_gbs, nv_gbs, mea
     nv, hb = int(nv_gbs * 1000), int(hbm_gbs * 1000)
     b0 = breakdown(topo, box, active, hot, dem, caps, bin_node, R, a.held, 0, nv, hb)
     bb = breakdown(topo, box, active, hot, dem, caps, bin_node, R, a.held, cand[best], nv, hb)
+    bh = breakdown(topo, box, active, hot, dem, caps, bin_node, R, a.held, 0, nv, hb, mode=M.PLACE_HASH)
     line = {"config": name, "k": k, "active_gpus": active, "gpus_per_switch": gps, "row_bytes": R,
             "n": n, "hbm_budget_rows_per_gpu": cap_gpu, "pre_sample_batches": a.batches, "held_out_batches": a.held,
             "mean_F_H": mean_fh, "candidates_r": cand, "t_star_us": [int(x) for x in ts],
-            "best_r": cand[best], "ddak": b0, "ddak_replicated": bb,
+            "best_r": cand[best], "ddak": b0, "ddak_replicated": bb, "hash": bh,
+            "ddak_over_hash_t_star": bh["t_star"] / max(1, b0["t_star"]),
             "pred_seeds_per_s_ddak": k * cfg["batch"] / (b0["t_star"] * 1e-6),
             "pred_seeds_per_s_best": k * cfg["batch"] / (bb["t_star"] * 1e-6),
             "search_s": t_search, "hotness_s": t_hot,
-            "assumed": {"nvlink_gbs": nv_gbs, "dram_gbs": 250.0, "upi_gbs": 62.0, "port_gbs": 55.6,
-                        "hbm_gbs": hbm_gbs}}
+            "capacities": {"nvlink_gbs": nv_gbs, "hbm_gbs": hbm_gbs,
+                           **{kk: kw.get(kk, dflt) for kk, dflt in (("dram_gbs", 250.0), ("upi_gbs", 62.0),
+                                                                    ("port_gbs", 55.6))}},
+            "provenance": provenance or {"port_gbs": "measured r01 (55.6)", "hbm_gbs": "MEASURED_PEAKS.json",
+                                         "nvlink_gbs": "B200_PROFILING.md peer copy", "dram_gbs": "assumed",
+                                         "upi_gbs": "assumed"}}
     print(f"{name} k={k} gpus={active} per-switch={gps}: T*(r) {list(zip(cand, [int(x) for x in ts]))} best r={cand[best]}; "
           f"DDAK T*={b0['t_star']} (ing {b0['t_ingest']}, nv {b0['t_nvlink']}, hbm {b0['t_hbm']}) "
           f"-> +repl T*={bb['t_star']} (ing {bb['t_ingest']}, nv {bb['t_nvlink']}, hbm {bb['t_hbm']}); "
-          f"pred {line['pred_seeds_per_s_ddak']/1e6:.2f} -> {line['pred_seeds_per_s_best']/1e6:.2f} M seeds/s "
+          f"pred {line['pred_seeds_per_s_ddak']/1e6:.2f} -> {line['pred_seeds_per_s_best']/1e6:.2f} M seeds/s; "
+          f"hash T*={bh['t_star']} UPI {bh['upi_bytes_per_batch']/1e6:.1f} MB vs DDAK {b0['upi_bytes_per_batch']/1e6:.1f} MB "
           f"(search {t_search:.1f} s)", flush=True)
     return line
 
@@ -131,7 +147,13 @@ def main():
     ap.add_argument("--subsets", action="store_true",
                     help="evaluate every class of active-GPU sets up to the box symmetry (P:L229-233)")
     ap.add_argument("--out", default="gpurun_out/plan_sim.jsonl")
+    ap.add_argument("--probe", default=None, help="tools/probe_box.py JSON: measured capacities for the graph")
     a = ap.parse_args()
+    box_kw, prov = None, None
+    if a.probe:
+        with open(a.probe) as f:
+            box_kw, prov = M.boxes.from_probe(json.load(f))
+        a.nvlink_gbs = prov.pop("nvlink_value")
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
         os.path.join(ROOT, "MEASURED_PEAKS.json")) else {"hbm_gbs": 6543.4}
     hbm_gbs = float(peaks["hbm_gbs"])
@@ -150,7 +172,8 @@ def main():
             subsets = (M.boxes.gpu_subset_classes(k, gpus_per_switch=gps) if a.subsets
                        else [M.boxes.spread_gpus(k, gpus_per_switch=gps)])
             for active in subsets:
-                line = evaluate(name, cfg, hot, dem, R, k, active, cap_gpu, a, hbm_gbs, nv_gbs, mean_fh, t_hot, gps)
+                line = evaluate(name, cfg, hot, dem, R, k, active, cap_gpu, a, hbm_gbs, a.nvlink_gbs, mean_fh, t_hot,
+                                gps, box_kw, prov)
                 fout.write(json.dumps(line) + "\n")
                 fout.flush()
         del hot, dem
