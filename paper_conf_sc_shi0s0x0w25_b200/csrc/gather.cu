@@ -171,29 +171,36 @@ __global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const ui
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     __syncwarp();
     const int64_t t0 = blockIdx.x, dt = gridDim.x;
-    // the row id of this lane in `tile` (loaded ahead of time: an id load never sits on the issue path)
-    auto load_id = [&](int64_t tile) -> int64_t {
+    // the source row of this lane in `tile`, resolved ahead of time (id load, then the placement lookup):
+    // neither dependent load sits on the issue path
+    auto load_id = [&](int64_t tile) -> const char* {
         const int64_t r = tile * rows_per_tile + lane;
-        return (tile < n_tiles && lane < rows_per_tile && r < n) ? __ldg(ids + r) : -1;
+        return (tile < n_tiles && lane < rows_per_tile && r < n) ? row_src(bins, placement, __ldg(ids + r), stride)
+                                                                 : nullptr;
     };
-    auto issue = [&](int64_t tile, int s, int64_t id) {
+    auto issue = [&](int64_t tile, int s, const char* src) {
         const int64_t row0 = tile * rows_per_tile;
         const int rows = (int)min((int64_t)rows_per_tile, n - row0);
         if (lane == 0) mbar_expect_tx(&full[s], (uint32_t)rows * R);
         __syncwarp();
-        if (lane < rows)
-            bulk_load(stage + ((size_t)s * rows_per_tile + lane) * R, row_src(bins, placement, id, stride), R, &full[s],
-                      pol_ld);
+        if (lane < rows) bulk_load(stage + ((size_t)s * rows_per_tile + lane) * R, src, R, &full[s], pol_ld);
     };
-    // prologue: all ids of the first kBulkStages tiles in flight together, then fill the pipeline
-    int64_t pre[kBulkStages];
+    // prologue: all ids of the first kBulkStages tiles in flight together, then their placement words, then
+    // fill the pipeline
+    int64_t pid[kBulkStages];
 #pragma unroll
-    for (int s = 0; s < kBulkStages; s++) pre[s] = load_id(t0 + s * dt);
+    for (int s = 0; s < kBulkStages; s++) {
+        const int64_t tile = t0 + s * dt, r = tile * rows_per_tile + lane;
+        pid[s] = (tile < n_tiles && lane < rows_per_tile && r < n) ? __ldg(ids + r) : -1;
+    }
+    const char* pre[kBulkStages];
+#pragma unroll
+    for (int s = 0; s < kBulkStages; s++) pre[s] = pid[s] >= 0 ? row_src(bins, placement, pid[s], stride) : nullptr;
     int64_t next = t0;
 #pragma unroll
     for (int s = 0; s < kBulkStages; s++, next += dt)
         if (next < n_tiles) issue(next, s, pre[s]);
-    int64_t next_id = load_id(next);
+    const char* next_id = load_id(next);
     // steady state: store the tile that landed, then refill the stage of the PREVIOUS tile, whose store
     // was issued one iteration ago (wait_group.read 1: every store but the newest has read its stage).
     int it = 0;
@@ -227,6 +234,7 @@ template <int kStages>
 __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__ CUtensorMap tmap,
                                                          const int64_t* __restrict__ ids, const int64_t* n_dev,
                                                          int64_t max_n, uint32_t R, int l2_load, int l2_store,
+                                                         const uint64_t* __restrict__ placement,
                                                          char* __restrict__ out) {
     extern __shared__ __align__(128) char stage[];  // kStages * 8 * G
     __shared__ __align__(8) uint64_t full[kStages];
@@ -239,11 +247,16 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
     // the count instead of after it: one dependent global round trip fewer before the first row request.
     // Ids past the count are never used (issue() replaces them by the tile's first row).
     int32_t pre[kStages];
+    int64_t pid[kStages];
 #pragma unroll
     for (int s = 0; s < kStages; s++) {
         const int64_t r = (t0 + s * dt) * kTma4Rows + lane;
-        pre[s] = r < max_n ? (int32_t)__ldg(ids + r) : -1;
+        pid[s] = r < max_n ? __ldg(ids + r) : -1;
     }
+    // with a placement map (one local bin, e.g. a DDAK layout on one GPU) the row coordinate is the slot
+#pragma unroll
+    for (int s = 0; s < kStages; s++)
+        pre[s] = pid[s] < 0 ? -1 : placement ? (int32_t)(dev::ld_rand(placement + pid[s]) & kSlotMask) : (int32_t)pid[s];
     const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
     const int64_t n_tiles = (n + kTma4Rows - 1) / kTma4Rows;
     if (lane == 0)
@@ -252,7 +265,9 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
     __syncwarp();
     auto load_id = [&](int64_t tile) -> int32_t {
         const int64_t r = tile * kTma4Rows + lane;
-        return (tile < n_tiles && r < n) ? (int32_t)__ldg(ids + r) : -1;
+        if (!(tile < n_tiles && r < n)) return -1;
+        const int64_t id = __ldg(ids + r);
+        return placement ? (int32_t)(dev::ld_rand(placement + id) & kSlotMask) : (int32_t)id;
     };
     auto issue = [&](int64_t tile, int s, int32_t id) {
         const int rows = (int)min((int64_t)kTma4Rows, n - tile * kTma4Rows);
@@ -553,7 +568,9 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
     for (int b = 0; b < ctx->n_bins; b++) all_local &= ctx->bin_owner[b] == ctx->rank;
     // auto: tile::gather4 for a replicated table whose row fits one box (<= 256 words), TMA bulk copies for
     // other local rows, LDG.128 for routed / remote rows
-    const bool tma4_ok = route == nullptr && ctx->n_bins == 1 && !ctx->placement && all_local && ctx->row_bytes / 4 <= 256;
+    // (a placement map with one local bin, e.g. DDAK on one GPU: the coordinate is the slot, < 2^31 rows)
+    const bool tma4_ok = route == nullptr && ctx->n_bins == 1 && all_local && ctx->row_bytes / 4 <= 256 &&
+                         ctx->n_vertices < (int64_t(1) << 31);
     const bool tma4 = tma4_ok && (ctx->gather_path == 3 || ctx->gather_path == 0);
     const bool bulk = ctx->gather_path == 2 || (ctx->gather_path == 0 && route == nullptr && all_local);
     if (tma4) {
@@ -564,7 +581,7 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
         const int64_t tiles = (max_n + kTma4Rows - 1) / kTma4Rows;
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)device_sms() * bps));
         gather_tma4_kernel<4><<<grid, 32, smem, stream>>>(ctx->tma_map, ids, n_dev, max_n, (uint32_t)ctx->row_bytes,
-                                                          ctx->l2_load_policy, ctx->l2_store_policy,
+                                                          ctx->l2_load_policy, ctx->l2_store_policy, ctx->placement,
                                                           reinterpret_cast<char*>(out));
         return cuda_check(cudaGetLastError(), "moment_gather: tma4 launch");
     }

@@ -203,6 +203,32 @@ def test_gather_replicated(orc, dim, dtype, path, monkeypatch):
         assert np.array_equal(o2[: count // 2], want[: count // 2]) and not o2[count // 2:].any()
 
 
+@pytest.mark.parametrize("path", ["auto", "ldg", "bulk", "tma4"])
+@pytest.mark.parametrize("dim,dtype", [(100, torch.float32), (128, torch.float32), (768, torch.float16)])
+def test_gather_one_local_bin_with_placement(orc, dim, dtype, path, monkeypatch):
+    """One local bin addressed through a placement map (a DDAK layout on one GPU: row v at a permuted
+    slot): tile::gather4 takes the slot as its row coordinate, the bulk gather resolves the placement one
+    tile ahead; every path byte-exact with the oracle's table[ids]."""
+    _need_gpu()
+    monkeypatch.setenv("MOMENT_GATHER_PATH", path)
+    n = 7000
+    table = W.feature_table(n, dim, dtype, device="cpu")
+    R = table.shape[1]
+    rng = np.random.default_rng(dim + 1)
+    slot_of = rng.permutation(n).astype(np.int64)
+    bin_tab = torch.zeros((n, R), dtype=torch.uint8)
+    bin_tab[torch.as_tensor(slot_of)] = table
+    bin_tab = bin_tab.to(DEV)
+    placement = torch.as_tensor(M.place_pack(np.zeros(n, np.int32), slot_of).view(np.int64), device=DEV)
+    ctx = M.Ctx(n_vertices=n, max_seeds=1, max_fanout=[1], device=0, row_bytes=R, bin_owner=[0],
+                bin_ptr=[bin_tab.data_ptr()], placement=placement)
+    for count in [1, 33, 4099, 50001]:
+        ids = torch.as_tensor(rng.integers(0, n, count), device=DEV)
+        out = torch.empty((count, R), dtype=torch.uint8, device=DEV)
+        ctx.gather(ids, out)
+        assert np.array_equal(out.cpu().numpy(), orc.gather(table.numpy(), ids.cpu().numpy()))
+
+
 def build_tiered(table, bin_of, slot_of, owners, host_bins, device=DEV):
     """Materialise bins from a placement: HBM bins as device buffers, host bins as pinned host memory."""
     R = table.shape[1]

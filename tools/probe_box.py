@@ -57,22 +57,14 @@ def numa_nodes():
 
 def gpu_numa(i):
     """NUMA node of GPU i's PCIe function (sysfs), 0 if unknown."""
-    try:
-        bus = torch.cuda.get_device_properties(i).pci_bus_id if hasattr(torch.cuda.get_device_properties(i), "pci_bus_id") else None
-    except Exception:  # noqa: BLE001
-        bus = None
-    if bus is None:
-        out = sh(f"nvidia-smi -i {i} --query-gpu=pci.bus_id --format=csv,noheader").strip()
-        bus = out or None
-    if bus:
-        bus = bus.lower()
+    bus = sh(f"nvidia-smi -i {i} --query-gpu=pci.bus_id --format=csv,noheader").strip().lower()
+    if bus and not bus.startswith("err"):
         if bus.count(":") == 2 and len(bus.split(":")[0]) == 8:
             bus = bus[4:]
         try:
             with open(f"/sys/bus/pci/devices/{bus}/numa_node") as f:
-                v = int(f.read().strip())
-                return max(v, 0)
-        except OSError:
+                return max(int(f.read().strip()), 0)
+        except (OSError, ValueError):
             pass
     return 0
 
