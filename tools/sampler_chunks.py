@@ -1,6 +1,6 @@
 """How many 64-byte DRAM atoms the C2 sampler must touch per batch (CPU, oracle-driven analysis).
 
-For the first 8 batches of C2: per hop, the frontier size, how many nodes take all their neighbours
+For the first 8 batches of C2 (or --config): per hop, the frontier size, how many nodes take all their neighbours
 (d <= k: one contiguous run) or draw Floyd positions (d > k), and the number of distinct 64-byte chunks of
 `indices` those reads touch (Floyd positions simulated uniformly, the chunk count does not depend on which
 k-subset it is); plus how much of the node visits a hub cache of the hottest adjacency lists would cover.
@@ -19,8 +19,14 @@ import workloads as W  # noqa: E402
 
 
 def main():
+    import argparse
+
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--batches", type=int, default=8)
+    a = ap.parse_args()
     oracle.build()
-    cfg = W.CONFIGS["C2"]
+    cfg = W.CONFIGS[a.config]
     t = time.time()
     g = W.rmat_csr(cfg["n"], cfg["m"])
     print("graph built in %.1f s" % (time.time() - t))
@@ -30,7 +36,7 @@ def main():
     rng = np.random.default_rng(0)
     fan = list(cfg["fanout"])
     tot, freq = {}, np.zeros(g.n, np.int64)
-    nb = 8
+    nb = a.batches
     for b in range(nb):
         r = oracle.sample(ip, ix, bs[b].numpy(), fan, W.batch_rng_seed(1, 0, 0, b))
         c = r["counts"]

@@ -53,16 +53,18 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--lanes", type=int, default=16)
     ap.add_argument("--batches", type=int, default=4000)
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--atoms", type=float, default=ATOMS_PER_BATCH, help="random atoms per batch of the config")
     a = ap.parse_args()
-    st = bench.build_state("C2", "cuda:0", 0, 1, a.lanes)
+    st = bench.build_state(a.config, "cuda:0", 0, 1, a.lanes)
     us_s = timed(st, a.batches, False)
     us_f = timed(st, a.batches, True)
-    floor = ATOMS_PER_BATCH / ATOM_RATE * 1e6
-    print(json.dumps({"config": "C2", "lanes": a.lanes, "sampling_only_us_per_batch": us_s,
-                      "full_step_us_per_batch": us_f, "random_atoms_per_batch": ATOMS_PER_BATCH,
+    floor = a.atoms / ATOM_RATE * 1e6
+    print(json.dumps({"config": a.config, "lanes": a.lanes, "sampling_only_us_per_batch": us_s,
+                      "full_step_us_per_batch": us_f, "random_atoms_per_batch": a.atoms,
                       "atom_rate_roofline_G_per_s": ATOM_RATE / 1e9,
                       "sampling_atom_floor_us": floor, "sampling_frac_of_atom_roofline": floor / us_s,
-                      "achieved_G_atoms_per_s": ATOMS_PER_BATCH / us_s / 1e3}))
+                      "achieved_G_atoms_per_s": a.atoms / us_s / 1e3}))
 
 
 if __name__ == "__main__":
