@@ -230,7 +230,7 @@ __global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const ui
 // own bulk copy (per-lane bulk groups). Rows past the end of a tile repeat the tile's first row and are
 // not stored.
 constexpr int kTma4Rows = 32;  // rows per tile = 8 groups of 4
-template <int kStages>
+template <int kStages, bool kPlacement>
 __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__ CUtensorMap tmap,
                                                          const int64_t* __restrict__ ids, const int64_t* n_dev,
                                                          int64_t max_n, uint32_t R, int l2_load, int l2_store,
@@ -253,11 +253,13 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
         const int64_t r = (t0 + s * dt) * kTma4Rows + lane;
         pid[s] = r < max_n ? __ldg(ids + r) : -1;
     }
-    // with a placement map (one local bin, e.g. a DDAK layout on one GPU) the row coordinate is the slot
+    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+    // kPlacement (one local bin behind a placement map, e.g. a DDAK layout on one GPU): the row coordinate is
+    // the slot, one more dependent load after the id (its own instantiation: the replicated path keeps the
+    // count load in flight together with the first ids)
 #pragma unroll
     for (int s = 0; s < kStages; s++)
-        pre[s] = pid[s] < 0 ? -1 : placement ? (int32_t)(dev::ld_rand(placement + pid[s]) & kSlotMask) : (int32_t)pid[s];
-    const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
+        pre[s] = kPlacement ? (pid[s] < 0 ? -1 : (int32_t)(dev::ld_rand(placement + pid[s]) & kSlotMask)) : (int32_t)pid[s];
     const int64_t n_tiles = (n + kTma4Rows - 1) / kTma4Rows;
     if (lane == 0)
         for (int s = 0; s < kStages; s++) mbar_init(&full[s], 1);
@@ -267,7 +269,7 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
         const int64_t r = tile * kTma4Rows + lane;
         if (!(tile < n_tiles && r < n)) return -1;
         const int64_t id = __ldg(ids + r);
-        return placement ? (int32_t)(dev::ld_rand(placement + id) & kSlotMask) : (int32_t)id;
+        return kPlacement ? (int32_t)(dev::ld_rand(placement + id) & kSlotMask) : (int32_t)id;
     };
     auto issue = [&](int64_t tile, int s, int32_t id) {
         const int rows = (int)min((int64_t)kTma4Rows, n - tile * kTma4Rows);
@@ -580,9 +582,15 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
         const size_t smem = (size_t)stages * 8 * G;
         const int64_t tiles = (max_n + kTma4Rows - 1) / kTma4Rows;
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)device_sms() * bps));
-        gather_tma4_kernel<4><<<grid, 32, smem, stream>>>(ctx->tma_map, ids, n_dev, max_n, (uint32_t)ctx->row_bytes,
-                                                          ctx->l2_load_policy, ctx->l2_store_policy, ctx->placement,
-                                                          reinterpret_cast<char*>(out));
+        if (ctx->placement)
+            gather_tma4_kernel<4, true><<<grid, 32, smem, stream>>>(ctx->tma_map, ids, n_dev, max_n, (uint32_t)ctx->row_bytes,
+                                                                    ctx->l2_load_policy, ctx->l2_store_policy,
+                                                                    ctx->placement, reinterpret_cast<char*>(out));
+        else
+            gather_tma4_kernel<4, false><<<grid, 32, smem, stream>>>(ctx->tma_map, ids, n_dev, max_n,
+                                                                     (uint32_t)ctx->row_bytes, ctx->l2_load_policy,
+                                                                     ctx->l2_store_policy, nullptr,
+                                                                     reinterpret_cast<char*>(out));
         return cuda_check(cudaGetLastError(), "moment_gather: tma4 launch");
     }
     if (bulk && route == nullptr) {
@@ -896,7 +904,7 @@ moment_status configure_gather_kernels(int carveout) {
                                   "carveout attribute"));
     for (const void* f : {(const void*)gather_bulk_kernel<2>, (const void*)gather_bulk_kernel<4>,
                           (const void*)gather_bulk_kernel<6>, (const void*)gather_bulk_kernel<8>,
-                          (const void*)gather_tma4_kernel<4>})
+                          (const void*)gather_tma4_kernel<4, false>, (const void*)gather_tma4_kernel<4, true>})
         MOMENT_TRY(cuda_check(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmemMax),
                               "bulk gather smem attribute"));
     return MOMENT_OK;
