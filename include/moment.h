@@ -264,7 +264,7 @@ typedef struct {
     const int64_t* indptr;  /* device [n_vertices + 1] */
     const int32_t* indices; /* device [n_edges] */
     int64_t n_vertices;
-    int64_t n_edges;
+    int64_t n_edges;        /* = indptr[n_vertices] (the caller's contract; 0 <= n_edges < 2^40 checked) */
 } moment_csr;
 
 #define MOMENT_SAMPLE_REPLACE 1u  /* sample with replacement (k draws whenever deg > 0) */

@@ -902,6 +902,10 @@ moment_status check_sample(const moment_ctx_s* ctx, const moment_csr* csr, const
     if (csr->n_vertices != ctx->n_vertices || !csr->indptr || !csr->indices)
         return fail(MOMENT_EINVAL, "moment_sample: csr has %lld vertices, ctx was created for %lld",
                     (long long)csr->n_vertices, (long long)ctx->n_vertices);
+    // n_edges picks the launch variant (the bitscan's neighbour prefetch) and must describe `indices`;
+    // indptr[n] == n_edges is the caller's contract (checking it would need a device read)
+    if (csr->n_edges < 0 || csr->n_edges >= (int64_t(1) << 40))
+        return fail(MOMENT_EINVAL, "moment_sample: n_edges %lld out of range", (long long)csr->n_edges);
     const int H = p->n_hops;
     if (H < 0 || H > ctx->max_hops || H > kMaxHops)
         return fail(MOMENT_EINVAL, "moment_sample: n_hops %d > max_hops %d", H, ctx->max_hops);
