@@ -257,9 +257,11 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
     // kPlacement (one local bin behind a placement map, e.g. a DDAK layout on one GPU): the row coordinate is
     // the slot, one more dependent load after the id (its own instantiation: the replicated path keeps the
     // count load in flight together with the first ids)
+    // (ids past the count are stale buffer contents: never looked up)
 #pragma unroll
     for (int s = 0; s < kStages; s++)
-        pre[s] = kPlacement ? (pid[s] < 0 ? -1 : (int32_t)(dev::ld_rand(placement + pid[s]) & kSlotMask)) : (int32_t)pid[s];
+        pre[s] = !kPlacement ? (int32_t)pid[s]
+                 : ((t0 + s * dt) * kTma4Rows + lane < n ? (int32_t)(dev::ld_rand(placement + pid[s]) & kSlotMask) : -1);
     const int64_t n_tiles = (n + kTma4Rows - 1) / kTma4Rows;
     if (lane == 0)
         for (int s = 0; s < kStages; s++) mbar_init(&full[s], 1);

@@ -88,3 +88,25 @@ def test_bench_partitioned_two_ranks_shared_gpu(placement):
     assert sum(t["bin_rows"]) == (1 << 16) - t["replicated_rows"]  # a partition of the non-replicated rows
     if placement == "ddak-rep":
         assert t["replicated_rows"] > 0
+
+
+@pytest.mark.gpu
+def test_bench_replicated_two_ranks_self_launched():
+    """`bench.py --gpus 2` outside torchrun re-launches itself under torch.distributed.run (here both ranks on
+    cuda:0 over gloo, MOMENT_BENCH_SHARED_GPU): one JSON line, n_gpus = 2, global batch 2 x 1024."""
+    line = _run(["--gpus", "2", "--config", "C1", "--steps", "10", "--warmup", "3", "--min-time", "0.1",
+                 "--e2e-min-time", "0.05"], env={"MOMENT_BENCH_SHARED_GPU": "1"})
+    assert line["n_gpus"] == 2 and line["config"]["global_batch"] == 2048 and "test_mode" in line["config"]
+    assert line["cpu_baseline"] is None  # rank 0 at N = 1 only
+
+
+def test_bench_refuses_more_ranks_than_gpus():
+    import torch
+
+    if torch.cuda.is_available() and torch.cuda.device_count() >= 2:
+        pytest.skip("box has 2+ GPUs")
+    e = dict(os.environ, WORLD_SIZE="2", RANK="0", LOCAL_RANK="0")
+    e.pop("MOMENT_BENCH_SHARED_GPU", None)
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--config", "C1"],
+                       capture_output=True, text=True, timeout=300, cwd=ROOT, env=e)
+    assert r.returncode != 0 and "visible GPUs" in (r.stderr + r.stdout)

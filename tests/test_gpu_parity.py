@@ -226,7 +226,16 @@ def test_gather_one_local_bin_with_placement(orc, dim, dtype, path, monkeypatch)
         ids = torch.as_tensor(rng.integers(0, n, count), device=DEV)
         out = torch.empty((count, R), dtype=torch.uint8, device=DEV)
         ctx.gather(ids, out)
-        assert np.array_equal(out.cpu().numpy(), orc.gather(table.numpy(), ids.cpu().numpy()))
+        want = orc.gather(table.numpy(), ids.cpu().numpy())
+        assert np.array_equal(out.cpu().numpy(), want)
+        # a device count below the buffer size, the buffer's tail holding stale, out-of-range ids (as F_H's
+        # buffer does past |F_H|): only the first n_dev rows are read and written
+        stale = ids.clone()
+        stale[count // 2:] = (1 << 40) + 12345
+        out2 = torch.zeros_like(out)
+        ctx.gather(stale, out2, n_dev=torch.tensor([count // 2], dtype=torch.int64, device=DEV))
+        o2 = out2.cpu().numpy()
+        assert np.array_equal(o2[: count // 2], want[: count // 2]) and not o2[count // 2:].any()
 
 
 def build_tiered(table, bin_of, slot_of, owners, host_bins, device=DEV):
