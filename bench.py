@@ -129,7 +129,7 @@ class PartState(State):
     peer rows are NVLink loads inside the gather kernel (no exchange: there is no host tier to relay)."""
 
     def __init__(self, name, device, rank, world, inflight, *, dist, shared, placement="ddak", presample=64,
-                 replicate_frac=1 / 16):
+                 replicate_frac=1 / 16, layout=None):
         import paper_conf_sc_shi0s0x0w25_b200 as M
 
         self.M = M
@@ -181,6 +181,14 @@ class PartState(State):
                                                    replicate_rows=r, traffic_mode=M.TRAFFIC_STANDALONE,
                                                    return_replica_access=True)
         self.t_place = time.perf_counter() - t1
+        if layout:  # plan reuse: rank 0 saves the layout; a saved one must match what DDAK recomputed
+            if os.path.exists(layout):
+                saved = M.layout.load(layout, topo)
+                if not (np.array_equal(saved["bin_of"], bin_of) and np.array_equal(saved["slot_of"], slot_of)):
+                    raise SystemExit(f"{layout}: saved layout differs from this run's placement")
+            elif rank == 0:
+                M.layout.save(layout, topo, bin_of=bin_of, slot_of=slot_of, bin_node=bin_node,
+                              capacity_rows=[cap] * world, replicate_rows=r, note=f"{name} {placement} k={world}")
         # P5: the plan's predicted per-batch time for this layout (in-sample demand per GPU per batch)
         N = topo.info()[0]
         d = np.zeros(N, np.int64)
@@ -535,6 +543,7 @@ def main():
                          "same with the hottest --replicate-frac of the rows in every GPU (R25)")
     ap.add_argument("--presample", type=int, default=64, help="pre-sample batches per rank for DDAK hotness (P2)")
     ap.add_argument("--replicate-frac", type=float, default=1 / 16)
+    ap.add_argument("--layout", default=None, help="partitioned: save the DDAK layout here (rank 0), or check a saved one")
     args = ap.parse_args()
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         spawn_ranks(args.gpus)
@@ -566,7 +575,7 @@ def main():
     P = max(1, min(args.inflight, args.steps))
     part = args.placement != "replicated"
     kw = dict(placement=args.placement, dist=dist, shared=shared, presample=args.presample,
-              replicate_frac=args.replicate_frac) if part else {}
+              replicate_frac=args.replicate_frac, layout=args.layout) if part else {}
     st = build_state(args.config, dev, rank, world, P, **kw)
     H = len(st.fanout)
     K = args.steps

@@ -6,3 +6,4 @@ The Python layer is argument marshalling only (`moment.py`); see DESIGN.md.
 from . import moment  # noqa: F401
 from .moment import *  # noqa: F401,F403
 from . import boxes  # noqa: F401,E402
+from . import layout  # noqa: F401,E402
