@@ -171,11 +171,13 @@ def test_peer_exchange_device_barrier_two_processes_one_gpu():
     assert all(r["ok"] for r in res), res
 
 
-def test_one_call_exchange_two_processes_one_gpu():
+@pytest.mark.parametrize("world", [2, 3])
+def test_one_call_exchange_processes_one_gpu(world):
     """moment_ctx_set_exchange: the whole relay exchange inside ONE moment_gather / moment_step call per batch
     (bucket, own reads, peer-store requests, device barrier, peer-store rows, device barrier), replayed from
-    the ctx's CUDA graph with no host barrier between batches; byte-exact with the oracle."""
+    the ctx's CUDA graph with no host barrier between batches; byte-exact with the oracle (2 and 3 processes
+    sharing cuda:0, every rank relaying for the others)."""
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
-    res = run_world(_rank_main, 2, "one_call")
+    res = run_world(_rank_main, world, "one_call")
     assert all(r["ok"] for r in res), res

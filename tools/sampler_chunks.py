@@ -24,11 +24,13 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", default="C2")
     ap.add_argument("--batches", type=int, default=8)
+    ap.add_argument("--device", default="cpu", help="where to generate the graph (cuda: fast, then copied to host)")
     a = ap.parse_args()
     oracle.build()
     cfg = W.CONFIGS[a.config]
     t = time.time()
-    g = W.rmat_csr(cfg["n"], cfg["m"])
+    g = W.rmat_csr(cfg["n"], cfg["m"], device=a.device)
+    g = W.Graph(g.indptr.cpu(), g.indices.cpu(), g.n, g.m)
     print("graph built in %.1f s" % (time.time() - t))
     ip, ix = g.indptr.numpy(), g.indices.numpy()
     deg = np.diff(ip)
