@@ -674,6 +674,23 @@ def main():
             L0.ctx.step(st.graph.indptr, st.graph.indices, pool[i][0], st.fanout, pool[i][1], L0.bufs, None,
                         stream=main_stream)
             per_bin += st.bins_of(L0.bufs.nodes, nF_pool[i]) * used.count(i)
+        # every rank: every row of one of its batches, gathered through the local and the peers' (CUDA-IPC
+        # mapped) bins, equals the generated bytes of its id (the oracle's table[ids]; the sampler is per rank
+        # and checked by the N = 1 parity subset)
+        i0 = used[0]
+        L0.ctx.step(st.graph.indptr, st.graph.indices, pool[i0][0], st.fanout, pool[i0][1], L0.bufs, L0.rows,
+                    stream=main_stream)
+        torch.cuda.synchronize()
+        nf0 = nF_pool[i0]
+        rows_ok = True
+        for c0 in range(0, nf0, 1 << 18):
+            c1 = min(nf0, c0 + (1 << 18))
+            rows_ok &= bool(torch.equal(L0.rows[c0:c1], W.feature_rows(L0.bufs.nodes[c0:c1], st.dim, st.dtype)))
+        okt = torch.tensor([int(rows_ok)], dtype=torch.int64, device=dev if not shared else "cpu")
+        if dist:
+            dist.all_reduce(okt, op=dist.ReduceOp.MIN)
+        if not int(okt):
+            raise AssertionError("partitioned gather: rows differ from their generated bytes on some rank")
         allb = [torch.zeros_like(per_bin) for _ in range(world)]
         if dist:
             if shared:
@@ -703,7 +720,8 @@ def main():
                  "plan": {"t_star_us": st.plan["t_star"], "t_nvlink_us": st.plan["t_nvlink"],
                           "t_hbm_us": st.plan["t_hbm"],
                           "note": "the plan predicts the gather per batch (P:L229-235, P:L339)"},
-                 "offline_s": {"hotness": st.t_hotness, "ddak": st.t_place}}
+                 "offline_s": {"hotness": st.t_hotness, "ddak": st.t_place},
+                 "rows_check": {"ranks": world, "rows_per_rank": "every row of one batch", "byte_exact": True}}
     # roofline pass: CUDA events around the dominant kernel (the gather) on its stream, one lane, one batch
     # at a time, over the pool
     n_roof = min(n_pool, 256)
