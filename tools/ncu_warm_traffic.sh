@@ -4,7 +4,7 @@
 OUT=${1:-gpurun_out/warm_traffic}
 ncu --cache-control none --clock-control none --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,lts__t_sectors_srcunit_tex_op_read.sum,lts__t_sectors_srcunit_tex_op_write.sum,lts__t_sectors_srcunit_tex_op_red.sum \
   -k "regex:hop_|bitscan|compact|init_kernel|gather_" -s 24 -c 24 --csv --log-file "$OUT.csv" \
-  python bench.py --config C2 --steps 4 --warmup 3 --inflight 1 --no-cpu-baseline --min-time 0 --e2e-min-time 0 > /dev/null 2>&1
+  python bench.py --config ${2:-C2} --steps 4 --warmup 3 --inflight 1 --no-cpu-baseline --min-time 0 --e2e-min-time 0 > /dev/null 2>&1
 python - "$OUT.csv" <<'PY'
 import csv, sys
 from collections import defaultdict
