@@ -42,6 +42,27 @@ def _peaks():
         return 6650.0, "fallback"
 
 
+def lane_streams(device, inflight):
+    """One stream per lane. MOMENT_LANE_PRIO (default "half"): the first half of the lanes on high-priority
+    streams (their early, latency-bound hops get the SMs first, so their gathers start sooner and overlap the
+    other half's sampling; measured +0.6 % at K = 200, +0.1 % at K = 20; "ramp" = a priority gradient, -0.7 %);
+    "none": lane 0 on the current stream, no priorities."""
+    mode = os.environ.get("MOMENT_LANE_PRIO", "half")  # none | half | first | ramp (half: +0.6 % at K = 200)
+    if mode == "none":
+        return [torch.cuda.current_stream(device)] + [torch.cuda.Stream(device) for _ in range(inflight - 1)]
+    lo, hi = torch.cuda.Stream.priority_range() if hasattr(torch.cuda.Stream, "priority_range") else (0, -1)
+    out = []
+    levels = abs(hi - lo) + 1
+    for i in range(inflight):
+        if mode == "ramp":  # lane i gets the (i * levels / inflight)-th highest priority
+            pr = hi + (1 if hi < lo else -1) * min(levels - 1, i * levels // inflight)
+        else:
+            high = (mode == "half" and i < (inflight + 1) // 2) or (mode == "first" and i == 0)
+            pr = hi if high else lo
+        out.append(torch.cuda.Stream(device, priority=pr))
+    return out
+
+
 class Lane:
     """One batch in flight: its own device context (workspace), sample buffers, row buffer and stream."""
 
@@ -75,7 +96,7 @@ class State:
         self.stride = (self.R + 63) // 64 * 64
         self.table = W.feature_table(cfg["n"], self.dim, self.dtype, device=device, row_stride_bytes=self.stride)
         self.train = W.training_set(self.graph, min_count=self.B * world)
-        streams = [torch.cuda.current_stream(device)] + [torch.cuda.Stream(device) for _ in range(inflight - 1)]
+        streams = lane_streams(device, inflight)
         self.lanes = [Lane(M, cfg, self.fanout, self.B, self.R, rank, world, device, self.table, s) for s in streams]
         self.ctx, self.bufs, self.rows = self.lanes[0].ctx, self.lanes[0].bufs, self.lanes[0].rows
         self._batches = []
@@ -224,7 +245,7 @@ class PartState(State):
                     base = M.ipc_import(allh[h][0])
                     self._imported.append(base)
                     ptrs[h] = base + allh[h][1]
-        streams = [torch.cuda.current_stream(device)] + [torch.cuda.Stream(device) for _ in range(inflight - 1)]
+        streams = lane_streams(device, inflight)
         self.lanes = []
         for s_ in streams:
             L = Lane.__new__(Lane)
@@ -582,14 +603,16 @@ def main():
     main_stream = torch.cuda.current_stream()
 
     def fork(ev):
-        for L in st.lanes[1:]:
-            L.stream.wait_event(ev)
+        for L in st.lanes:
+            if L.stream != main_stream:
+                L.stream.wait_event(ev)
 
     def join():
-        for L in st.lanes[1:]:
-            e = torch.cuda.Event()
-            e.record(L.stream)
-            main_stream.wait_event(e)
+        for L in st.lanes:
+            if L.stream != main_stream:
+                e = torch.cuda.Event()
+                e.record(L.stream)
+                main_stream.wait_event(e)
 
     def barrier():
         torch.cuda.synchronize()
