@@ -686,7 +686,9 @@ __device__ __forceinline__ void block_sum2(int64_t& x, int64_t& y, int64_t (*red
 // All hops' offsets and src in one wait-free pass: a tile's first edge position is the sum of the edge
 // counts of the tiles before it, which the hop kernels accumulated per tile (no chained scan, no waiting
 // on other blocks); the hop's base is the sum over the earlier hops' tiles.
-__global__ void __launch_bounds__(kSampleTile, MOMENT_SAMPLE_MIN_BLOCKS) compact_kernel(CompactArgs a) {
+// 4 blocks/SM minimum (<= 64 registers): its grid is capped at 2 blocks/SM, and the samplers' 40-register cap
+// made it spill (48 B); measured +1.3 % bench at K = 20, +0.5 % per step at 16 lanes (tools/ab_lib.sh)
+__global__ void __launch_bounds__(kSampleTile, 4) compact_kernel(CompactArgs a) {
     constexpr int kCopyUnroll = 8;  // padded slots per thread in flight (id load -> lidx load -> src store)
     __shared__ int64_t s_red[kSampleTile / 32];
     __shared__ int64_t s_red2[kSampleTile / 32][2];
