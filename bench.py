@@ -870,10 +870,12 @@ def main():
                     "d2h_bytes_per_step": (2 * H + 1) * 8,
                     "api": "moment_step_host (C ABI) per step, same K-step regions, median of "
                            f"{len(e2e_ms_all)}",
-                    "copies_declared": "H2D: the step's 1024 int64 seeds from pinned host memory; D2H: the "
-                                       "step's counts (|F_0..F_H|, E_0..E_{H-1}) into pinned memory. F_H, offsets, "
-                                       "src and the gathered rows stay in HBM for the on-GPU consumer (the GNN "
-                                       "layer, sage.py) and are not copied to the host"},
+                    "copies_declared": "H2D: the step's 1024 int64 seeds, read from pinned host memory over PCIe "
+                                       "by the first hop's kernel (zero-copy); D2H: the step's counts (|F_0..F_H|, "
+                                       "E_0..E_{H-1}) stored into pinned host memory by the compaction's last block "
+                                       "(pageable buffers would go through cudaMemcpyAsync). F_H, offsets, src and "
+                                       "the gathered rows stay in HBM for the on-GPU consumer (the GNN layer, "
+                                       "sage.py) and are not copied to the host"},
             "gpu_launches": st.launches_per_step() * K,
             "clocks": ck,
         }

@@ -462,11 +462,13 @@ moment_status moment_step(moment_ctx_t ctx, const moment_csr* csr, const int64_t
                           void* stream);
 
 /* ================================================================================================
- * End-to-end step with HOST buffers (the e2e leg of the benchmark): copies seeds host->device, samples,
- * gathers F_H into d_rows (NULL: sample only), copies the 2H+1 counts device->host into counts_host. All of
- * it is enqueued on `stream`; counts_host is valid once the stream has reached the copy (synchronise the
- * stream or an event). seeds_host / counts_host should be pinned; seeds_host must stay unchanged until the
- * H2D copy has executed. Several steps may be in flight on different ctxs / streams.
+ * End-to-end step with HOST buffers (the e2e leg of the benchmark): moves the seeds host->device, samples,
+ * gathers F_H into d_rows (NULL: sample only), moves the 2H+1 counts device->host into counts_host. All of
+ * it is enqueued on `stream`; counts_host is valid once the stream has completed the step (synchronise the
+ * stream or an event). Pinned (page-locked, device-mapped) buffers cross PCIe inside the step's kernels: the
+ * first hop reads the seeds from host memory, the compaction's last block stores the counts (no copy-engine
+ * operation); pageable buffers go through cudaMemcpyAsync. seeds_host must stay unchanged until the step's
+ * first kernel has run. Several steps may be in flight on different ctxs / streams.
  * ================================================================================================ */
 moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds_host,
                                int64_t n_seeds, const moment_sample_params* params,

@@ -246,7 +246,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
         o_owner = cv.take<int32_t>(a->n_bins);
     }
     const int64_t o_seed = cv.take<int64_t>(a->max_seeds);
-    const int64_t o_call = cv.take<uint64_t>(2);
+    const int64_t o_call = cv.take<uint64_t>(3);
     c->ws_bytes = cv.off;
     cudaError_t e = cudaMalloc(&c->ws, c->ws_bytes);
     if (e != cudaSuccess) {
@@ -387,11 +387,12 @@ extern "C" moment_status moment_ctx_workspace_bytes(moment_ctx_t ctx, int64_t* b
 
 namespace {
 
-__global__ void set_call_kernel(uint64_t* call, uint64_t rng_seed, const int64_t* seeds, unsigned long long* zero,
-                                int64_t n_zero) {
+__global__ void set_call_kernel(uint64_t* call, uint64_t rng_seed, const int64_t* seeds, int64_t* counts_host,
+                                unsigned long long* zero, int64_t n_zero) {
     if (threadIdx.x == 0) {
         call[0] = rng_seed;
         call[1] = reinterpret_cast<uint64_t>(seeds);
+        call[2] = reinterpret_cast<uint64_t>(counts_host);  // mapped host counts (moment_step_host) or 0
     }
     for (int64_t j = threadIdx.x; j < n_zero; j += blockDim.x) zero[j] = 0;  // hop 0's compaction tile sums
 }
@@ -400,8 +401,9 @@ __global__ void set_call_kernel(uint64_t* call, uint64_t rng_seed, const int64_t
 // kernel whose parameters carry the values: ordered before the call's kernels on `s`, and safe inside a
 // caller's stream capture (the values are baked into the captured node). It also zeroes the first hop's
 // compaction tile sums (the later hops' are zeroed by the scan before them).
-moment_status write_call(moment_ctx_s* c, uint64_t rng_seed, const int64_t* seeds, int64_t n_seeds, cudaStream_t s) {
-    set_call_kernel<<<1, 32, 0, s>>>(c->d_call, rng_seed, seeds, c->tile_edges,
+moment_status write_call(moment_ctx_s* c, uint64_t rng_seed, const int64_t* seeds, int64_t n_seeds, cudaStream_t s,
+                         int64_t* counts_host = nullptr) {
+    set_call_kernel<<<1, 32, 0, s>>>(c->d_call, rng_seed, seeds, counts_host, c->tile_edges,
                                      std::min<int64_t>((n_seeds + kSampleTile - 1) / kSampleTile, c->n_tile_edges));
     return cuda_check(cudaGetLastError(), "call block");
 }
@@ -465,6 +467,18 @@ moment_status run_step(moment_ctx_s* c, const moment_csr* csr, int64_t n_seeds, 
         c->step_key.rows = rows;
     }
     return cuda_check(cudaGraphLaunch(c->step_exec, s), "moment_step: graph launch");
+}
+
+// The device address of a pinned, mapped host buffer (cudaHostAlloc / registered memory; the same address under
+// unified addressing), or null for pageable memory.
+template <typename T>
+T* mapped_host_ptr(T* p) {
+    cudaPointerAttributes a{};
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();  // pageable memory on old drivers reports an error: clear it
+        return nullptr;
+    }
+    return a.type == cudaMemoryTypeHost && a.devicePointer ? static_cast<T*>(a.devicePointer) : nullptr;
 }
 
 moment_status check_rows(const moment_ctx_s* c, void* rows, const moment_sample_out* out) {
@@ -572,9 +586,19 @@ extern "C" moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* cs
     MOMENT_TRY(check_sample(ctx, csr, ctx->d_seed_stage, n_seeds, params, out));
     MOMENT_TRY(check_rows(ctx, d_rows, out));
     cudaStream_t s = static_cast<cudaStream_t>(stream);
-    MOMENT_TRY(cuda_check(cudaMemcpyAsync(ctx->d_seed_stage, seeds_host, n_seeds * sizeof(int64_t), cudaMemcpyHostToDevice, s), "moment_step_host: H2D"));
-    MOMENT_TRY(write_call(ctx, params->rng_seed, ctx->d_seed_stage, n_seeds, s));
+    // pinned (page-locked, device-mapped) host buffers move over PCIe inside the step's own kernels: the first
+    // hop reads the seeds from host memory and the compaction's last block stores the counts there (no
+    // copy-engine operation on the step's critical path); pageable buffers go through cudaMemcpyAsync
+    const int64_t* seeds_dev = mapped_host_ptr(seeds_host);
+    int64_t* counts_dev = mapped_host_ptr(counts_host);
+    if (!seeds_dev) {
+        MOMENT_TRY(cuda_check(cudaMemcpyAsync(ctx->d_seed_stage, seeds_host, n_seeds * sizeof(int64_t),
+                                              cudaMemcpyHostToDevice, s), "moment_step_host: H2D"));
+        seeds_dev = ctx->d_seed_stage;
+    }
+    MOMENT_TRY(write_call(ctx, params->rng_seed, seeds_dev, n_seeds, s, counts_dev));
     MOMENT_TRY(run_step(ctx, csr, n_seeds, params, out, d_rows, s));
+    if (counts_dev) return MOMENT_OK;
     const int H = params->n_hops;
     return cuda_check(cudaMemcpyAsync(counts_host, out->counts, (2 * H + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s),
                       "moment_step_host: D2H");

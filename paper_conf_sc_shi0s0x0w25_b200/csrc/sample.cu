@@ -633,6 +633,8 @@ struct CompactArgs {
     const uint2* srel;   // sparse scan with rank relabelling: hop h's tables at srel + h * srel_stride and
     const uint2* trel[kMaxHops];  //   trel[h], else null
     int64_t srel_stride;
+    const uint64_t* call;  // the call block: [2] = mapped host counts of moment_step_host, or 0
+    uint32_t* done;        // blocks finished (zeroed per call with the tickets)
 };
 
 // Sparse scan's two-level tables: is v new at hop hh, and at which position?
@@ -808,6 +810,21 @@ __global__ void __launch_bounds__(kSampleTile, 4) compact_kernel(CompactArgs a) 
             }
         }
         __syncthreads();  // s_red / s_red2 / s_excl / s_cnt are reused by the next tile
+    }
+    // moment_step_host with mapped host counts: the last block to finish stores the call's 2H + 1 counts into
+    // host memory (every block's writes are visible to it: fence, then the done-counter ticket)
+    if (a.call && a.call[2]) {
+        __shared__ bool s_last;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            __threadfence();
+            s_last = atomicAdd(a.done, 1u) == gridDim.x - 1;
+        }
+        __syncthreads();
+        if (s_last && threadIdx.x < 2 * a.H + 1) {
+            __threadfence();
+            reinterpret_cast<volatile int64_t*>(a.call[2])[threadIdx.x] = *reinterpret_cast<volatile int64_t*>(a.counts + threadIdx.x);
+        }
     }
     const int64_t FH = a.counts[a.H];
     for (int64_t i = (int64_t)blockIdx.x * kSampleTile + threadIdx.x; i < FH; i += (int64_t)gridDim.x * kSampleTile)
@@ -1015,6 +1032,8 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
     ca.srel_stride = ctx->srel_stride;
     ca.tile_edges = ctx->tile_edges;
     ca.H = H;
+    ca.call = call;
+    ca.done = ctx->tickets;  // tickets[0]: compaction blocks done (zeroed by the call's init)
     const int grid = (int)std::max<int64_t>(
         1, std::min<int64_t>(std::max(ca.tb[H], (F_bound + 1023) / 1024), (int64_t)device_sms() * ctx->compact_grid_per_sm));
     compact_kernel<<<grid, kSampleTile, 0, stream>>>(ca);

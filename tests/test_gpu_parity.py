@@ -365,14 +365,25 @@ def test_step_host_matches_device_path(orc, c1):
     seeds = W.epoch_batches(train, 1024, 0)[0]
     bufs = M.SampleBuffers.allocate(1024, [10, 5], n, DEV)
     rows = torch.empty((bufs.nodes.numel(), R), dtype=torch.uint8, device=DEV)
-    counts_h = torch.zeros(5, dtype=torch.int64).pin_memory()
-    seeds_h = seeds.cpu().pin_memory()
-    ctx.step_host(g.indptr, g.indices, seeds_h, [10, 5], 77, bufs, rows, counts_h)
-    torch.cuda.synchronize()
-    want = orc.sample(g.indptr.cpu().numpy(), g.indices.cpu().numpy(), seeds_h.numpy(), [10, 5], 77)
-    assert np.array_equal(counts_h.numpy(), want["counts"])
+    want = orc.sample(g.indptr.cpu().numpy(), g.indices.cpu().numpy(), seeds.cpu().numpy(), [10, 5], 77)
     nF = int(want["counts"][2])
-    assert np.array_equal(rows[:nF].cpu().numpy(), orc.gather(table.cpu().numpy(), want["nodes"]))
+    # pinned buffers: the kernels read the seeds and write the counts over PCIe themselves; pageable ones go
+    # through cudaMemcpyAsync; several steps back to back reuse the graph with new host pointers
+    for pinned in (True, False, True):
+        counts_h = torch.full((5,), -1, dtype=torch.int64)
+        seeds_h = seeds.cpu().clone()
+        if pinned:
+            counts_h, seeds_h = counts_h.pin_memory(), seeds_h.pin_memory()
+        rows.zero_()
+        ctx.step_host(g.indptr, g.indices, seeds_h, [10, 5], 77, bufs, rows, counts_h)
+        torch.cuda.synchronize()
+        assert np.array_equal(counts_h.numpy(), want["counts"]), pinned
+        assert np.array_equal(rows[:nF].cpu().numpy(), orc.gather(table.cpu().numpy(), want["nodes"]))
+        # the device path after a host step: the call block's host-counts slot is cleared
+        bufs.counts.zero_()
+        ctx.step(g.indptr, g.indices, seeds, [10, 5], 77, bufs, rows)
+        torch.cuda.synchronize()
+        assert np.array_equal(bufs.counts.cpu().numpy(), want["counts"])
 
 
 def test_c2_full_size_bench_configuration(orc):
