@@ -110,3 +110,15 @@ def test_bench_refuses_more_ranks_than_gpus():
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--config", "C1"],
                        capture_output=True, text=True, timeout=300, cwd=ROOT, env=e)
     assert r.returncode != 0 and "visible GPUs" in (r.stderr + r.stdout)
+
+
+@pytest.mark.gpu
+def test_bench_partitioned_layout_reuse(tmp_path):
+    """--layout: the first run saves the DDAK layout (placement + topology hash), a second run checks that it
+    recomputes the identical placement (plan reuse)."""
+    lay = str(tmp_path / "c1.npz")
+    args = ["--config", "C1", "--placement", "ddak-rep", "--steps", "5", "--warmup", "3", "--min-time", "0.05",
+            "--e2e-min-time", "0.02", "--presample", "8", "--no-cpu-baseline", "--layout", lay]
+    _run(args)
+    assert os.path.exists(lay)
+    _run(args)
