@@ -137,6 +137,7 @@ class State:
 
 
 NVLINK_GBS = 770.0  # measured B200 peer copy per direction (B200_PROFILING.md; 900 GB/s nominal)
+PORT_GBS = 55.6     # measured pinned H2D copy of a pool B200 (profiles/r02_probe.json; Gen5 x16 raw 63.0)
 PRESAMPLE_EPOCH = 2**32 - 1  # R18: the pre-sample batches use their own rng stream
 
 
@@ -149,7 +150,7 @@ class PartState(State):
     peer rows are NVLink loads inside the gather kernel (no exchange: there is no host tier to relay)."""
 
     def __init__(self, name, device, rank, world, inflight, *, dist, shared, placement="ddak", presample=64,
-                 replicate_frac=1 / 16, layout=None):
+                 replicate_frac=1 / 16, layout=None, cache_gib=32.0):
         import paper_conf_sc_shi0s0x0w25_b200 as M
 
         self.M = M
@@ -160,7 +161,12 @@ class PartState(State):
         self.B = cfg["batch"]
         H = len(self.fanout)
         self.dim, self.dtype = cfg["dim"], cfg["dtype"]
-        self.graph = W.rmat_csr(cfg["n"], cfg["m"], device=device)
+        for turn in range(world if shared else 1):  # ranks sharing one GPU (test mode) build one at a time
+            if not shared or turn == rank:
+                self.graph = W.rmat_csr(cfg["n"], cfg["m"], device=device)
+                torch.cuda.empty_cache()
+            if shared and dist is not None:
+                dist.barrier()
         n = self.graph.n
         self.R = self.dim * torch.empty(0, dtype=self.dtype).element_size()
         self.stride = (self.R + 63) // 64 * 64
@@ -193,14 +199,26 @@ class PartState(State):
         hbm_gbs = _peaks()[0]
         box = M.boxes.hgx_b200(8, hbm_gbs=hbm_gbs, active=active)
         topo = box.topology()
-        bin_node = [box.hbm_bin[g] for g in active]
+        tiered = placement == "ddak-tiered"
+        bin_node = [box.hbm_bin[g] for g in active] + (box.host_bin if tiered else [])
         r = int(n * replicate_frac) if placement == "ddak-rep" and world > 1 else 0
-        cap = r + -(-(n - r) // world)
+        if tiered:  # a cache_gib HBM cache per GPU, the rest in one host-DRAM bin per socket (C4 / C5)
+            cap = min(n, int(cache_gib * (1 << 30)) // self.stride)
+            caps = [cap] * world + [n] * len(box.host_bin)
+        else:
+            cap = r + -(-(n - r) // world)
+            caps = [cap] * world
         t1 = time.perf_counter()
-        bin_of, slot_of, A, U, T, rep_acc = M.place(topo, hot_np, [cap] * world, bin_node=bin_node,
+        bin_of, slot_of, A, U, T, rep_acc = M.place(topo, hot_np, caps, bin_node=bin_node,
                                                    replicate_rows=r, traffic_mode=M.TRAFFIC_STANDALONE,
                                                    return_replica_access=True)
         self.t_place = time.perf_counter() - t1
+        # host bins hold a ring of r_phys rows (SURVEY 8(d) fallback: the C4 / C5 tables exceed the host), so every
+        # tier stores row(v) := feature(v mod r_phys) and a host row of v sits at slot v mod r_phys
+        self.r_phys = min(n, 1 << 22) if tiered else n
+        if tiered:
+            host = bin_of >= world
+            slot_of[host] = np.nonzero(host)[0] % self.r_phys
         if layout:  # plan reuse: rank 0 saves the layout; a saved one must match what DDAK recomputed
             if os.path.exists(layout):
                 saved = M.layout.load(layout, topo)
@@ -208,7 +226,7 @@ class PartState(State):
                     raise SystemExit(f"{layout}: saved layout differs from this run's placement")
             elif rank == 0:
                 M.layout.save(layout, topo, bin_of=bin_of, slot_of=slot_of, bin_node=bin_node,
-                              capacity_rows=[cap] * world, replicate_rows=r, note=f"{name} {placement} k={world}")
+                              capacity_rows=caps, replicate_rows=r, note=f"{name} {placement} k={world}")
         # P5: the plan's predicted per-batch time for this layout (in-sample demand per GPU per batch)
         N = topo.info()[0]
         d = np.zeros(N, np.int64)
@@ -218,6 +236,14 @@ class PartState(State):
                            replica_demand=int(rep_acc) * self.R // (presample * world)).info()
         self.placement_mode, self.replicated_rows = placement, r
         self.bin_rows = [int(x) for x in U]
+        self.n_bins = len(bin_node)
+        # quota x[j][h] of every host bin (the plan's path decomposition, rank order = active order): the share
+        # of this rank's bin-j rows read over GPU h's PCIe port and relayed to it (R11, R12)
+        quota = np.zeros((self.n_bins, world), np.int64)
+        for i, v in enumerate(bin_node):
+            if i >= world:
+                quota[i] = self.plan["quota"][v]
+        self.quota = quota
         # this rank's HBM bin: replicas at slots 0..r-1, then its partition
         mine = np.nonzero((bin_of == rank) | (bin_of == M.BIN_REPLICA))[0]
         rows_mine = r + int(U[rank])
@@ -226,8 +252,18 @@ class PartState(State):
         for c0 in range(0, len(mine), ch):
             ids = torch.as_tensor(mine[c0:c0 + ch], device=device)
             sl = torch.as_tensor(slot_of[mine[c0:c0 + ch]], device=device)
-            self.table[sl, :self.R] = W.feature_rows(ids, self.dim, self.dtype)
+            self.table[sl, :self.R] = W.feature_rows(ids % self.r_phys, self.dim, self.dtype)
         del mine
+        self.host_bins = []
+        if tiered:  # every rank pins its own copy of the host rings (each rank reads them over its own port)
+            for _ in box.host_bin:
+                h = torch.empty((self.r_phys, self.stride), dtype=torch.uint8).pin_memory()
+                for c0 in range(0, self.r_phys, ch):
+                    c1 = min(self.r_phys, c0 + ch)
+                    blk = torch.zeros((c1 - c0, self.stride), dtype=torch.uint8, device=device)
+                    blk[:, :self.R] = W.feature_rows(torch.arange(c0, c1, device=device), self.dim, self.dtype)
+                    h[c0:c1].copy_(blk)
+                self.host_bins.append(h)
         packed = M.place_pack_rank(bin_of, slot_of, rank) if r else M.place_pack(bin_of, slot_of)
         self.placement = torch.as_tensor(packed.view(np.int64), device=device)
         del packed, bin_of, slot_of
@@ -246,13 +282,25 @@ class PartState(State):
                     ptrs[h] = base + allh[h][1]
         streams = lane_streams(device, inflight)
         self.lanes = []
+        self.exchanges = []
+        owners = list(range(world)) + [-1] * len(self.host_bins)
+        ptrs = ptrs + [h.data_ptr() for h in self.host_bins]
         for s_ in streams:
             L = Lane.__new__(Lane)
             L.ctx = M.Ctx(n_vertices=n, max_seeds=self.B, max_fanout=self.fanout, rank=rank, world=world,
-                          device=dev_idx, row_bytes=self.R, row_stride=self.stride, bin_owner=list(range(world)),
-                          bin_ptr=ptrs, placement=self.placement)
+                          device=dev_idx, row_bytes=self.R, row_stride=self.stride, bin_owner=owners,
+                          bin_ptr=ptrs, placement=self.placement, quota=self.quota if tiered else None)
             L.bufs = M.SampleBuffers.allocate(self.B, self.fanout, n, device)
-            L.rows = torch.empty((L.bufs.nodes.numel(), self.R), dtype=torch.uint8, device=device)
+            if tiered and world > 1:
+                # relays through other ranks: this lane's batch is ONE collective moment_step (the relay exchange
+                # inside it; moment_ctx_set_exchange), into the exchange's registered output
+                from paper_conf_sc_shi0s0x0w25_b200.exchange import PeerExchange
+
+                px = PeerExchange(L.ctx, L.bufs.nodes.numel(), self.R, device, timeout_s=60.0)
+                self.exchanges.append(px)
+                L.rows = px.out
+            else:
+                L.rows = torch.empty((L.bufs.nodes.numel(), self.R), dtype=torch.uint8, device=device)
             L.stream = s_
             self.lanes.append(L)
         self.ctx, self.bufs, self.rows = self.lanes[0].ctx, self.lanes[0].bufs, self.lanes[0].rows
@@ -264,13 +312,33 @@ class PartState(State):
         b = torch.bitwise_right_shift(self.placement[nodes[:nF]], 40)
         return torch.bincount(b, minlength=self.world)
 
+    def queues_of(self, nodes, nF):
+        """Rows of a batch per route queue q = bin * world + via (moment_bucket: HBM bins via their owner, host
+        bins via the quota's relay rank), for the per-tier accounting after the timed region."""
+        M, dev = self.M, nodes.device
+        Q = self.n_bins * self.world
+        route = torch.empty(max(1, nF), dtype=torch.int32, device=dev)
+        qoff = torch.empty(Q + 1, dtype=torch.int64, device=dev)
+        qpos = torch.empty(max(1, nF), dtype=torch.int64, device=dev)
+        self.lanes[0].ctx.bucket(nodes, route, qoff, qpos, max_n=nF)
+        return qoff[1:] - qoff[:-1]
+
     def close(self, dist):
         torch.cuda.synchronize()
         if dist is not None:
             dist.barrier()
+        for px in self.exchanges:
+            px.close()
+        self.exchanges = []
         for base in self._imported:
             self.M.ipc_close(base)
         self._imported = []
+
+
+def feature_check_ids(st, nodes):
+    """Ids whose generated bytes a gathered row must equal (tiered layouts store feature(v mod r_phys))."""
+    r_phys = getattr(st, "r_phys", None)
+    return nodes % r_phys if r_phys else nodes
 
 
 def build_state(name, device="cuda:0", rank=0, world=1, inflight=1, **kw):
@@ -450,7 +518,7 @@ def partition_parity(st, pool):
             ok = (np.array_equal(got["counts"], r["counts"]) and np.array_equal(got["nodes"], r["nodes"])
                   and all(np.array_equal(got["offsets"][h], r["offsets"][h]) and
                           np.array_equal(got["src"][h], r["src"][h]) for h in range(H)))
-            ids = torch.as_tensor(r["nodes"], device=L.rows.device)
+            ids = feature_check_ids(st, torch.as_tensor(r["nodes"], device=L.rows.device))
             for c0 in range(0, nF, 1 << 18):
                 ok &= bool(torch.equal(L.rows[c0:min(nF, c0 + (1 << 18))],
                                        W.feature_rows(ids[c0:c0 + (1 << 18)], st.dim, st.dtype)))
@@ -557,10 +625,13 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=10.0, help="seconds of oracle time for cpu_baseline")
     # 12-16 measured best on C2 (29.5-29.7 M seeds/s vs 27.7 at 8, 28.4 at 24)
     ap.add_argument("--inflight", type=int, default=16, help="batches in flight per GPU (one stream each)")
-    ap.add_argument("--placement", default="replicated", choices=["replicated", "ddak", "ddak-rep"],
+    ap.add_argument("--placement", default="replicated", choices=["replicated", "ddak", "ddak-rep", "ddak-tiered"],
                     help="replicated: every GPU holds the whole table (C2 'all features in HBM'); ddak: the table "
                          "partitioned over the GPUs' HBM by DDAK (C3), peer rows read over NVLink; ddak-rep: the "
-                         "same with the hottest --replicate-frac of the rows in every GPU (R25)")
+                         "same with the hottest --replicate-frac of the rows in every GPU (R25); ddak-tiered: a "
+                         "--cache-gib HBM cache per GPU and one pinned host bin per socket (C4 / C5), host rows "
+                         "routed by the plan's quotas and relayed through peer ranks (one-call exchange)")
+    ap.add_argument("--cache-gib", type=float, default=32.0, help="ddak-tiered: HBM cache per GPU")
     ap.add_argument("--presample", type=int, default=64, help="pre-sample batches per rank for DDAK hotness (P2)")
     ap.add_argument("--replicate-frac", type=float, default=1 / 16)
     ap.add_argument("--layout", default=None, help="partitioned: save the DDAK layout here (rank 0), or check a saved one")
@@ -595,7 +666,7 @@ def main():
     P = max(1, min(args.inflight, args.steps))
     part = args.placement != "replicated"
     kw = dict(placement=args.placement, dist=dist, shared=shared, presample=args.presample,
-              replicate_frac=args.replicate_frac, layout=args.layout) if part else {}
+              replicate_frac=args.replicate_frac, layout=args.layout, cache_gib=args.cache_gib) if part else {}
     st = build_state(args.config, dev, rank, world, P, **kw)
     H = len(st.fanout)
     K = args.steps
@@ -691,11 +762,14 @@ def main():
     if part:
         # rows per owning bin of the median region's batches (deterministic: rerun on lane 0), then every
         # rank's counts, so each rank also knows how many of its bin's rows its peers read over NVLink
-        per_bin = torch.zeros(world, dtype=torch.int64, device=dev)
+        tiered = st.placement_mode == "ddak-tiered"
+        per_bin = torch.zeros(st.n_bins * world if tiered else world, dtype=torch.int64, device=dev)
         for i in sorted(set(used)):
             L0.ctx.step(st.graph.indptr, st.graph.indices, pool[i][0], st.fanout, pool[i][1], L0.bufs, None,
                         stream=main_stream)
-            per_bin += st.bins_of(L0.bufs.nodes, nF_pool[i]) * used.count(i)
+            # tiered: rows per route queue (bin, via rank); else rows per owning HBM bin
+            cnt = st.queues_of(L0.bufs.nodes, nF_pool[i]) if tiered else st.bins_of(L0.bufs.nodes, nF_pool[i])
+            per_bin += cnt * used.count(i)
         # every rank: every row of one of its batches, gathered through the local and the peers' (CUDA-IPC
         # mapped) bins, equals the generated bytes of its id (the oracle's table[ids]; the sampler is per rank
         # and checked by the N = 1 parity subset)
@@ -707,7 +781,8 @@ def main():
         rows_ok = True
         for c0 in range(0, nf0, 1 << 18):
             c1 = min(nf0, c0 + (1 << 18))
-            rows_ok &= bool(torch.equal(L0.rows[c0:c1], W.feature_rows(L0.bufs.nodes[c0:c1], st.dim, st.dtype)))
+            rows_ok &= bool(torch.equal(L0.rows[c0:c1],
+                                        W.feature_rows(feature_check_ids(st, L0.bufs.nodes[c0:c1]), st.dim, st.dtype)))
         okt = torch.tensor([int(rows_ok)], dtype=torch.int64, device=dev if not shared else "cpu")
         if dist:
             dist.all_reduce(okt, op=dist.ReduceOp.MIN)
@@ -716,28 +791,46 @@ def main():
         allb = [torch.zeros_like(per_bin) for _ in range(world)]
         if dist:
             if shared:
-                allc = [torch.zeros(world, dtype=torch.int64) for _ in range(world)]
+                allc = [torch.zeros(per_bin.numel(), dtype=torch.int64) for _ in range(world)]
                 dist.all_gather(allc, per_bin.cpu())
                 allb = [c.to(dev) for c in allc]
             else:
                 dist.all_gather(allb, per_bin)
         else:
             allb = [per_bin]
-        mat = torch.stack(allb).cpu().numpy() / K  # [requester][owner] rows per batch
-        local = mat[rank, rank]
-        peer_in = mat[rank].sum() - local
-        peer_out = mat[:, rank].sum() - local
+        mat = torch.stack(allb).cpu().numpy() / K  # [requester][owner] (tiered: [requester][bin * world + via])
+        host_direct = relayed_in = served_relays = 0.0
+        if tiered:
+            q = lambda g, b, via: mat[g, b * world + via]  # noqa: E731
+            local = q(rank, rank, rank)
+            peer_in = sum(q(rank, b, b) for b in range(world) if b != rank)
+            peer_out = sum(q(g, rank, rank) for g in range(world) if g != rank)
+            hosts = range(world, st.n_bins)
+            host_direct = sum(q(rank, j, rank) for j in hosts)
+            relayed_in = sum(q(rank, j, h) for j in hosts for h in range(world) if h != rank)
+            served_relays = sum(q(g, j, rank) for g in range(world) if g != rank for j in hosts)
+        else:
+            local = mat[rank, rank]
+            peer_in = mat[rank].sum() - local
+            peer_out = mat[:, rank].sum() - local
         nf_b = nF_region / K
         hbm_b = (local + peer_out) * st.R + nf_b * (st.R + 8) + samp_bytes / K
         t_hbm = hbm_b / (_peaks()[0] * 1e9)
-        t_nvl = max(peer_in, peer_out) * st.R / (NVLINK_GBS * 1e9)
+        nv_in, nv_out = (peer_in + relayed_in) * st.R, (peer_out + served_relays) * st.R
+        t_nvl = max(nv_in, nv_out) / (NVLINK_GBS * 1e9)
+        pcie_b = (host_direct + served_relays) * st.R
+        t_pcie = pcie_b / (PORT_GBS * 1e9)
         t_meas = ms / K / 1000
+        t_all = {"hbm": t_hbm, "nvlink": t_nvl, "pcie": t_pcie}
         tiers = {"placement": st.placement_mode, "replicated_rows": st.replicated_rows, "bin_rows": st.bin_rows,
-                 "rows_per_batch": {"local_hbm": local, "peer_in_nvlink": peer_in, "served_to_peers_nvlink": peer_out},
-                 "bytes_per_batch": {"hbm": hbm_b, "nvlink_in": peer_in * st.R, "nvlink_out": peer_out * st.R},
-                 "t_us": {"hbm": t_hbm * 1e6, "nvlink": t_nvl * 1e6, "measured": t_meas * 1e6},
-                 "binding": "nvlink" if t_nvl > t_hbm else "hbm", "frac": max(t_hbm, t_nvl) / t_meas,
-                 "peaks": {"hbm_gbs": _peaks()[0], "nvlink_gbs": NVLINK_GBS,
+                 "rows_per_batch": {"local_hbm": local, "peer_in_nvlink": peer_in, "served_to_peers_nvlink": peer_out,
+                                    "host_direct_pcie": host_direct, "host_relayed_to_me": relayed_in,
+                                    "host_served_for_peers": served_relays},
+                 "bytes_per_batch": {"hbm": hbm_b, "nvlink_in": nv_in, "nvlink_out": nv_out, "pcie_in": pcie_b},
+                 "t_us": {"hbm": t_hbm * 1e6, "nvlink": t_nvl * 1e6, "pcie": t_pcie * 1e6, "measured": t_meas * 1e6},
+                 "binding": max(t_all, key=t_all.get), "frac": max(t_all.values()) / t_meas,
+                 "quota": st.quota.tolist() if tiered else None,
+                 "peaks": {"hbm_gbs": _peaks()[0], "nvlink_gbs": NVLINK_GBS, "pcie_port_gbs": PORT_GBS,
                            "nvlink_source": "measured B200 peer copy per direction (B200_PROFILING.md; 900 nominal)"},
                  "plan": {"t_star_us": st.plan["t_star"], "t_nvlink_us": st.plan["t_nvlink"],
                           "t_hbm_us": st.plan["t_hbm"],
@@ -882,10 +975,14 @@ def main():
             tiers["plan"]["gather_us_measured"] = gather_ms * 1000
             line["tiers"] = tiers
             line["config"]["parallelism"] = f"dp{world}, features DDAK-partitioned over {world} HBM bins" + (
-                f" + {st.replicated_rows} replicated rows" if st.replicated_rows else "")
+                f" + {st.replicated_rows} replicated rows" if st.replicated_rows else "") + (
+                f" (HBM caches of {args.cache_gib:g} GiB) + {st.n_bins - world} pinned host bins (rings of "
+                f"{st.r_phys} rows), quota-routed relays" if st.placement_mode == "ddak-tiered" else "")
             line["config"]["l2"] = "no flush: inputs larger than L2 (features %.2f GB over all GPUs, CSR %.2f GB)" % (
                 st.graph.n * st.stride / 1e9, (st.graph.indptr.numel() * 8 + st.graph.indices.numel() * 4) / 1e9)
-            line["roofline"]["kernel"] = "gather_kernel (placement map; peer rows over NVLink)"
+            line["roofline"]["kernel"] = ("gather_kernel (placement map; peer rows over NVLink)" +
+                                          ("; host rows over PCIe, relayed by peers inside moment_step"
+                                           if st.placement_mode == "ddak-tiered" else ""))
             line["roofline"]["traffic"] = None
             line["roofline"]["launch_shares"] = None
             line["roofline"]["why_this_kernel"] = None

@@ -122,3 +122,35 @@ def test_bench_partitioned_layout_reuse(tmp_path):
     _run(args)
     assert os.path.exists(lay)
     _run(args)
+
+
+@pytest.mark.gpu
+def test_bench_tiered_one_rank():
+    """N = 1, ddak-tiered: a small HBM cache + pinned host bins read zero-copy; every gathered row of the parity
+    subset byte-exact; host rows accounted over PCIe."""
+    line = _run(["--config", "C1", "--placement", "ddak-tiered", "--cache-gib", "0.008", "--steps", "10", "--warmup",
+                 "3", "--min-time", "0.1", "--e2e-min-time", "0.05", "--presample", "8"])
+    assert line["cpu_baseline"]["parity"]["bit_exact"]
+    t = line["tiers"]
+    assert t["rows_per_batch"]["host_direct_pcie"] > 0 and t["rows_per_batch"]["local_hbm"] > 0
+    assert t["rows_per_batch"]["host_relayed_to_me"] == 0
+
+
+@pytest.mark.gpu
+def test_bench_tiered_two_ranks_shared_gpu():
+    """N = 2 ranks sharing cuda:0 (test mode): HBM caches + host bins, the plan's quotas, relays through the peer
+    rank inside every collective moment_step (moment_ctx_set_exchange); every rank's rows of one batch
+    byte-exact; relayed rows one rank receives are the rows the other serves."""
+    line = _run_torchrun(2, ["--gpus", "2", "--config", "C1", "--placement", "ddak-tiered", "--cache-gib", "0.004",
+                             "--steps", "6", "--warmup", "3", "--inflight", "2", "--min-time", "0.05",
+                             "--e2e-min-time", "0.02", "--presample", "64"],
+                         env={"MOMENT_BENCH_SHARED_GPU": "1"})
+    t = line["tiers"]
+    assert t["rows_check"]["byte_exact"] and line["n_gpus"] == 2
+    r = t["rows_per_batch"]
+    assert r["peer_in_nvlink"] > 0
+    # the two GPUs sit on different sockets (spread_gpus): the plan ingests each socket's host bin through its
+    # own GPU's port, so rank 0 reads host bin 0 directly and gets host bin 1's rows relayed by rank 1
+    q = t["quota"]
+    assert len(q) == 4 and q[2][0] > 0 and q[2][1] == 0 and q[3][0] == 0 and q[3][1] > 0
+    assert r["host_direct_pcie"] > 0 and r["host_relayed_to_me"] > 0 and r["host_served_for_peers"] > 0
