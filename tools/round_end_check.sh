@@ -1,10 +1,11 @@
 #!/bin/bash
-# Full GPU suite, smoke, bench repeats, launch list and one-step ncu of C2 on the current build.
+# Full GPU suite, smoke, the driver's bench commands, launch list and one-step ncu of C2 on the current build.
 mkdir -p gpurun_out
-timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.txt 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.txt
+timeout 1800 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.txt 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.txt
 timeout 300 python -c "import __graft_entry__ as g; g.smoke(); print('smoke ok')" > gpurun_out/smoke.txt 2>&1
-for i in 1 2 3; do timeout 600 python bench.py > gpurun_out/bench_$i.json 2> gpurun_out/bench_$i.err; done
-timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err
-timeout 600 bash tools/ncu_launches.sh gpurun_out/launches.csv C2 8 > gpurun_out/launch_list.txt 2>&1
+for i in 1 2; do timeout 600 python3 bench.py --gpus 1 --steps 20 --warmup 5 > gpurun_out/bench_$i.json 2> gpurun_out/bench_$i.err; done
+timeout 600 python3 bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err
+timeout 600 python3 bench.py --impl reference --gpus 1 --steps 20 --warmup 5 > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err
+timeout 600 bash tools/ncu_launches.sh gpurun_out/launches.csv C2 8 20 5 16 > gpurun_out/launch_list.txt 2>&1
 timeout 900 bash tools/ncu_full.sh gpurun_out/prof_full_C2 C2 > gpurun_out/ncu_full_C2.txt 2>&1
 rm -f gpurun_out/*.ncu-rep
