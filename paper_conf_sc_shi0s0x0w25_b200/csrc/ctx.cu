@@ -145,7 +145,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     c->bin_owner.assign(a->bin_owner, a->bin_owner + a->n_bins);
     c->bin_ptr.assign(a->bin_ptr, a->bin_ptr + a->n_bins);
     c->placement = a->placement;
-    c->n_sms = device_sms();
+    device_sms();  // query (and cache) the device's multiprocessor count once, outside any stream capture
     if (const char* gp = std::getenv("MOMENT_GATHER_PATH")) {
         const std::string v(gp);
         c->gather_path = v == "ldg" ? 1 : (v == "bulk" ? 2 : (v == "tma4" ? 3 : 0));

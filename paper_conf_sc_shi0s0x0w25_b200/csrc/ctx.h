@@ -44,7 +44,6 @@ struct moment_ctx_s {
     int32_t hop_warp_segmented = 1;   // k <= 32: k-lane groups packed in a warp (MOMENT_HOP_WARP=0: 2^n tiles)
     int32_t init_in_hop0 = 1;         // the first hop's sampler also initialises the call (MOMENT_INIT_KERNEL=1: separate)
     int32_t bulk_stages = 4, bulk_blocks_per_sm = 4, bulk_stage_kb = 14;  // bulk gather shape (MOMENT_BULK="S,B,KB")
-    int32_t n_sms = 148;  // multiprocessors of the ctx's device (cudaDevAttrMultiProcessorCount)
     std::vector<int32_t> bin_owner;
     std::vector<void*> bin_ptr;
     const uint64_t* placement = nullptr;
