@@ -40,7 +40,8 @@ struct moment_ctx_s {
     // dense bitscan prefetches each new id's first neighbour line (MOMENT_SCAN_PREFETCH=0/1; -1 = only when the
     // CSR has <= 8 M edges)
     int32_t scan_prefetch = -1;
-    int32_t hop_nodes_per_group = 2;  // nodes per lane group on large frontiers (1, 2, 4, 8)
+    int32_t hop_nodes_per_group = 1;  // nodes per lane group on large frontiers (1, 2, 4, 8); round 2 build: 1
+                                      // beats 2 by ~1 % per step (tools/knob_sweep_r02.sh), 4 loses 2.5 %
     int32_t hop_warp_segmented = 1;   // k <= 32: k-lane groups packed in a warp (MOMENT_HOP_WARP=0: 2^n tiles)
     int32_t init_in_hop0 = 1;         // the first hop's sampler also initialises the call (MOMENT_INIT_KERNEL=1: separate)
     int32_t bulk_stages = 4, bulk_blocks_per_sm = 4, bulk_stage_kb = 14;  // bulk gather shape (MOMENT_BULK="S,B,KB")
