@@ -36,8 +36,9 @@ constexpr int kScanTileWords = kBitscanTileWords;   // words per tile
 static_assert(kScanWords % 4 == 0, "bitscan loads whole uint4s");
 constexpr int kMaxHops = 16;
 #ifndef MOMENT_SAMPLE_MIN_BLOCKS
-#define MOMENT_SAMPLE_MIN_BLOCKS 6  // __launch_bounds__ min blocks per SM of the sampler kernels (<= 40 registers:
-                                    // measured +5-8 % vs uncapped at 1 and 8 batches in flight)
+#define MOMENT_SAMPLE_MIN_BLOCKS 8  // __launch_bounds__ min blocks per SM of the sampler kernels (<= 32 registers,
+                                    // the SM's full 2048 threads: round 2, one node per group, +1.5 % per step vs 6 /
+                                    // 40 registers, which measured +5-8 % over uncapped in round 1)
 #endif
 constexpr uint64_t kBaseReady = 1ull << 63;
 
