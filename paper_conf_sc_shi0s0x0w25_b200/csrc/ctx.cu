@@ -283,16 +283,21 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     c->d_call = reinterpret_cast<uint64_t*>(w + o_call);
     moment_status st = MOMENT_OK;
     do {
-        {  // kernel attributes, once per device. Shared-memory carveout: MOMENT_CARVEOUT (percent), default
-           // -1 = driver's per-kernel choice (measured best: a forced 100 % starves compact of L1, 2x slower)
+        {  // kernel attributes, once per device. Shared-memory carveout preference (percent of the unified
+           // L1 / shared storage): the sampler kernels ask for 25 % (L1 for their random CSR / rank-table reads:
+           // +2.4 % at K = 20, +0.4 % at K = 200; 0 % forces reconfigurations, 100 % starves compact of L1, 2x
+           // slower), the gathers keep the driver's per-kernel choice (-1). MOMENT_CARVEOUT sets both,
+           // MOMENT_CARVEOUT_SAMPLE / _GATHER one group (tools/sweep_carveout.sh)
             static std::mutex mu;
             static uint64_t done = 0;
             std::lock_guard<std::mutex> lock(mu);
             if (a->device < 64 && !(done >> a->device & 1)) {
                 const char* cv_env = std::getenv("MOMENT_CARVEOUT");
-                const int carve = cv_env ? std::atoi(cv_env) : -1;
-                if ((st = configure_sample_kernels(carve)) != MOMENT_OK) break;
-                if ((st = configure_gather_kernels(carve)) != MOMENT_OK) break;
+                int carve_s = cv_env ? std::atoi(cv_env) : 25, carve_g = cv_env ? std::atoi(cv_env) : -1;
+                if (const char* v = std::getenv("MOMENT_CARVEOUT_SAMPLE")) carve_s = std::atoi(v);
+                if (const char* v = std::getenv("MOMENT_CARVEOUT_GATHER")) carve_g = std::atoi(v);
+                if ((st = configure_sample_kernels(carve_s)) != MOMENT_OK) break;
+                if ((st = configure_gather_kernels(carve_g)) != MOMENT_OK) break;
                 done |= 1ull << a->device;
             }
         }
