@@ -624,7 +624,10 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0, help="seconds of oracle time for cpu_baseline")
     # 12-16 measured best on C2 (29.5-29.7 M seeds/s vs 27.7 at 8, 28.4 at 24)
-    ap.add_argument("--inflight", type=int, default=16, help="batches in flight per GPU (one stream each)")
+    ap.add_argument("--inflight", type=int, default=0,
+                    help="batches in flight per GPU (one stream each); 0 = auto: 16 for short regions (K <= 24: "
+                         "fill and drain dominate, 20 lanes lose 1 %% at K = 20), 32 for longer ones when a lane's row "
+                         "buffer is small (C2 K = 200: 38.8 vs 37.8 M seeds/s at 16), else 16")
     ap.add_argument("--placement", default="replicated", choices=["replicated", "ddak", "ddak-rep", "ddak-tiered"],
                     help="replicated: every GPU holds the whole table (C2 'all features in HBM'); ddak: the table "
                          "partitioned over the GPUs' HBM by DDAK (C3), peer rows read over NVLink; ddak-rep: the "
@@ -663,6 +666,13 @@ def main():
             dist.init_process_group("gloo")
         else:
             dist.init_process_group("nccl", device_id=torch.device(dev))
+    if args.inflight <= 0:
+        cfg_ = W.CONFIGS[args.config]
+        fb = cfg_["batch"]
+        for k_ in cfg_["fanout"]:
+            fb = min(fb + fb * k_, cfg_["n"])
+        row_buf = fb * cfg_["dim"] * torch.empty(0, dtype=cfg_["dtype"]).element_size()
+        args.inflight = 16 if args.steps <= 24 or row_buf > (1 << 30) else 32
     P = max(1, min(args.inflight, args.steps))
     part = args.placement != "replicated"
     kw = dict(placement=args.placement, dist=dist, shared=shared, presample=args.presample,
