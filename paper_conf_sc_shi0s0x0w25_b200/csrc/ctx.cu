@@ -330,6 +330,7 @@ extern "C" moment_status moment_ctx_free(moment_ctx_t ctx) {
     cudaGetDevice(&cur);
     cudaSetDevice(ctx->device);
     if (ctx->step_exec) cudaGraphExecDestroy(ctx->step_exec);
+    if (ctx->step_graph) cudaGraphDestroy(ctx->step_graph);
     if (ctx->cap_stream) cudaStreamDestroy(ctx->cap_stream);
     if (ctx->cap_side) cudaStreamDestroy(ctx->cap_side);
     if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
@@ -367,6 +368,8 @@ extern "C" moment_status moment_ctx_set_exchange(moment_ctx_t ctx, const moment_
     if (ctx->step_exec) {  // a cached step graph captured without the exchange is stale
         cudaGraphExecDestroy(ctx->step_exec);
         ctx->step_exec = nullptr;
+        cudaGraphDestroy(ctx->step_graph);
+        ctx->step_graph = nullptr;
     }
     return MOMENT_OK;
 }
@@ -425,12 +428,44 @@ bool same_key(const moment_ctx_s::StepKey& k, const moment_csr* csr, int64_t n_s
 
 // One sample + gather, replayed from a cached CUDA graph (captured on first use of a shape); falls back to
 // direct launches while the caller's stream is itself being captured.
+// The call-block kernel's parameters for one call (the graph's first node; updated per launch).
+struct CallParams {
+    uint64_t* call;
+    uint64_t rng_seed;
+    const int64_t* seeds;
+    int64_t* counts_host;
+    unsigned long long* zero;
+    int64_t n_zero;
+};
+
+moment_status set_call_node(moment_ctx_s* c, const CallParams& cp) {
+    void* args[] = {(void*)&cp.call, (void*)&cp.rng_seed, (void*)&cp.seeds, (void*)&cp.counts_host, (void*)&cp.zero,
+                    (void*)&cp.n_zero};
+    cudaKernelNodeParams kp{};
+    kp.func = (void*)set_call_kernel;
+    kp.gridDim = dim3(1);
+    kp.blockDim = dim3(32);
+    kp.sharedMemBytes = 0;
+    kp.kernelParams = args;
+    return cuda_check(cudaGraphExecKernelNodeSetParams(c->step_exec, c->call_node, &kp), "moment_step: call node");
+}
+
+// One step (moment_step / moment_step_host): the call block (rng seed, seeds pointer, host counts pointer) is
+// written by set_call_kernel, then sample + gather. From a CUDA graph cached in the ctx, the call kernel is the
+// graph's first node and its parameters are replaced per launch (cudaGraphExecKernelNodeSetParams), so a step
+// is one graph launch with no separate kernel launch in front of it (measured: the separate launch left a
+// ~5 us gap before the first hop). While the caller's stream is being captured, or with MOMENT_NO_GRAPH, the
+// kernels are launched directly.
 moment_status run_step(moment_ctx_s* c, const moment_csr* csr, int64_t n_seeds, const moment_sample_params* p,
-                       const moment_sample_out* out, void* rows, cudaStream_t s) {
+                       const moment_sample_out* out, void* rows, cudaStream_t s, const int64_t* seeds,
+                       int64_t* counts_host = nullptr) {
     const int H = p->n_hops;
+    const CallParams cp{c->d_call, p->rng_seed, seeds, counts_host, c->tile_edges,
+                        std::min<int64_t>((n_seeds + kSampleTile - 1) / kSampleTile, c->n_tile_edges)};
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
     MOMENT_TRY(cuda_check(cudaStreamIsCapturing(s, &cs), "moment_step"));
     if (cs != cudaStreamCaptureStatusNone || std::getenv("MOMENT_NO_GRAPH")) {
+        MOMENT_TRY(write_call(c, p->rng_seed, seeds, n_seeds, s, counts_host));
         MOMENT_TRY(launch_sample(c, csr, c->d_call, n_seeds, p, out, s));
         if (rows) MOMENT_TRY(launch_gather_any(c, out->nodes, out->counts + H, out->cap_nodes, rows, s));
         return MOMENT_OK;
@@ -441,9 +476,15 @@ moment_status run_step(moment_ctx_s* c, const moment_csr* csr, int64_t n_seeds, 
             cudaGraphExecDestroy(c->step_exec);
             c->step_exec = nullptr;
         }
+        if (c->step_graph) {
+            cudaGraphDestroy(c->step_graph);
+            c->step_graph = nullptr;
+        }
         MOMENT_TRY(cuda_check(cudaStreamBeginCapture(c->cap_stream, cudaStreamCaptureModeThreadLocal), "capture"));
         const bool fork = rows && c->step_fork;
-        moment_status st = launch_sample(c, csr, c->d_call, n_seeds, p, out, c->cap_stream, fork ? c->ev_fork : nullptr);
+        moment_status st = write_call(c, p->rng_seed, seeds, n_seeds, c->cap_stream, counts_host);
+        if (st == MOMENT_OK)
+            st = launch_sample(c, csr, c->d_call, n_seeds, p, out, c->cap_stream, fork ? c->ev_fork : nullptr);
         if (st == MOMENT_OK && rows && !fork)
             st = launch_gather_any(c, out->nodes, out->counts + H, out->cap_nodes, rows, c->cap_stream);
         if (st == MOMENT_OK && fork) {  // gather on a branch that joins after the compaction
@@ -460,9 +501,19 @@ moment_status run_step(moment_ctx_s* c, const moment_csr* csr, int64_t n_seeds, 
             return st;
         }
         MOMENT_TRY(cuda_check(e, "moment_step: end capture"));
+        // the call kernel is the graph's only root (captured first; everything else depends on it)
+        size_t n_roots = 1;
+        e = cudaGraphGetRootNodes(g, &c->call_node, &n_roots);
+        if (e != cudaSuccess || n_roots != 1) {
+            cudaGraphDestroy(g);
+            return fail(MOMENT_ECUDA, "moment_step: captured graph has %zu roots", n_roots);
+        }
         e = cudaGraphInstantiate(&c->step_exec, g, 0);
-        cudaGraphDestroy(g);
-        MOMENT_TRY(cuda_check(e, "moment_step: instantiate"));
+        if (e != cudaSuccess) {
+            cudaGraphDestroy(g);
+            MOMENT_TRY(cuda_check(e, "moment_step: instantiate"));
+        }
+        c->step_graph = g;  // kept: the call node handle refers to it
         c->step_key.indptr = csr->indptr;
         c->step_key.indices = csr->indices;
         c->step_key.n_seeds = n_seeds;
@@ -471,6 +522,7 @@ moment_status run_step(moment_ctx_s* c, const moment_csr* csr, int64_t n_seeds, 
         c->step_key.out = *out;
         c->step_key.rows = rows;
     }
+    MOMENT_TRY(set_call_node(c, cp));
     return cuda_check(cudaGraphLaunch(c->step_exec, s), "moment_step: graph launch");
 }
 
@@ -514,8 +566,7 @@ extern "C" moment_status moment_step(moment_ctx_t ctx, const moment_csr* csr, co
     MOMENT_TRY(check_sample(ctx, csr, seeds, n_seeds, params, out));
     MOMENT_TRY(check_rows(ctx, d_rows, out));
     cudaStream_t s = static_cast<cudaStream_t>(stream);
-    MOMENT_TRY(write_call(ctx, params->rng_seed, seeds, n_seeds, s));
-    return run_step(ctx, csr, n_seeds, params, out, d_rows, s);
+    return run_step(ctx, csr, n_seeds, params, out, d_rows, s, seeds);
 }
 
 extern "C" moment_status moment_sample_check(moment_ctx_t ctx, void* stream) {
@@ -601,8 +652,7 @@ extern "C" moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* cs
                                               cudaMemcpyHostToDevice, s), "moment_step_host: H2D"));
         seeds_dev = ctx->d_seed_stage;
     }
-    MOMENT_TRY(write_call(ctx, params->rng_seed, seeds_dev, n_seeds, s, counts_dev));
-    MOMENT_TRY(run_step(ctx, csr, n_seeds, params, out, d_rows, s));
+    MOMENT_TRY(run_step(ctx, csr, n_seeds, params, out, d_rows, s, seeds_dev, counts_dev));
     if (counts_dev) return MOMENT_OK;
     const int H = params->n_hops;
     return cuda_check(cudaMemcpyAsync(counts_host, out->counts, (2 * H + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s),

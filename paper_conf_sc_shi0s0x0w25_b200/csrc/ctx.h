@@ -104,6 +104,8 @@ struct moment_ctx_s {
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     int32_t step_fork = 1;  // MOMENT_STEP_FORK=0: gather after compact on one chain
     cudaGraphExec_t step_exec = nullptr;
+    cudaGraph_t step_graph = nullptr;     // the captured graph (kept: call_node refers to it)
+    cudaGraphNode_t call_node = nullptr;  // its set_call kernel node, re-parameterised per launch
     struct StepKey {
         const void* indptr = nullptr;
         const void* indices = nullptr;
