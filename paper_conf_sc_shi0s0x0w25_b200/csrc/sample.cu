@@ -461,7 +461,15 @@ struct ScanArgs {
 // kPrefetch: a separate instantiation, so the default scan's code is not touched by the prefetch branch (the
 // runtime-flag version slowed the C2 scans by ~20 % with the flag off)
 template <bool kPrefetch>
-__global__ void __launch_bounds__(kBitscanThreads) bitscan_kernel(ScanArgs a) {
+// Register caps (round 2): with 16+ batches in flight the SMs' register files decide how many of the lanes'
+// kernels are resident at once, so the dense bitscan is held to 40 registers (3 x 512-thread blocks per SM;
+// uncapped it took 80) and the compaction to 40 (6 x 256-thread blocks per SM, 6 slots in flight; was 64 with
+// 8): sampling-only 13.3 -> 11.5 us per batch at 16 lanes, the full step -1 %, the driver's K = 20 +2 %
+// (tools/ab_multi.sh, profiles/r02_sampler_experiments.txt)
+#ifndef MOMENT_SCAN_MINB
+#define MOMENT_SCAN_MINB 3
+#endif
+__global__ void __launch_bounds__(kBitscanThreads, MOMENT_SCAN_MINB) bitscan_kernel(ScanArgs a) {
     __shared__ int64_t s_red[kBitscanThreads / 32];
     __shared__ uint32_t s_tile;
     __shared__ int s_nearest;
@@ -689,10 +697,17 @@ __device__ __forceinline__ void block_sum2(int64_t& x, int64_t& y, int64_t (*red
 // All hops' offsets and src in one wait-free pass: a tile's first edge position is the sum of the edge
 // counts of the tiles before it, which the hop kernels accumulated per tile (no chained scan, no waiting
 // on other blocks); the hop's base is the sum over the earlier hops' tiles.
-// 4 blocks/SM minimum (<= 64 registers): its grid is capped at 2 blocks/SM, and the samplers' 40-register cap
-// made it spill (48 B); measured +1.3 % bench at K = 20, +0.5 % per step at 16 lanes (tools/ab_lib.sh)
-__global__ void __launch_bounds__(kSampleTile, 4) compact_kernel(CompactArgs a) {
-    constexpr int kCopyUnroll = 8;  // padded slots per thread in flight (id load -> lidx load -> src store)
+// 6 blocks/SM minimum (<= 40 registers, 6 slots in flight per thread; its grid is capped at 2 blocks/SM):
+// round 1 held it at 64 registers (8 slots: spilled at 40), round 2 measured the smaller footprint faster once
+// many lanes' kernels compete for the register files (see MOMENT_SCAN_MINB)
+#ifndef MOMENT_COMPACT_MINB
+#define MOMENT_COMPACT_MINB 6  // 40 registers (see MOMENT_SCAN_MINB)
+#endif
+#ifndef MOMENT_COMPACT_UNROLL
+#define MOMENT_COMPACT_UNROLL 6  // 8 spills at 40 registers
+#endif
+__global__ void __launch_bounds__(kSampleTile, MOMENT_COMPACT_MINB) compact_kernel(CompactArgs a) {
+    constexpr int kCopyUnroll = MOMENT_COMPACT_UNROLL;  // padded slots per thread in flight (id -> rel / lidx -> src)
     __shared__ int64_t s_red[kSampleTile / 32];
     __shared__ int64_t s_red2[kSampleTile / 32][2];
     __shared__ int32_t s_excl[kSampleTile], s_cnt[kSampleTile];
