@@ -460,7 +460,6 @@ struct ScanArgs {
 // F_{h+1} = F_h ++ ascending ids set in (newbits & ~visited).
 // kPrefetch: a separate instantiation, so the default scan's code is not touched by the prefetch branch (the
 // runtime-flag version slowed the C2 scans by ~20 % with the flag off)
-template <bool kPrefetch>
 // Register caps (round 2): with 16+ batches in flight the SMs' register files decide how many of the lanes'
 // kernels are resident at once, so the dense bitscan is held to 40 registers (3 x 512-thread blocks per SM;
 // uncapped it took 80) and the compaction to 40 (6 x 256-thread blocks per SM, 6 slots in flight; was 64 with
@@ -469,6 +468,7 @@ template <bool kPrefetch>
 #ifndef MOMENT_SCAN_MINB
 #define MOMENT_SCAN_MINB 3
 #endif
+template <bool kPrefetch>
 __global__ void __launch_bounds__(kBitscanThreads, MOMENT_SCAN_MINB) bitscan_kernel(ScanArgs a) {
     __shared__ int64_t s_red[kBitscanThreads / 32];
     __shared__ uint32_t s_tile;
