@@ -40,7 +40,8 @@ struct moment_ctx_s {
     // dense bitscan prefetches each new id's first neighbour line (MOMENT_SCAN_PREFETCH=0/1; -1 = only when the
     // CSR has <= 8 M edges)
     int32_t scan_prefetch = -1;
-    int32_t hop_nodes_per_group = 1;  // nodes per lane group on large frontiers (1, 2, 4, 8); round 2 build: 1
+    int32_t hop_nodes_per_group = 2;  // nodes per lane group on large frontiers (1, 2, 4): 2 since the round-2 register
+                                      // caps (C2 K = 200 39.9 -> 40.3, K = 20 36.6 -> 36.8 M seeds/s)
                                       // beats 2 by ~1 % per step (tools/knob_sweep_r02.sh), 4 loses 2.5 %
     int32_t hop_warp_segmented = 1;   // k <= 32: k-lane groups packed in a warp (MOMENT_HOP_WARP=0: 2^n tiles)
     int32_t init_in_hop0 = 1;         // the first hop's sampler also initialises the call (MOMENT_INIT_KERNEL=1: separate)
