@@ -152,6 +152,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     }
     if (const char* v = std::getenv("MOMENT_TMA_PROMO")) c->tma_promo = std::max(0, std::min(3, std::atoi(v)));
     if (const char* v = std::getenv("MOMENT_TMA4_BLOCKS")) c->tma4_blocks_per_sm = std::max(1, std::atoi(v));
+    if (const char* v = std::getenv("MOMENT_TMA4_ROWS")) c->tma4_rows = std::atoi(v);
     if (const char* v = std::getenv("MOMENT_BULK"))
         std::sscanf(v, "%d,%d,%d", &c->bulk_stages, &c->bulk_blocks_per_sm, &c->bulk_stage_kb);
     if (const char* v = std::getenv("MOMENT_HOP_GRID")) c->hop_grid_per_sm = std::max(1, std::atoi(v));

@@ -27,7 +27,14 @@ struct moment_ctx_s {
     // L2 promotion of the gathered rows: 64 B (measured: a 400-byte row then costs 448 B of DRAM reads instead
     // of the 512 B whole 128-byte lines the default fetches; MOMENT_TMA_PROMO: 0 none, 1 64B, 2 128B, 3 256B)
     int32_t tma_promo = 1;
-    int32_t tma4_blocks_per_sm = 2;  // 1-warp gather4 blocks per SM, 4 stages of 8 x 4 rows (MOMENT_TMA4_BLOCKS)
+    // gather4 launch shape: 1-warp blocks of 4 stages x tma4_rows rows, tma4_blocks_per_sm per SM (MOMENT_TMA4_BLOCKS,
+    // MOMENT_TMA4_ROWS = 8 / 16 / 32). A lone launch streams faster with more issuing warps per SM (1: 0.55 of the
+    // copy peak, 2: 0.61-0.73, 3-4: 0.72-0.74), while inside the saturated step the gather should hold little
+    // shared memory per SM (co-resident sampler kernels want L1): 16-row tiles x 3 blocks (80 KB per SM) keep the
+    // lone launch at 0.72 and cut the step 25.9 -> 25.2 us vs round 1's 32 x 2 (106 KB per SM)
+    // (profiles/r02_sampler_experiments.txt)
+    int32_t tma4_blocks_per_sm = 3;
+    int32_t tma4_rows = 16;
     int32_t l2_load_policy = 0, l2_store_policy = 1;  // bulk gather L2 hints: 0 normal, 1 evict_first, 2 evict_last
     // launch shapes, re-tuned after rank relabelling with 16 batches in flight (C2 bench 33.5 -> 36.5 M
     // seeds/s, C3 10.5 -> 10.9 against the earlier 4 / 1 / 4 / 3): MOMENT_HOP_GRID, MOMENT_COMPACT_GRID,

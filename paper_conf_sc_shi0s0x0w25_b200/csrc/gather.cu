@@ -229,8 +229,8 @@ __global__ void __launch_bounds__(32) gather_bulk_kernel(BinTable bins, const ui
 // reads. Each group of 4 rows lands at a 128-byte aligned smem slot (G bytes) and is stored back with its
 // own bulk copy (per-lane bulk groups). Rows past the end of a tile repeat the tile's first row and are
 // not stored.
-constexpr int kTma4Rows = 32;  // rows per tile = 8 groups of 4
-template <int kStages, bool kPlacement>
+constexpr int kTma4Rows = 32;  // rows per tile = 8 groups of 4 (kRows = 16 / 8: 4 / 2 groups; ctx tma4_rows)
+template <int kStages, bool kPlacement, int kRows = kTma4Rows>
 __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__ CUtensorMap tmap,
                                                          const int64_t* __restrict__ ids, const int64_t* n_dev,
                                                          int64_t max_n, uint32_t R, int l2_load, int l2_store,
@@ -250,7 +250,7 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
     int64_t pid[kStages];
 #pragma unroll
     for (int s = 0; s < kStages; s++) {
-        const int64_t r = (t0 + s * dt) * kTma4Rows + lane;
+        const int64_t r = (t0 + s * dt) * kRows + lane;
         pid[s] = r < max_n ? __ldg(ids + r) : -1;
     }
     const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
@@ -261,24 +261,24 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
 #pragma unroll
     for (int s = 0; s < kStages; s++)
         pre[s] = !kPlacement ? (int32_t)pid[s]
-                 : ((t0 + s * dt) * kTma4Rows + lane < n ? (int32_t)(dev::ld_rand(placement + pid[s]) & kSlotMask) : -1);
-    const int64_t n_tiles = (n + kTma4Rows - 1) / kTma4Rows;
+                 : ((t0 + s * dt) * kRows + lane < n ? (int32_t)(dev::ld_rand(placement + pid[s]) & kSlotMask) : -1);
+    const int64_t n_tiles = (n + kRows - 1) / kRows;
     if (lane == 0)
         for (int s = 0; s < kStages; s++) mbar_init(&full[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     __syncwarp();
     auto load_id = [&](int64_t tile) -> int32_t {
-        const int64_t r = tile * kTma4Rows + lane;
+        const int64_t r = tile * kRows + lane;
         if (!(tile < n_tiles && r < n)) return -1;
         const int64_t id = __ldg(ids + r);
         return kPlacement ? (int32_t)(dev::ld_rand(placement + id) & kSlotMask) : (int32_t)id;
     };
     auto issue = [&](int64_t tile, int s, int32_t id) {
-        const int rows = (int)min((int64_t)kTma4Rows, n - tile * kTma4Rows);
+        const int rows = (int)min((int64_t)kRows, n - tile * kRows);
         const int groups = (rows + 3) >> 2;
         const int32_t first = __shfl_sync(0xffffffffu, id, 0);
         const int32_t rid = lane < rows ? id : first;
-        const int g = lane & 7;
+        const int g = lane & (kRows / 4 - 1);
         const int32_t r0 = __shfl_sync(0xffffffffu, rid, 4 * g), r1 = __shfl_sync(0xffffffffu, rid, 4 * g + 1);
         const int32_t r2 = __shfl_sync(0xffffffffu, rid, 4 * g + 2), r3 = __shfl_sync(0xffffffffu, rid, 4 * g + 3);
         if (lane == 0) mbar_expect_tx(&full[s], (uint32_t)groups * 4u * R);
@@ -287,13 +287,13 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
             if (l2_load)  // L2 eviction priority of the fetched rows (MOMENT_GATHER_L2 first digit)
                 asm volatile(
                     "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes.L2::cache_hint "
-                    "[%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(smem_u32(stage + ((size_t)s * 8 + lane) * G)),
+                    "[%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(smem_u32(stage + ((size_t)s * (kRows / 4) + lane) * G)),
                     "l"(&tmap), "r"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(&full[s])), "l"(pol_ld)
                     : "memory");
             else
                 asm volatile(
                     "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes [%0], [%1, {%2, "
-                    "%3, %4, %5, %6}], [%7];" ::"r"(smem_u32(stage + ((size_t)s * 8 + lane) * G)),
+                    "%3, %4, %5, %6}], [%7];" ::"r"(smem_u32(stage + ((size_t)s * (kRows / 4) + lane) * G)),
                     "l"(&tmap), "r"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(&full[s]))
                     : "memory");
         }
@@ -307,11 +307,11 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
     for (int64_t tile = t0; tile < n_tiles; tile += dt, it++) {
         const int s = it % kStages;
         mbar_wait(&full[s], (uint32_t)((it / kStages) & 1));
-        const int64_t row0 = tile * kTma4Rows;
-        const int rows = (int)min((int64_t)kTma4Rows, n - row0);
+        const int64_t row0 = tile * kRows;
+        const int rows = (int)min((int64_t)kRows, n - row0);
         const int groups = (rows + 3) >> 2;
         if (lane < groups) {
-            bulk_store(out + (row0 + 4 * lane) * (int64_t)R, stage + ((size_t)s * 8 + lane) * G,
+            bulk_store(out + (row0 + 4 * lane) * (int64_t)R, stage + ((size_t)s * (kRows / 4) + lane) * G,
                        (uint32_t)min(4, rows - 4 * lane) * R, pol_st);
         }
         if (it > 0) bulk_wait_read<1>();  // this lane's store of the previous tile has read its slot
@@ -580,19 +580,23 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
     if (tma4) {
         if (ctx->tma_base != ctx->bin_ptr[0]) MOMENT_TRY(encode_table_map(ctx));
         const uint32_t G = (uint32_t)((4 * ctx->row_bytes + 127) & ~int64_t(127));
-        const int stages = 4, bps = ctx->tma4_blocks_per_sm;
-        const size_t smem = (size_t)stages * 8 * G;
-        const int64_t tiles = (max_n + kTma4Rows - 1) / kTma4Rows;
+        const int stages = 4, bps = ctx->tma4_blocks_per_sm, rows_t = ctx->tma4_rows <= 8 ? 8 : ctx->tma4_rows <= 16 ? 16 : 32;
+        const size_t smem = (size_t)stages * (rows_t / 4) * G;
+        const int64_t tiles = (max_n + rows_t - 1) / rows_t;
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)device_sms() * bps));
-        if (ctx->placement)
-            gather_tma4_kernel<4, true><<<grid, 32, smem, stream>>>(ctx->tma_map, ids, n_dev, max_n, (uint32_t)ctx->row_bytes,
-                                                                    ctx->l2_load_policy, ctx->l2_store_policy,
-                                                                    ctx->placement, reinterpret_cast<char*>(out));
-        else
-            gather_tma4_kernel<4, false><<<grid, 32, smem, stream>>>(ctx->tma_map, ids, n_dev, max_n,
-                                                                     (uint32_t)ctx->row_bytes, ctx->l2_load_policy,
-                                                                     ctx->l2_store_policy, nullptr,
-                                                                     reinterpret_cast<char*>(out));
+        auto launch = [&](auto kern) {
+            kern<<<grid, 32, smem, stream>>>(ctx->tma_map, ids, n_dev, max_n, (uint32_t)ctx->row_bytes, ctx->l2_load_policy,
+                                             ctx->l2_store_policy, ctx->placement, reinterpret_cast<char*>(out));
+        };
+        if (ctx->placement) {
+            if (rows_t == 8) launch(gather_tma4_kernel<4, true, 8>);
+            else if (rows_t == 16) launch(gather_tma4_kernel<4, true, 16>);
+            else launch(gather_tma4_kernel<4, true>);
+        } else {
+            if (rows_t == 8) launch(gather_tma4_kernel<4, false, 8>);
+            else if (rows_t == 16) launch(gather_tma4_kernel<4, false, 16>);
+            else launch(gather_tma4_kernel<4, false>);
+        }
         return cuda_check(cudaGetLastError(), "moment_gather: tma4 launch");
     }
     if (bulk && route == nullptr) {
@@ -906,7 +910,9 @@ moment_status configure_gather_kernels(int carveout) {
                                   "carveout attribute"));
     for (const void* f : {(const void*)gather_bulk_kernel<2>, (const void*)gather_bulk_kernel<4>,
                           (const void*)gather_bulk_kernel<6>, (const void*)gather_bulk_kernel<8>,
-                          (const void*)gather_tma4_kernel<4, false>, (const void*)gather_tma4_kernel<4, true>})
+                          (const void*)gather_tma4_kernel<4, false>, (const void*)gather_tma4_kernel<4, true>,
+                          (const void*)gather_tma4_kernel<4, false, 16>, (const void*)gather_tma4_kernel<4, true, 16>,
+                          (const void*)gather_tma4_kernel<4, false, 8>, (const void*)gather_tma4_kernel<4, true, 8>})
         MOMENT_TRY(cuda_check(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmemMax),
                               "bulk gather smem attribute"));
     return MOMENT_OK;

@@ -176,17 +176,26 @@ def test_sample_reused_ctx_many_batches(orc, c1, sparse, relabel, monkeypatch):
         assert_same_sample(got, want)
 
 
-@pytest.mark.parametrize("path", ["auto", "ldg", "bulk", "tma4"])
+def _gather_path_env(monkeypatch, path):
+    """MOMENT_GATHER_PATH; "tma4-rN": tile::gather4 with N-row tiles (MOMENT_TMA4_ROWS; default 16)."""
+    if path.startswith("tma4-r"):
+        monkeypatch.setenv("MOMENT_TMA4_ROWS", path[len("tma4-r"):])
+        path = "tma4"
+    monkeypatch.setenv("MOMENT_GATHER_PATH", path)
+    return path
+
+
+@pytest.mark.parametrize("path", ["auto", "ldg", "bulk", "tma4", "tma4-r8", "tma4-r32"])
 @pytest.mark.parametrize("dim,dtype", [(4, torch.float32), (12, torch.float32), (100, torch.float32),
                                        (128, torch.float32), (768, torch.float16), (1024, torch.float32)])
 def test_gather_replicated(orc, dim, dtype, path, monkeypatch):
     _need_gpu()
-    monkeypatch.setenv("MOMENT_GATHER_PATH", path)
+    path = _gather_path_env(monkeypatch, path)
     n = 5000
     table = W.feature_table(n, dim, dtype, device=DEV)
     R = table.shape[1]
     rng = np.random.default_rng(dim)
-    # counts past one round of tiles (148 SMs x 3 blocks x 32 rows) exercise the ragged last round
+    # counts past one round of tiles (148 SMs x 3 blocks x 16 rows) exercise the ragged last round
     for count in [1, 31, 1000, 4099] + ([15000, 50001] if path == "tma4" else []):
         ids = torch.as_tensor(rng.integers(0, n, count), device=DEV)
         ctx = M.Ctx(n_vertices=n, max_seeds=1, max_fanout=[1], device=0, row_bytes=R, bin_owner=[0],
@@ -203,14 +212,14 @@ def test_gather_replicated(orc, dim, dtype, path, monkeypatch):
         assert np.array_equal(o2[: count // 2], want[: count // 2]) and not o2[count // 2:].any()
 
 
-@pytest.mark.parametrize("path", ["auto", "ldg", "bulk", "tma4"])
+@pytest.mark.parametrize("path", ["auto", "ldg", "bulk", "tma4", "tma4-r8", "tma4-r32"])
 @pytest.mark.parametrize("dim,dtype", [(100, torch.float32), (128, torch.float32), (768, torch.float16)])
 def test_gather_one_local_bin_with_placement(orc, dim, dtype, path, monkeypatch):
     """One local bin addressed through a placement map (a DDAK layout on one GPU: row v at a permuted
     slot): tile::gather4 takes the slot as its row coordinate, the bulk gather resolves the placement one
     tile ahead; every path byte-exact with the oracle's table[ids]."""
     _need_gpu()
-    monkeypatch.setenv("MOMENT_GATHER_PATH", path)
+    path = _gather_path_env(monkeypatch, path)
     n = 7000
     table = W.feature_table(n, dim, dtype, device="cpu")
     R = table.shape[1]
