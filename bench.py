@@ -117,6 +117,9 @@ class State:
         H = len(self.fanout)
         L = self.lanes[lane]
         s = stream if stream is not None else L.stream
+        if ev is None and stream is None:  # the lane's prepared moment_step (one ctypes call per step)
+            self.bound(lane)(seeds, rng_seed)
+            return
         if ev is None:
             L.ctx.step(self.graph.indptr, self.graph.indices, seeds, self.fanout, rng_seed, L.bufs, L.rows, stream=s)
             return
@@ -125,11 +128,20 @@ class State:
         L.ctx.gather(L.bufs.nodes, L.rows, n_dev=L.bufs.counts[H:H + 1], max_n=L.bufs.nodes.numel(), stream=s)
         ev[1].record(s)
 
+    def bound(self, lane, host=False):
+        """The lane's moment_step (host: moment_step_host) prepared once on its stream (Ctx.bind_step)."""
+        L = self.lanes[lane]
+        key = "run_host" if host else "run"
+        run = L.__dict__.get(key)
+        if run is None:
+            run = L.ctx.bind_step(self.graph.indptr, self.graph.indices, self.fanout, L.bufs, L.rows, stream=L.stream,
+                                  host=host)
+            setattr(L, key, run)
+        return run
+
     def step_host(self, seeds_host, rng_seed, counts_host, lane=0):
         """The same step through moment_step_host: host seeds in, host counts out (asynchronous)."""
-        L = self.lanes[lane]
-        L.ctx.step_host(self.graph.indptr, self.graph.indices, seeds_host, self.fanout, rng_seed, L.bufs, L.rows,
-                        counts_host, stream=L.stream)
+        self.bound(lane, host=True)(seeds_host, rng_seed, counts_host)
 
     def launches_per_step(self):
         # set_call, (sample, bitscan) per hop (the first hop's sampler also initialises the call), compact, gather
@@ -743,9 +755,11 @@ def main():
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)  # per region, the slowest rank
         return tt.cpu().tolist()
 
+    runs = [st.bound(lane) for lane in range(P)]  # one ctypes call per step (Ctx.bind_step)
+
     def dev_step(i, lane):
-        b = pool[i % n_pool]
-        st.step(b[0], b[1], lane=lane)
+        seeds, rng_seed = pool[i % n_pool]
+        runs[lane](seeds, rng_seed)
 
     reg_ms = repeats(dev_step, args.min_time)
     ck = clocks.stop()
@@ -908,8 +922,10 @@ def main():
         st.step_host(seeds_pinned[i], pool[i][1], counts_pinned[i % K], lane=i)
     torch.cuda.synchronize()
 
+    runs_h = [st.bound(lane, host=True) for lane in range(P)]
+
     def host_step(i, lane):
-        st.step_host(seeds_pinned[i % n_pool], pool[i % n_pool][1], counts_pinned[i % K], lane=lane)
+        runs_h[lane](seeds_pinned[i % n_pool], pool[i % n_pool][1], counts_pinned[i % K])
 
     e2e_ms_all = repeats(host_step, args.e2e_min_time)
     e2e_ms = statistics.median(e2e_ms_all)

@@ -483,6 +483,36 @@ class Ctx:
                                  _stream(stream)))
         return out
 
+    def bind_step(self, indptr, indices, fanout, out: SampleBuffers, rows, *, flags: int = 0, stream=None,
+                  host: bool = False):
+        """moment_step (host=False: run(seeds, rng_seed)) or moment_step_host (host=True: run(seeds_host,
+        rng_seed, counts_host)) prepared for one (graph, fanout, buffers, rows, stream): the returned callable
+        marshals only the per-batch pointers and the rng seed (the argument structs are built once), so issuing
+        a step costs one ctypes call."""
+        a = self._args(indptr, indices, fanout, flags, out)
+        params, csr_r, par_r, so_r = a[1], a[4], a[5], a[6]
+        h, rows_p, sp = self.handle, _ptr(rows), _stream(stream)
+        if host:
+            fn = lib().moment_step_host
+
+            def run(seeds_host, rng_seed: int, counts_host):
+                params.rng_seed = rng_seed & 0xFFFFFFFFFFFFFFFF
+                st = fn(h, csr_r, seeds_host.data_ptr(), seeds_host.numel(), par_r, so_r, rows_p,
+                        counts_host.data_ptr(), sp)
+                if st:
+                    _check(st)
+        else:
+            fn = lib().moment_step
+
+            def run(seeds, rng_seed: int):
+                params.rng_seed = rng_seed & 0xFFFFFFFFFFFFFFFF
+                st = fn(h, csr_r, seeds.data_ptr(), seeds.numel(), par_r, so_r, rows_p, sp)
+                if st:
+                    _check(st)
+
+        run.keep = (self, a, out, rows)  # the prepared structs, buffers and ctx live as long as the callable
+        return run
+
     def step_host(self, indptr, indices, seeds_host, fanout, rng_seed: int, out: SampleBuffers, rows, counts_host,
                   *, flags: int = 0, stream=None):
         """moment_step_host: host seeds in, host counts out, all asynchronous on `stream`."""

@@ -395,6 +395,42 @@ def test_step_host_matches_device_path(orc, c1):
         assert np.array_equal(bufs.counts.cpu().numpy(), want["counts"])
 
 
+def test_bind_step_matches_oracle(orc, c1):
+    """Ctx.bind_step (the prepared moment_step / moment_step_host the bench issues): per-call seeds, rng seed and
+    host counts reach the kernels; interleaved with the unprepared calls on the same ctx."""
+    cfg, g = c1
+    n = g.n
+    table = W.feature_table(n, 128, torch.float32, device=DEV)
+    R = table.shape[1]
+    ctx = M.Ctx(n_vertices=n, max_seeds=1024, max_fanout=[10, 5], device=0, row_bytes=R, bin_owner=[0],
+                bin_ptr=[table.data_ptr()])
+    bufs = M.SampleBuffers.allocate(1024, [10, 5], n, DEV)
+    rows = torch.empty((bufs.nodes.numel(), R), dtype=torch.uint8, device=DEV)
+    s = torch.cuda.Stream()
+    run = ctx.bind_step(g.indptr, g.indices, [10, 5], bufs, rows, stream=s)
+    run_h = ctx.bind_step(g.indptr, g.indices, [10, 5], bufs, rows, stream=s, host=True)
+    batches = W.epoch_batches(W.training_set(g, min_count=4096), 1024, 0)
+    ip, ix, tab = g.indptr.cpu().numpy(), g.indices.cpu().numpy(), table.cpu().numpy()
+    for b in range(4):
+        seeds = batches[b]
+        rng = W.batch_rng_seed(9, 0, 0, b)
+        want = orc.sample(ip, ix, seeds.cpu().numpy(), [10, 5], rng)
+        nF = int(want["counts"][2])
+        if b % 2 == 0:
+            run(seeds, rng)
+            s.synchronize()
+            assert np.array_equal(bufs.counts.cpu().numpy(), want["counts"])
+        else:
+            counts_h = torch.full((5,), -1, dtype=torch.int64).pin_memory()
+            seeds_h = seeds.cpu().pin_memory()  # read by the first hop's kernel over PCIe: kept alive until the sync
+            run_h(seeds_h, rng, counts_h)
+            s.synchronize()
+            assert np.array_equal(counts_h.numpy(), want["counts"])
+        assert_same_sample(bufs.result(), want)
+        assert np.array_equal(rows[:nF].cpu().numpy(), orc.gather(tab, want["nodes"]))
+        ctx.step(g.indptr, g.indices, batches[(b + 1) % len(batches)], [10, 5], rng + 1, bufs, rows, stream=s)
+
+
 def test_c2_full_size_bench_configuration(orc):
     """C2 at BASELINE size, in bench.py's launch configuration: whole-batch sample parity + every gathered row."""
     _need_gpu()
