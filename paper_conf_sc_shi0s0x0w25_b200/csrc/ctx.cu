@@ -161,6 +161,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     if (const char* v = std::getenv("MOMENT_HOP_Q")) c->hop_nodes_per_group = std::max(1, std::atoi(v));
     if (const char* v = std::getenv("MOMENT_HOP_WARP")) c->hop_warp_segmented = std::atoi(v) != 0;
     if (const char* v = std::getenv("MOMENT_STEP_FORK")) c->step_fork = std::atoi(v) != 0;
+    c->no_graph = std::getenv("MOMENT_NO_GRAPH") != nullptr;
     if (const char* v = std::getenv("MOMENT_INIT_KERNEL")) c->init_in_hop0 = std::atoi(v) == 0;
     if (const char* v = std::getenv("MOMENT_COMPACT_GRID")) c->compact_grid_per_sm = std::max(1, std::atoi(v));
     c->sparse_scan = (a->n_vertices + 31) / 32 > kSparseScanMinWords;
@@ -465,7 +466,7 @@ moment_status run_step(moment_ctx_s* c, const moment_csr* csr, int64_t n_seeds, 
                         std::min<int64_t>((n_seeds + kSampleTile - 1) / kSampleTile, c->n_tile_edges)};
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
     MOMENT_TRY(cuda_check(cudaStreamIsCapturing(s, &cs), "moment_step"));
-    if (cs != cudaStreamCaptureStatusNone || std::getenv("MOMENT_NO_GRAPH")) {
+    if (cs != cudaStreamCaptureStatusNone || c->no_graph) {
         MOMENT_TRY(write_call(c, p->rng_seed, seeds, n_seeds, s, counts_host));
         MOMENT_TRY(launch_sample(c, csr, c->d_call, n_seeds, p, out, s));
         if (rows) MOMENT_TRY(launch_gather_any(c, out->nodes, out->counts + H, out->cap_nodes, rows, s));

@@ -111,6 +111,7 @@ struct moment_ctx_s {
     cudaStream_t cap_stream = nullptr, cap_side = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     int32_t step_fork = 1;  // MOMENT_STEP_FORK=0: gather after compact on one chain
+    bool no_graph = false;  // MOMENT_NO_GRAPH (read at creation): moment_step launches the kernels directly
     cudaGraphExec_t step_exec = nullptr;
     cudaGraph_t step_graph = nullptr;     // the captured graph (kept: call_node refers to it)
     cudaGraphNode_t call_node = nullptr;  // its set_call kernel node, re-parameterised per launch
