@@ -723,13 +723,15 @@ def main():
     barrier()
 
     def region(step_fn, first):
-        """One timed region: exactly K steps, barrier + synchronize on both sides, device time (ms)."""
+        """One timed region: exactly K steps, barrier + synchronize on both sides, device time (ms). Steps are
+        issued P at a time (step first + j on lane j mod P): step_fn(i0, k) enqueues steps i0 .. i0 + k - 1 on
+        lanes 0 .. k - 1 in one moment_step_batch call."""
         barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(main_stream)
         fork(e0)
-        for j in range(K):
-            step_fn(first + j, j % P)
+        for j0 in range(0, K, P):
+            step_fn(first + j0, min(P, K - j0))
         join()
         e1.record(main_stream)
         barrier()
@@ -755,11 +757,21 @@ def main():
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)  # per region, the slowest rank
         return tt.cpu().tolist()
 
-    runs = [st.bound(lane) for lane in range(P)]  # one ctypes call per step (Ctx.bind_step)
+    pool_seeds, pool_rng = [b[0] for b in pool], [b[1] for b in pool]
 
-    def dev_step(i, lane):
-        seeds, rng_seed = pool[i % n_pool]
-        runs[lane](seeds, rng_seed)
+    def pool_slice(i0, k):
+        a = i0 % n_pool
+        if a + k <= n_pool:
+            return pool_seeds[a:a + k], pool_rng[a:a + k]
+        idx = [(i0 + j) % n_pool for j in range(k)]
+        return [pool_seeds[i] for i in idx], [pool_rng[i] for i in idx]
+
+    # every lane's step prepared once; P steps per ctypes call (moment_step_batch)
+    batch = st.M.StepBatch([L.ctx for L in st.lanes], st.graph.indptr, st.graph.indices, st.fanout,
+                           [L.bufs for L in st.lanes], [L.rows for L in st.lanes], [L.stream for L in st.lanes])
+
+    def dev_step(i0, k):
+        batch.run(*pool_slice(i0, k))
 
     reg_ms = repeats(dev_step, args.min_time)
     ck = clocks.stop()
@@ -922,10 +934,16 @@ def main():
         st.step_host(seeds_pinned[i], pool[i][1], counts_pinned[i % K], lane=i)
     torch.cuda.synchronize()
 
-    runs_h = [st.bound(lane, host=True) for lane in range(P)]
+    batch_h = st.M.StepBatch([L.ctx for L in st.lanes], st.graph.indptr, st.graph.indices, st.fanout,
+                             [L.bufs for L in st.lanes], [L.rows for L in st.lanes], [L.stream for L in st.lanes],
+                             host=True)
+    pinned_list = [seeds_pinned[i] for i in range(n_pool)]
+    counts_list = [counts_pinned[i] for i in range(K)]
 
-    def host_step(i, lane):
-        runs_h[lane](seeds_pinned[i % n_pool], pool[i % n_pool][1], counts_pinned[i % K])
+    def host_step(i0, k):
+        idx = [(i0 + j) % n_pool for j in range(k)]
+        batch_h.run([pinned_list[i] for i in idx], [pool_rng[i] for i in idx],
+                    [counts_list[(i0 + j) % K] for j in range(k)])
 
     e2e_ms_all = repeats(host_step, args.e2e_min_time)
     e2e_ms = statistics.median(e2e_ms_all)
@@ -948,7 +966,8 @@ def main():
                        "timing": f"each timed region = exactly {K} steps per GPU (barrier + synchronize on both "
                                  f"sides, CUDA events, max over ranks); {n_regions} regions (>= {args.min_time:g} s "
                                  f"of device time, so nvidia-smi samples the clocks inside them), median reported; "
-                                 f"warm-up {args.warmup} steps on each of the {P} lanes",
+                                 f"warm-up {args.warmup} steps on each of the {P} lanes; steps issued {P} per "
+                                 f"moment_step_batch call (one per lane)",
                        "region_ms": {"median": ms, "min": min(reg_ms), "max": max(reg_ms), "n": n_regions},
                        "l2": "no flush: inputs larger than L2 (features %.2f GB, CSR %.2f GB)" % (
                            st.table.numel() / 1e9, (st.graph.indptr.numel() * 8 + st.graph.indices.numel() * 4) / 1e9),
@@ -986,7 +1005,8 @@ def main():
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_val, "unit": "seeds/s", "h2d_bytes_per_step": st.B * 8,
                     "d2h_bytes_per_step": (2 * H + 1) * 8,
-                    "api": "moment_step_host (C ABI) per step, same K-step regions, median of "
+                    "api": "moment_step_batch with host buffers (= moment_step_host per step, C ABI), same K-step "
+                           "regions, median of "
                            f"{len(e2e_ms_all)}",
                     "copies_declared": "H2D: the step's 1024 int64 seeds, read from pinned host memory over PCIe "
                                        "by the first hop's kernel (zero-copy); D2H: the step's counts (|F_0..F_H|, "

@@ -452,10 +452,10 @@ moment_status moment_ipc_close(void* dptr);
  * d_rows must then be its registered output: the step is then collective, see above). The 2H + 3
  * kernels are replayed from a CUDA graph cached in the ctx (captured on the first call of a given shape:
  * csr, n_seeds, fanout, flags, out and d_rows pointers; re-captured when any of them changes), so the host
- * cost per step is two launches. The per-batch rng_seed and seeds pointer reach the kernels through a
- * 16-byte device call block written by a one-thread kernel launched just before the graph. If `stream` is
- * being captured by the caller, the kernels are launched directly instead (capture-safe). Same outputs as
- * moment_sample + moment_gather.
+ * cost per step is one graph launch. The per-batch rng_seed and seeds pointer reach the kernels through a
+ * 24-byte device call block written by the graph's first node, a one-warp kernel whose parameters are
+ * replaced per launch. If `stream` is being captured by the caller, the kernels are launched directly
+ * instead (capture-safe). Same outputs as moment_sample + moment_gather.
  * ================================================================================================ */
 moment_status moment_step(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds, int64_t n_seeds,
                           const moment_sample_params* params, const moment_sample_out* out, void* d_rows,
@@ -473,6 +473,19 @@ moment_status moment_step(moment_ctx_t ctx, const moment_csr* csr, const int64_t
 moment_status moment_step_host(moment_ctx_t ctx, const moment_csr* csr, const int64_t* seeds_host,
                                int64_t n_seeds, const moment_sample_params* params,
                                const moment_sample_out* out, void* d_rows, int64_t* counts_host, void* stream);
+
+/* ================================================================================================
+ * Several steps in one call: the batches in flight of a pipelined loop, one per ctx. Step i is
+ * moment_step(ctxs[i], csr, seeds[i], n_seeds, params with rng_seed = rng_seeds[i], &outs[i], d_rows[i],
+ * streams[i]), or with counts_host != NULL moment_step_host(..., seeds[i] on the host, ..., counts_host[i],
+ * streams[i]). The n ctxs must be distinct (each owns its workspace and graph); params->rng_seed is
+ * ignored. Arrays are host arrays of n entries owned by the caller. Steps are validated and enqueued in
+ * order; the first failing step's status is returned and the steps before it stay enqueued.
+ * ================================================================================================ */
+moment_status moment_step_batch(int32_t n, const moment_ctx_t* ctxs, const moment_csr* csr,
+                                const int64_t* const* seeds, int64_t n_seeds, const moment_sample_params* params,
+                                const uint64_t* rng_seeds, const moment_sample_out* outs, void* const* d_rows,
+                                int64_t* const* counts_host, void* const* streams);
 
 /* ================================================================================================
  * Consumer: GraphSAGE mean aggregation over one sampled block — the sparse part of a

@@ -571,6 +571,28 @@ extern "C" moment_status moment_step(moment_ctx_t ctx, const moment_csr* csr, co
     return run_step(ctx, csr, n_seeds, params, out, d_rows, s, seeds);
 }
 
+extern "C" moment_status moment_step_batch(int32_t n, const moment_ctx_t* ctxs, const moment_csr* csr,
+                                           const int64_t* const* seeds, int64_t n_seeds,
+                                           const moment_sample_params* params, const uint64_t* rng_seeds,
+                                           const moment_sample_out* outs, void* const* d_rows,
+                                           int64_t* const* counts_host, void* const* streams) {
+    if (n < 0 || (n > 0 && (!ctxs || !seeds || !params || !rng_seeds || !outs || !streams)))
+        return fail(MOMENT_EINVAL, "moment_step_batch: null argument");
+    for (int i = 0; i < n; i++)
+        for (int j = 0; j < i; j++)
+            if (ctxs[i] == ctxs[j]) return fail(MOMENT_EINVAL, "moment_step_batch: ctxs[%d] repeats ctxs[%d]", i, j);
+    moment_sample_params p = *params;
+    for (int i = 0; i < n; i++) {
+        p.rng_seed = rng_seeds[i];
+        void* rows = d_rows ? d_rows[i] : nullptr;
+        const moment_status st =
+            counts_host ? moment_step_host(ctxs[i], csr, seeds[i], n_seeds, &p, &outs[i], rows, counts_host[i], streams[i])
+                        : moment_step(ctxs[i], csr, seeds[i], n_seeds, &p, &outs[i], rows, streams[i]);
+        if (st != MOMENT_OK) return st;
+    }
+    return MOMENT_OK;
+}
+
 extern "C" moment_status moment_sample_check(moment_ctx_t ctx, void* stream) {
     MOMENT_TRY(check_ctx(ctx, "moment_sample_check"));
     uint32_t flag = 0;

@@ -31,7 +31,7 @@ EXPORTED = [
     "moment_topology_free", "moment_maxflow", "moment_place", "moment_place_pack", "moment_place_pack_rank", "moment_plan",
     "moment_plan_info", "moment_plan_free", "moment_replicate_search", "moment_ctx_create", "moment_ctx_free", "moment_ctx_workspace_bytes", "moment_sample_bounds",
     "moment_sample", "moment_sample_check", "moment_hotness", "moment_bucket", "moment_gather", "moment_gather_group",
-    "moment_step", "moment_step_host", "moment_gather_routed", "moment_relay_pack", "moment_relay_serve",
+    "moment_step", "moment_step_host", "moment_step_batch", "moment_gather_routed", "moment_relay_pack", "moment_relay_serve",
     "moment_relay_scatter", "moment_relay_push", "moment_relay_serve_push", "moment_ipc_export", "moment_ipc_import",
     "moment_ipc_close", "moment_sage_mean", "moment_sage_mean_backward", "moment_signal_barrier",
     "moment_ctx_set_exchange", "moment_exchange_status",
@@ -142,6 +142,7 @@ def lib():
             "moment_gather_group": ([P, I32, P, P, I64, P, P], I32),
             "moment_step": ([P, P, P, I64, P, P, P, P], I32),
             "moment_step_host": ([P, P, P, I64, P, P, P, P, P], I32),
+            "moment_step_batch": ([I32, P, P, P, I64, P, P, P, P, P, P], I32),
             "moment_gather_routed": ([P, P, P, I64, P, P, P], I32),
             "moment_relay_pack": ([P, P, I64, P, P, P, P, P], I32),
             "moment_relay_serve": ([P, P, P, I64, P, P], I32),
@@ -397,6 +398,50 @@ class SampleBuffers:
             ob += F[h] + 1
             eb += E[h]
         return {"nodes": nodes, "offsets": offs, "src": srcs, "counts": counts}
+
+
+class StepBatch:
+    """moment_step_batch over a fixed set of ctxs (one per batch in flight) with their sample buffers, row
+    buffers and streams, prepared once: run(seeds, rng_seeds[, counts_host]) issues len(seeds) <= len(ctxs)
+    steps on the first ctxs in one ctypes call (host=True: moment_step_host, seeds in pinned host memory)."""
+
+    def __init__(self, ctxs, indptr, indices, fanout, outs, rows, streams, *, flags: int = 0, host: bool = False):
+        n = len(ctxs)
+        if not (n == len(outs) == len(rows) == len(streams)) or n == 0:
+            raise ValueError("StepBatch: one out, rows buffer and stream per ctx")
+        f = _np(fanout, np.int32)
+        self._csr = Csr(indptr.data_ptr(), indices.data_ptr(), indptr.numel() - 1, indices.numel())
+        self._params = SampleParams(len(f), f.ctypes.data, 0, flags)
+        self._ctxs = (P * n)(*[c.handle.value for c in ctxs])
+        self._outs = (SampleOut * n)(*[o.struct() for o in outs])
+        self._rows = (P * n)(*[_ptr(r) for r in rows])
+        self._streams = (P * n)(*[_stream(s) for s in streams])
+        self._seeds, self._rng, self._counts = (P * n)(), (U64 * n)(), (P * n)()
+        self._refs = (C.byref(self._csr), C.byref(self._params))
+        self._host, self._n = host, n
+        self._keep = (list(ctxs), list(outs), list(rows), list(streams), f, indptr, indices)
+        self._fn = lib().moment_step_batch
+
+    def run(self, seeds, rng_seeds, counts_host=None):
+        k = len(seeds)
+        if k > self._n or len(rng_seeds) != k or (self._host != (counts_host is not None)):
+            raise ValueError("StepBatch.run: at most one batch per ctx, one rng seed per batch, counts iff host")
+        sp, rs = self._seeds, self._rng
+        n_seeds = seeds[0].numel()
+        for i in range(k):
+            if seeds[i].numel() != n_seeds:
+                raise ValueError("StepBatch.run: batches of different sizes")
+            sp[i] = seeds[i].data_ptr()
+            rs[i] = rng_seeds[i] & 0xFFFFFFFFFFFFFFFF
+        ch = None
+        if counts_host is not None:
+            ch = self._counts
+            for i in range(k):
+                ch[i] = counts_host[i].data_ptr()
+        st = self._fn(k, self._ctxs, self._refs[0], sp, n_seeds, self._refs[1], rs, self._outs, self._rows, ch,
+                      self._streams)
+        if st:
+            _check(st)
 
 
 class Ctx:

@@ -431,6 +431,46 @@ def test_bind_step_matches_oracle(orc, c1):
         ctx.step(g.indptr, g.indices, batches[(b + 1) % len(batches)], [10, 5], rng + 1, bufs, rows, stream=s)
 
 
+def test_step_batch_matches_oracle(orc, c1):
+    """moment_step_batch (StepBatch): one call enqueues one step per ctx, device and host variants, fewer
+    batches than ctxs, and a repeated ctx is refused."""
+    cfg, g = c1
+    n = g.n
+    table = W.feature_table(n, 128, torch.float32, device=DEV)
+    R = table.shape[1]
+    P = 3
+    ctxs = [M.Ctx(n_vertices=n, max_seeds=1024, max_fanout=[10, 5], device=0, row_bytes=R, bin_owner=[0],
+                  bin_ptr=[table.data_ptr()]) for _ in range(P)]
+    bufs = [M.SampleBuffers.allocate(1024, [10, 5], n, DEV) for _ in range(P)]
+    rows = [torch.empty((b.nodes.numel(), R), dtype=torch.uint8, device=DEV) for b in bufs]
+    streams = [torch.cuda.Stream() for _ in range(P)]
+    sb = M.StepBatch(ctxs, g.indptr, g.indices, [10, 5], bufs, rows, streams)
+    sbh = M.StepBatch(ctxs, g.indptr, g.indices, [10, 5], bufs, rows, streams, host=True)
+    batches = W.epoch_batches(W.training_set(g, min_count=4096), 1024, 0)
+    ip, ix, tab = g.indptr.cpu().numpy(), g.indices.cpu().numpy(), table.cpu().numpy()
+    for k, host in [(3, False), (2, True), (3, True), (1, False)]:
+        seeds = [batches[(i + k) % len(batches)] for i in range(k)]
+        rngs = [W.batch_rng_seed(11, k, int(host), i) for i in range(k)]
+        if host:
+            seeds_h = [x.cpu().pin_memory() for x in seeds]
+            counts_h = [torch.full((5,), -1, dtype=torch.int64).pin_memory() for _ in range(k)]
+            sbh.run(seeds_h, rngs, counts_h)
+        else:
+            sb.run(seeds, rngs)
+        torch.cuda.synchronize()
+        for i in range(k):
+            want = orc.sample(ip, ix, seeds[i].cpu().numpy(), [10, 5], rngs[i])
+            assert_same_sample(bufs[i].result(), want)
+            if host:
+                assert np.array_equal(counts_h[i].numpy(), want["counts"])
+            nF = int(want["counts"][2])
+            assert np.array_equal(rows[i][:nF].cpu().numpy(), orc.gather(tab, want["nodes"]))
+    bad = M.StepBatch([ctxs[0], ctxs[0]], g.indptr, g.indices, [10, 5], bufs[:2], rows[:2], streams[:2])
+    with pytest.raises(M.MomentError) as e:
+        bad.run(batches[:2], [1, 2])
+    assert e.value.status == M.EINVAL
+
+
 def test_c2_full_size_bench_configuration(orc):
     """C2 at BASELINE size, in bench.py's launch configuration: whole-batch sample parity + every gathered row."""
     _need_gpu()
