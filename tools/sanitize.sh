@@ -5,7 +5,7 @@
 # Usage: bash tools/sanitize.sh [outdir]   -> one log per tool + a summary line each
 OUT=${1:-gpurun_out/sanitize}
 mkdir -p "$OUT"
-SEL="one_local_bin_with_placement or c1_full_size or handmade or empty_batch or tiered_and_bucket or group_relay or step_graph or step_host or gather_replicated or reused_ctx or replicated_hot or sage_mean_on_sampled"
+SEL="step_batch or bind_step or one_local_bin_with_placement or c1_full_size or handmade or empty_batch or tiered_and_bucket or group_relay or step_graph or step_host or gather_replicated or reused_ctx or replicated_hot or sage_mean_on_sampled"
 # initcheck shadows every byte torch allocates (slow): it runs on the hand-made graphs and an empty batch only
 for tool in memcheck racecheck synccheck initcheck; do
     sel="$SEL"
