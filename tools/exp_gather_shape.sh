@@ -1,7 +1,8 @@
 #!/bin/bash
-# gather4 launch shapes (blocks per SM x pipeline stages x store lag) in the step and alone: full step at 16 lanes
-# (tools/exp_variants.py) and the bench at K = 20 (value + the single-launch roofline), two repeats.
-S=${SHAPES:-"- MOMENT_TMA4_BLOCKS=1 MOMENT_TMA4_BLOCKS=1,MOMENT_TMA4_STAGES=6,MOMENT_TMA4_LAG=3 MOMENT_TMA4_BLOCKS=1,MOMENT_TMA4_STAGES=8,MOMENT_TMA4_LAG=4 MOMENT_TMA4_BLOCKS=1,MOMENT_TMA4_STAGES=4,MOMENT_TMA4_LAG=2 MOMENT_TMA4_STAGES=4,MOMENT_TMA4_LAG=2"}
+# gather4 launch shapes (tile rows x blocks per SM: MOMENT_TMA4_ROWS, MOMENT_TMA4_BLOCKS) in the step and alone:
+# full step at 16 lanes (tools/exp_variants.py) and the bench at K = 20 (value + the single-launch roofline), two
+# repeats. (The stage-count / store-lag rows of profiles/r02_sampler_experiments.txt came from experiment builds.)
+S=${SHAPES:-"- MOMENT_TMA4_ROWS=32,MOMENT_TMA4_BLOCKS=2 MOMENT_TMA4_ROWS=16,MOMENT_TMA4_BLOCKS=2 MOMENT_TMA4_ROWS=8,MOMENT_TMA4_BLOCKS=6"}
 python tools/exp_variants.py --config C2 --lanes 16 $S
 for r in 1 2; do for kv in $S; do
   e=""; [ "$kv" != "-" ] && e=$(echo $kv | tr ',' ' ')
