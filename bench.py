@@ -554,6 +554,27 @@ def profile_summary(name):
         return {}
 
 
+# The sampler's bound is the DRAM random-access rate, not bytes: the random 64-byte atoms a batch must touch
+# (indptr line per frontier node + distinct chunks of `indices` holding the chosen positions; tools/sampler_chunks.py,
+# mean of 8 batches) and the measured rate of random loads (tools/exp_ld_granularity.cu, ld.global.nc.L2::64B).
+SAMPLER_ATOMS = {"C2": (267750, "profiles/r02_sampler_chunks.txt"), "C3": (368168, "profiles/r02_sampler_chunks_C3.txt")}
+ATOM_RATE = 36.96e9  # random loads/s, profiles/r02_sampler_experiments.txt
+
+
+def step_floor(name, gather_bytes, peak_gbs, step_ms):
+    """A floor for the whole step with sampling and gathering sharing DRAM: the gather's algorithmic bytes at the
+    copy peak plus the sampler's random atoms at the random-access rate (null for configs without an atom count)."""
+    if name not in SAMPLER_ATOMS:
+        return None
+    atoms, src = SAMPLER_ATOMS[name]
+    g_us = gather_bytes / (peak_gbs * 1e9) * 1e6
+    s_us = atoms / ATOM_RATE * 1e6
+    return {"gather_us": g_us, "sampler_atoms": atoms, "atom_rate_G_per_s": ATOM_RATE / 1e9, "sampler_us": s_us,
+            "floor_us": g_us + s_us, "step_us": step_ms * 1e3, "frac": (g_us + s_us) / (step_ms * 1e3),
+            "how": f"gather alg bytes / copy peak + sampler random 64-byte atoms ({src}) / random-access rate; "
+                   "frac = floor / the median region's time per step"}
+
+
 def profile_traffic(name):
     """Per-launch DRAM bytes of the gather kernel from the committed ncu --set full summary, if any."""
     return profile_summary(name).get("dram_bytes_per_launch")
@@ -981,6 +1002,7 @@ def main():
                               "frac": (samp_bytes + gath_bytes) / K / (ms / K / 1000) / 1e9 / peak,
                               "how": "whole step (all 8(a) rows H1-H6): algorithmic bytes of the median region's "
                                      "batches / its device time, per GPU"},
+            "step_floor": step_floor(args.config, gath_bytes / K, peak, ms / K),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": profile_traffic(args.config), "kernel": "gather_tma4_kernel",
                          "launch_shares": profile_summary(args.config).get("launch_shares"),
