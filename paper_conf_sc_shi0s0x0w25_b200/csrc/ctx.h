@@ -137,8 +137,14 @@ inline moment_status cuda_check(cudaError_t e, const char* what) {
 inline moment_status cuda_pending(const char* what) { return cuda_check(cudaPeekAtLastError(), what); }
 
 constexpr int kSampleTile = 256;     // frontier nodes per sampler tile
-constexpr int kBitscanWordsPerThread = 4;  // one uint4 per thread (16 measured slower: 13.1 vs 7.6 us/launch)
-constexpr int kBitscanThreads = 512;  // 2048-word tiles: +1.3 % at K = 20 over 256 (1024: -2 %; tools/ab_lib.sh)
+#ifndef MOMENT_BITSCAN_WORDS
+#define MOMENT_BITSCAN_WORDS 4
+#endif
+constexpr int kBitscanWordsPerThread = MOMENT_BITSCAN_WORDS;  // one uint4 per thread (16 measured slower: 13.1 vs 7.6 us/launch)
+#ifndef MOMENT_BITSCAN_THREADS
+#define MOMENT_BITSCAN_THREADS 512
+#endif
+constexpr int kBitscanThreads = MOMENT_BITSCAN_THREADS;  // 2048-word tiles: +1.3 % at K = 20 over 256 (1024: -2 %)
 constexpr int kBitscanTileWords = kBitscanWordsPerThread * kBitscanThreads;  // 1024 words = 32768 ids
 constexpr int64_t kSparseScanMinWords = 1 << 18;  // > 8.4 M vertices: C3-C5 scan sparsely, C1/C2 densely
 constexpr int kBucketTile = 1024;    // requests per bucketing tile
