@@ -40,7 +40,6 @@ constexpr int kMaxHops = 16;
                                     // the SM's full 2048 threads: round 2, one node per group, +1.5 % per step vs 6 /
                                     // 40 registers, which measured +5-8 % over uncapped in round 1)
 #endif
-constexpr uint64_t kBaseReady = 1ull << 63;
 
 struct HopArgs {
     const int64_t* indptr;
