@@ -163,6 +163,7 @@ extern "C" moment_status moment_ctx_create(const moment_ctx_args* a, moment_ctx_
     if (const char* v = std::getenv("MOMENT_STEP_FORK")) c->step_fork = std::atoi(v) != 0;
     c->no_graph = std::getenv("MOMENT_NO_GRAPH") != nullptr;
     if (const char* v = std::getenv("MOMENT_INIT_KERNEL")) c->init_in_hop0 = std::atoi(v) == 0;
+    if (const char* v = std::getenv("MOMENT_VISITED_MEMSET")) c->visited_memset = std::atoi(v);
     if (const char* v = std::getenv("MOMENT_COMPACT_GRID")) c->compact_grid_per_sm = std::max(1, std::atoi(v));
     c->sparse_scan = (a->n_vertices + 31) / 32 > kSparseScanMinWords;
     if (const char* v = std::getenv("MOMENT_SPARSE_SCAN")) c->sparse_scan = std::atoi(v) != 0;

@@ -40,7 +40,11 @@ struct moment_ctx_s {
     // seeds/s, C3 10.5 -> 10.9 against the earlier 4 / 1 / 4 / 3): MOMENT_HOP_GRID, MOMENT_COMPACT_GRID,
     // MOMENT_HOP_Q, MOMENT_TMA4_BLOCKS (1 block per SM: +4 % more on C2 but the single-launch gather drops to
     // 0.55 of the copy peak)
-    int32_t hop_grid_per_sm = 1, compact_grid_per_sm = 2;  // launch caps (blocks per SM, grid-stride beyond)
+    int32_t hop_grid_per_sm = 1, compact_grid_per_sm = 2;
+    // the visited bitmap is cleared by a memset node after the compaction (one sequential n/8-byte write) instead
+    // of one random store per F_H member in the compaction (MOMENT_VISITED_MEMSET=0): C2 step 25.1 -> 24.7 us,
+    // C3 91.9 -> 89.0 us at 16 lanes (round 2, tools/exp_variants.py)
+    int32_t visited_memset = 1;  // launch caps (blocks per SM, grid-stride beyond)
     // L2 prefetch of the next hop's indptr lines by the sampler (MOMENT_HOP_PREFETCH=0/1; -1 = on with the dense
     // scan only: C2 36.5 -> 36.9 M seeds/s, C3 (sparse, 0.9 GB indptr) 10.85 -> 10.81, profiles/r01_hop_prefetch.txt)
     int32_t hop_prefetch = -1;

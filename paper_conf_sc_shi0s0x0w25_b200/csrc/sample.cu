@@ -841,6 +841,7 @@ __global__ void __launch_bounds__(kSampleTile, MOMENT_COMPACT_MINB) compact_kern
             reinterpret_cast<volatile int64_t*>(a.call[2])[threadIdx.x] = *reinterpret_cast<volatile int64_t*>(a.counts + threadIdx.x);
         }
     }
+    if (!a.visited) return;  // cleared by a memset after the kernel instead (MOMENT_VISITED_MEMSET)
     const int64_t FH = a.counts[a.H];
     for (int64_t i = (int64_t)blockIdx.x * kSampleTile + threadIdx.x; i < FH; i += (int64_t)gridDim.x * kSampleTile)
         a.visited[a.nodes[i] >> 5] = 0u;
@@ -1040,7 +1041,7 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
     ca.counts = out->counts;
     ca.nodes = out->nodes;
     ca.lidx = ctx->lidx;
-    ca.visited = ctx->visited;
+    ca.visited = ctx->visited_memset ? nullptr : ctx->visited;
     ca.rel = ctx->sparse_scan ? nullptr : ctx->rel;
     ca.rel_stride = ctx->rel_stride;
     ca.srel = ctx->srel;
@@ -1052,6 +1053,9 @@ moment_status launch_sample(moment_ctx_s* ctx, const moment_csr* csr, const uint
     const int grid = (int)std::max<int64_t>(
         1, std::min<int64_t>(std::max(ca.tb[H], (F_bound + 1023) / 1024), (int64_t)device_sms() * ctx->compact_grid_per_sm));
     compact_kernel<<<grid, kSampleTile, 0, stream>>>(ca);
+    if (ctx->visited_memset)
+        MOMENT_TRY(cuda_check(cudaMemsetAsync(ctx->visited, 0, (size_t)ctx->n_words * sizeof(uint32_t), stream),
+                              "moment_sample: visited reset"));
     return cuda_check(cudaGetLastError(), "moment_sample: launch");
 }
 
