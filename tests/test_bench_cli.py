@@ -154,3 +154,17 @@ def test_bench_tiered_two_ranks_shared_gpu():
     q = t["quota"]
     assert len(q) == 4 and q[2][0] > 0 and q[2][1] == 0 and q[3][0] == 0 and q[3][1] > 0
     assert r["host_direct_pcie"] > 0 and r["host_relayed_to_me"] > 0 and r["host_served_for_peers"] > 0
+
+
+def test_step_floor_arithmetic():
+    """bench.step_floor: the gather's bytes at the copy peak plus the sampler's random atoms at the measured
+    random-access rate (C2: 97.6 MB at 6536 GB/s = 14.93 us, 267 750 atoms at 36.96 G/s = 7.24 us)."""
+    sys.path.insert(0, ROOT)
+    import bench
+
+    f = bench.step_floor("C2", 97.6e6, 6536.0, 0.0246)
+    assert abs(f["gather_us"] - 97.6e6 / 6536e9 * 1e6) < 1e-9
+    assert abs(f["sampler_us"] - 267750 / 36.96e9 * 1e6) < 1e-9
+    assert abs(f["floor_us"] - (f["gather_us"] + f["sampler_us"])) < 1e-9
+    assert abs(f["frac"] - f["floor_us"] / 24.6) < 1e-9 and 0.8 < f["frac"] < 1.0
+    assert bench.step_floor("C1", 1e6, 6536.0, 0.01) is None
