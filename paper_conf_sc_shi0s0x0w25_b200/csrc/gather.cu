@@ -251,7 +251,7 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
 #pragma unroll
     for (int s = 0; s < kStages; s++) {
         const int64_t r = (t0 + s * dt) * kRows + lane;
-        pid[s] = r < max_n ? __ldg(ids + r) : -1;
+        pid[s] = (lane < kRows && r < max_n) ? __ldg(ids + r) : -1;  // lanes past the tile's rows load nothing
     }
     const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
     // kPlacement (one local bin behind a placement map, e.g. a DDAK layout on one GPU): the row coordinate is
@@ -261,7 +261,7 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
 #pragma unroll
     for (int s = 0; s < kStages; s++)
         pre[s] = !kPlacement ? (int32_t)pid[s]
-                 : ((t0 + s * dt) * kRows + lane < n ? (int32_t)(dev::ld_rand(placement + pid[s]) & kSlotMask) : -1);
+                 : (lane < kRows && (t0 + s * dt) * kRows + lane < n ? (int32_t)(dev::ld_rand(placement + pid[s]) & kSlotMask) : -1);
     const int64_t n_tiles = (n + kRows - 1) / kRows;
     if (lane == 0)
         for (int s = 0; s < kStages; s++) mbar_init(&full[s], 1);
@@ -269,7 +269,7 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
     __syncwarp();
     auto load_id = [&](int64_t tile) -> int32_t {
         const int64_t r = tile * kRows + lane;
-        if (!(tile < n_tiles && r < n)) return -1;
+        if (!(lane < kRows && tile < n_tiles && r < n)) return -1;
         const int64_t id = __ldg(ids + r);
         return kPlacement ? (int32_t)(dev::ld_rand(placement + id) & kSlotMask) : (int32_t)id;
     };
@@ -580,7 +580,10 @@ moment_status launch_gather(moment_ctx_s* ctx, const int64_t* ids, const int64_t
     if (tma4) {
         if (ctx->tma_base != ctx->bin_ptr[0]) MOMENT_TRY(encode_table_map(ctx));
         const uint32_t G = (uint32_t)((4 * ctx->row_bytes + 127) & ~int64_t(127));
-        const int stages = 4, bps = ctx->tma4_blocks_per_sm, rows_t = ctx->tma4_rows <= 8 ? 8 : ctx->tma4_rows <= 16 ? 16 : 32;
+        // launch shape (ctx.h): 16-row tiles x 3 blocks/SM for both instantiations (behind a placement map, C3 DDAK:
+        // 32 x 2 streams a lone launch at 0.62 instead of 0.57 but the bench runs 1.5 % slower)
+        const int stages = 4, bps = ctx->tma4_blocks_per_sm;
+        const int rows_t = ctx->tma4_rows <= 8 ? 8 : ctx->tma4_rows <= 16 ? 16 : 32;
         const size_t smem = (size_t)stages * (rows_t / 4) * G;
         const int64_t tiles = (max_n + rows_t - 1) / rows_t;
         const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, (int64_t)device_sms() * bps));
