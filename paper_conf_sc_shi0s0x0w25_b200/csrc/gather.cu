@@ -251,7 +251,10 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
 #pragma unroll
     for (int s = 0; s < kStages; s++) {
         const int64_t r = (t0 + s * dt) * kRows + lane;
-        pid[s] = (lane < kRows && r < max_n) ? __ldg(ids + r) : -1;  // lanes past the tile's rows load nothing
+        // lanes past the tile's rows: their loads (the next tile's ids) act as a prefetch in the replicated
+        // instantiation (single launch 0.70 -> 0.71 with them); behind a placement map they would add a random
+        // lookup per row, so there they load nothing
+        pid[s] = ((!kPlacement || lane < kRows) && r < max_n) ? __ldg(ids + r) : -1;
     }
     const int64_t n = n_dev ? min(*n_dev, max_n) : max_n;
     // kPlacement (one local bin behind a placement map, e.g. a DDAK layout on one GPU): the row coordinate is
@@ -269,7 +272,7 @@ __global__ void __launch_bounds__(32) gather_tma4_kernel(const __grid_constant__
     __syncwarp();
     auto load_id = [&](int64_t tile) -> int32_t {
         const int64_t r = tile * kRows + lane;
-        if (!(lane < kRows && tile < n_tiles && r < n)) return -1;
+        if (!((!kPlacement || lane < kRows) && tile < n_tiles && r < n)) return -1;
         const int64_t id = __ldg(ids + r);
         return kPlacement ? (int32_t)(dev::ld_rand(placement + id) & kSlotMask) : (int32_t)id;
     };
