@@ -29,6 +29,15 @@ def test_library_exports_every_declared_symbol():
     assert L.moment_version() >= 1
 
 
+def test_step_batch_argument_checks_on_host():
+    """moment_step_batch validates its arrays on the host before touching CUDA: n = 0 is a no-op, null arrays
+    with n > 0 are EINVAL (runs without a GPU)."""
+    L = M.lib()
+    assert L.moment_step_batch(0, None, None, None, 0, None, None, None, None, None, None) == M.OK
+    st = L.moment_step_batch(2, None, None, None, 1024, None, None, None, None, None, None)
+    assert st == M.EINVAL and b"null" in L.moment_last_error()
+
+
 def flow_certificate(n, links, s, t, value, flow):
     bal = [0] * n
     for (u, v, c), f in zip(links, flow):
