@@ -897,8 +897,13 @@ void launch_sample_warp_q(const HopArgs& a, int64_t max_F, cudaStream_t stream, 
         <<<(int)std::min<int64_t>(blocks, (int64_t)device_sms() * a.grid_per_sm), 256, 0, stream>>>(a, in);
 }
 
+#ifndef MOMENT_HOP_BIG_F
+// frontier bound from which a lane group takes big_q nodes per step: C2's and C3's hops 1 and 2 (bounds 16 k and
+// 180 k); round 2: lowered from 65536 (hop 2 only), C2 step 24.65 -> 23.95 us, C3 89.0 -> 86.9 us at 16 lanes
+#define MOMENT_HOP_BIG_F 8192
+#endif
 void launch_sample_warp(const HopArgs& a, int64_t max_F, int big_q, cudaStream_t stream) {
-    if (max_F < 65536 || big_q <= 1) launch_sample_warp_q<1>(a, max_F, stream);
+    if (max_F < MOMENT_HOP_BIG_F || big_q <= 1) launch_sample_warp_q<1>(a, max_F, stream);
     else if (big_q <= 2) launch_sample_warp_q<2>(a, max_F, stream);
     else launch_sample_warp_q<4>(a, max_F, stream);
 }
